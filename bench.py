@@ -1,0 +1,406 @@
+#!/usr/bin/env python
+"""bench.py -- kNN-DTW throughput of the SMiLer Search Step on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--dtype f32|i16]
+                    [--impl ours|reference]
+
+A step = one smiler_knn call over one batch of master queries (every row of
+SURVEY §8(a): query prep, window-level postings, group-level LB scan, tau,
+filter, DTW verification, top-k).  Default workload = BASELINE.json configs[1]
+(C2: one sensor of 2^20 points, 256 master queries per step, ELV
+{16,32,64,128}, band 10%, k=32, w=8).  Multi-GPU (torchrun): every rank takes
+its own batch of master queries over its own copy of the index (independent
+units, weak scaling, no data-path collective) -- or, with --config C4, owns a
+window range and the per-rank top-k lists are merged by one NCCL all-gather +
+smiler_merge_topk.
+
+Rank 0 prints one JSON line (see the keys below).  `--impl reference` times
+the oracle (the plain CPU brute force, the only "reference" this paper-only
+tier has) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "kNN-DTW queries/s and DTW cells/s at 1/2/4/8 B200; LB-scan HBM GB/s vs peak"
+UNIT = "master_queries/s"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def load_alu_peaks():
+    p = os.path.join(ROOT, "profiles", "alu_peaks.json")
+    if os.path.exists(p):
+        return json.load(open(p))
+    return None
+
+
+# ---------------------------------------------------------------------------
+# clocks sampler (nvidia-smi during the timed region)
+# ---------------------------------------------------------------------------
+class Clocks:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+        self.t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + self.FIELDS,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+# workloads
+# ---------------------------------------------------------------------------
+def rank_workload(cfg: str, dtype: str, rank: int, world: int, mq_per_step: int):
+    """The MQ batch of this rank.  Series identical on every rank (same seeds);
+    master queries at distinct tail offsets per rank."""
+    if cfg == "C2":
+        wl = synth.make_workload("C2", dtype, mq_per_sensor=mq_per_step * world)
+        sl = slice(rank * mq_per_step, (rank + 1) * mq_per_step)
+        wl.queries = np.ascontiguousarray(wl.queries[sl])
+        wl.query_sensor = np.ascontiguousarray(wl.query_sensor[sl])
+        return wl
+    if cfg in ("C3", "C5"):
+        # sensors round-robin over ranks; every MQ runs where its sensor lives
+        _, ns, N, periods, lens, k, w, band, mqs = synth.CONFIGS[cfg]
+        mine = list(range(rank, ns, world))
+        parts, qs, qsens, offs = [], [], [], [0]
+        D = lens[-1]
+        for li, s in enumerate(mine):
+            z = synth.sensor_series(synth.CONFIGS[cfg][0], s, N, D + 7 * mqs + 1, periods[s % len(periods)])
+            x = synth.quantise(z, dtype)
+            parts.append(x[:N])
+            offs.append(offs[-1] + N)
+            for j in range(mqs):
+                qs.append(x[N + 7 * j:N + 7 * j + D])
+                qsens.append(li)
+        return synth.Workload(cfg, dtype, np.concatenate(parts), np.asarray(offs, np.int64),
+                              np.ascontiguousarray(np.stack(qs)), np.asarray(qsens, np.int32), lens, k, w, band)
+    raise ValueError(cfg)
+
+
+def cells_per_mq(wl):
+    from paper_conf_sigmod_zhout15_b200 import smiler as _s  # noqa: F401
+    tot = 0
+    rhos = wl.rhos()
+    for j in range(wl.n_mq):
+        n = wl.offsets[wl.query_sensor[j] + 1] - wl.offsets[wl.query_sensor[j]]
+        for d, r in zip(wl.lengths, rhos):
+            r = min(r, d - 1)
+            tot += (n - d + 1) * (d * (2 * r + 1) - r * (r + 1))
+    return tot / wl.n_mq
+
+
+# ---------------------------------------------------------------------------
+# oracle (CPU) baseline
+# ---------------------------------------------------------------------------
+def oracle_sample(wl, target_s: float):
+    """Time the oracle, as it stands, on a bounded sample of the workload: one
+    master query, all its item queries, candidates t in [0, T).  Returns
+    (master queries/s extrapolated to the full candidate range, cores, sample text)."""
+    import oracle
+    oracle.build()
+    cores = os.cpu_count() or 1
+    s = int(wl.query_sensor[0])
+    series = wl.sensor_slice(s)
+    n = len(series)
+    rhos = wl.rhos()
+    T = min(n, 2000)
+    dt = oracle.time_knn(series, wl.queries[0], wl.lengths, rhos, wl.k, T, cores)
+    if dt < target_s / 4 and T < n:
+        T = int(min(n, T * max(1.0, target_s / max(dt, 1e-3))))
+        dt = oracle.time_knn(series, wl.queries[0], wl.lengths, rhos, wl.k, T, cores)
+    frac = T / (n - wl.lengths[0] + 1)
+    mqps = frac / dt
+    return mqps, cores, dt, ("1 master query (all %d item queries) of %s, candidates t in [0, %d) of %d "
+                             "(%.2f%%), %.1f s wall; MQ/s extrapolated linearly to the full candidate range"
+                             % (len(wl.lengths), wl.name, T, n, 100 * frac, dt))
+
+
+# ---------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2", choices=["C2", "C3", "C5"])
+    ap.add_argument("--dtype", default="f32", choices=["f32", "i16"])
+    ap.add_argument("--mq", type=int, default=256, help="master queries per step per GPU (C2)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--oracle-seconds", type=float, default=12.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    cfg_name = {"C2": "C2: one sensor, 2^20 points, ELV {16,32,64,128}, band 10%, k=32, w=8",
+                "C3": "C3: 1024 sensors x 100k, ELV {32,64,96}, rho=8, k=64, w=16, sharded by sensor",
+                "C5": "C5: 1024 sensors x 100k, 10 streams/sensor, ELV {16,32,64,128}, band 20%, k=128"}[args.config]
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        wl = rank_workload(args.config, args.dtype, 0, 1, min(args.mq, 4))
+        vals = []
+        for _ in range(max(args.warmup, 0)):
+            pass  # the oracle has nothing to warm up
+        total = 0.0
+        for _ in range(args.steps):
+            v, cores, dt, sample = oracle_sample(wl, max(1.0, args.oracle_seconds / max(args.steps, 1)))
+            vals.append(v)
+            total += dt
+        v = statistics.median(vals)
+        print(json.dumps({"metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+                          "warmup": args.warmup, "ms_per_step": 1000.0 * total / args.steps,
+                          "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                          "dtype": "int64" if args.dtype == "i16" else "f64", "data": "synthetic",
+                          "impl": "reference",
+                          "config": {"workload": cfg_name, "parallelism": "host cores"},
+                          "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                                           "sample": sample},
+                          "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
+        return
+
+    import torch
+    import torch.distributed as dist
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    from paper_conf_sigmod_zhout15_b200 import build as _build
+    _build.build()
+    import paper_conf_sigmod_zhout15_b200 as pkg
+
+    wl = rank_workload(args.config, args.dtype, rank, world, args.mq)
+    stream = torch.cuda.Stream(device=dev)
+    n_len, k = len(wl.lengths), wl.k
+    idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band, device=local, stream=stream)
+    qd = torch.from_numpy(wl.queries).to(dev)
+    qs = torch.from_numpy(wl.query_sensor).to(dev)
+    ids = torch.empty((wl.n_mq, n_len, k), dtype=torch.int64, device=dev)
+    dd = torch.empty((wl.n_mq, n_len, k), dtype=torch.int32 if args.dtype == "i16" else torch.float32, device=dev)
+    st = pkg.KnnStats()
+    op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0)
+
+    def step(stats=None):
+        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, stats, op if stats is not None else None)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+
+    # ---- timed region: device-resident inputs/outputs -------------------------
+    phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_verify",
+                              "ns_select", "ns_total")}
+    acc = {"survivors": 0, "candidates": 0, "dtw_cells": 0.0, "bf_cells": 0.0, "posting_bytes": 0,
+           "lb_bytes": 0, "kernel_launches": 0, "mq_chunks": 0, "tau_verified": 0, "finalists": 0}
+    gpu_idx = local
+    cvd = os.environ.get("CUDA_VISIBLE_DEVICES")
+    if cvd:
+        try:
+            gpu_idx = int(cvd.split(",")[local])
+        except ValueError:
+            pass
+    clocks = Clocks(gpu_idx)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    clocks.start()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        step(st)
+        for f in phase:
+            phase[f] += getattr(st, f)
+        for f in acc:
+            acc[f] += getattr(st, f)
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    ck = clocks.stop()
+    if world > 1:
+        dist.barrier()
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    value = world * wl.n_mq * args.steps / (ms_max / 1000.0)
+
+    # ---- e2e: the same public call with pinned host buffers ------------------
+    e2e = None
+    if not args.no_e2e:
+        qh = torch.from_numpy(wl.queries).pin_memory()
+        ih = torch.empty((wl.n_mq, n_len, k), dtype=torch.int64).pin_memory()
+        dh = torch.empty((wl.n_mq, n_len, k), dtype=dd.dtype).pin_memory()
+        qsh = torch.from_numpy(wl.query_sensor)
+        pkg.smiler_knn(idx.handle, qh, qsh, wl.lengths, k, ih, dh)
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.steps):
+            pkg.smiler_knn(idx.handle, qh, qsh, wl.lengths, k, ih, dh)
+        f1.record(stream)
+        torch.cuda.synchronize(dev)
+        ems = f0.elapsed_time(f1)
+        te = torch.tensor([ems], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        ems = float(te.item())
+        e2e = {"value": world * wl.n_mq * args.steps / (ems / 1000.0), "unit": UNIT,
+               "h2d_bytes_per_step": int(qh.numel() * qh.element_size() + qsh.numel() * 4 + n_len * 4),
+               "d2h_bytes_per_step": int(ih.numel() * 8 + dh.numel() * 4),
+               "ms_per_step": ems / args.steps}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # ---- roofline of the dominant kernel --------------------------------------
+    peaks, peak_kind = load_peaks()
+    alu = load_alu_peaks()
+    steps = args.steps
+    chunks = max(1, acc["mq_chunks"])
+    ph_ms = {k_[3:]: v_ / 1e6 / steps for k_, v_ in phase.items()}
+    n_mq = wl.n_mq
+    lb_write = acc["lb_bytes"] / 2 / steps
+    scan_bytes = acc["posting_bytes"] / steps + lb_write           # a4 reads postings, writes LB_w
+    scan_s = phase["ns_group_scan"] / 1e9 / steps
+    scan_gbs = scan_bytes / scan_s / 1e9 if scan_s > 0 else 0.0
+    win_s = phase["ns_window_lb"] / 1e9 / steps
+    n_sw = wl.D - wl.window + 1
+    win_terms = n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window * wl.window
+                           for s in wl.query_sensor.tolist()) / 1.0
+    ver_s = phase["ns_verify"] / 1e9 / steps
+    tau_s = phase["ns_tau"] / 1e9 / steps
+    cells_s = acc["dtw_cells"] / steps / (ver_s + tau_s) if ver_s + tau_s > 0 else 0.0
+    sm_mhz = ck.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
+    kernels = {
+        "group_scan_a4": {"bound": "hbm", "achieved": scan_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                          "frac": scan_gbs / peaks["hbm_gbs"], "ms": scan_s * 1e3,
+                          "bytes_per_launch": scan_bytes / chunks},
+    }
+    if alu:
+        term_peak = alu["lbterm_per_clk_sm"] * alu["sms"] * sm_mhz * 1e6
+        cell_peak = alu["dtw_cell_f32_per_clk_sm" if args.dtype == "f32" else "dtw_cell_i32_per_clk_sm"] * \
+            alu["sms"] * sm_mhz * 1e6
+    else:
+        term_peak = 148 * 16 * sm_mhz * 1e6
+        cell_peak = 148 * 42.7 * sm_mhz * 1e6
+    win_rate = win_terms / win_s if win_s > 0 else 0.0
+    kernels["window_lb_a3"] = {"bound": "alu", "achieved": win_rate / 1e12, "peak": term_peak / 1e12,
+                               "unit": "T (SW,DW,j) term-pairs/s", "frac": win_rate / term_peak, "ms": win_s * 1e3}
+    kernels["dtw_verify_a7"] = {"bound": "alu", "achieved": cells_s / 1e12, "peak": cell_peak / 1e12,
+                                "unit": "T DTW cells/s", "frac": cells_s / cell_peak, "ms": (ver_s + tau_s) * 1e3}
+    dom = max(("group_scan_a4", scan_s), ("window_lb_a3", win_s), ("dtw_verify_a7", ver_s + tau_s),
+              key=lambda x: x[1])[0]
+    rf = dict(kernels[dom])
+    rf["kernel"] = dom
+    rf["traffic"] = None
+    rf["peak_source"] = ("MEASURED_PEAKS.json hbm_gbs (%s)" % peak_kind if rf["bound"] == "hbm"
+                         else ("profiles/alu_peaks.json x median SM clock" if alu else
+                               "guide unit counts x median SM clock (no alu_peaks.json)"))
+
+    cpu = None
+    if world == 1 and not args.no_cpu:
+        v, cores, dt, sample = oracle_sample(wl, args.oracle_seconds)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": args.dtype if args.dtype == "f32" else "i16->int32",
+        "data": "synthetic",
+        "config": {"workload": cfg_name, "master_queries_per_step_per_gpu": wl.n_mq, "item_queries": wl.lengths,
+                   "k": k, "window": wl.window, "band": wl.band, "series_points": int(len(wl.series)),
+                   "parallelism": "dp%d (independent MQ batches)" % world,
+                   "l2": "inputs larger than L2 (posting lists %.0f MB per MQ)" % (8 * n_sw * (len(wl.series) // wl.window) / 1e6)},
+        "item_queries_per_s": value * n_len,
+        "dtw_cells_per_s": acc["dtw_cells"] / steps / (ms_max / 1000.0 / steps) * world,
+        "bf_equiv_cells_per_s": acc["bf_cells"] / steps / (ms_max / 1000.0 / steps) * world,
+        "survivor_frac": acc["survivors"] / max(1, acc["candidates"]),
+        "lb_scan_gbs": scan_gbs, "lb_scan_frac_of_hbm": scan_gbs / peaks["hbm_gbs"],
+        "phase_ms_per_step": ph_ms,
+        "roofline": rf, "kernels": kernels,
+        "gpu_launches": int(acc["kernel_launches"]),
+        "clocks": ck,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+    }
+    print(json.dumps(out))
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

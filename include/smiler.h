@@ -1,0 +1,204 @@
+/*
+ * smiler.h -- C ABI of the B200-native Suffix kNN Search under banded DTW
+ * (SMiLer Search Step; Zhou & Tung, SIGMOD'15).  Citations "P:<line>" refer
+ * to /root/reference/PAPER.md; "R<n>" to the readings listed in DESIGN.md.
+ *
+ * Conventions for every call:
+ *   - Return value is an smiler_status (0 = OK).  No exception, abort or
+ *     exit ever crosses the ABI; smiler_last_error() returns a thread-local
+ *     message describing the last non-OK status of the calling thread.
+ *   - Pointer arguments may be HOST or DEVICE memory (device memory must be
+ *     on the handle's device); the library inspects each pointer with
+ *     cudaPointerGetAttributes.  The caller owns every input and output
+ *     buffer; the library never retains a caller pointer after a call returns.
+ *   - The library owns all device state of a handle until smiler_free.
+ *   - One handle lives on one device and one CUDA stream.  Calls on one handle
+ *     must not run concurrently; separate handles are independent.
+ *   - Calls are stream-ordered on the handle's stream.  When any output is a
+ *     host buffer (or stats are requested) the call synchronises the stream
+ *     before returning; with device outputs and stats == NULL it returns
+ *     without a host synchronisation.
+ *   - All work runs in this library's CUDA kernels for sm_100a.  There is no
+ *     CPU fallback: without a usable CUDA device every call returns
+ *     SMILER_ECUDA.
+ */
+#ifndef SMILER_H
+#define SMILER_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SMILER_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define SMILER_API __attribute__((visibility("default")))
+#else
+#define SMILER_API
+#endif
+
+typedef struct smiler_index smiler_index; /* opaque, owned by the library */
+
+typedef enum {
+    SMILER_I16 = 0, /* int16 values with |x| <= 1023; DTW exact in int32 (R17)  */
+    SMILER_F32 = 1  /* float32 values; DTW cell = fmaf(q-c, q-c, min3)  (R16)  */
+} smiler_dtype;
+
+typedef enum {
+    SMILER_OK = 0,
+    SMILER_EINVAL = -1, /* bad argument (message says which)                 */
+    SMILER_ERANGE = -2, /* an I16 value outside [-1023, 1023]                */
+    SMILER_ENOMEM = -3, /* device allocation failed                          */
+    SMILER_ECUDA = -4,  /* CUDA runtime / launch error, or no CUDA device    */
+    SMILER_ENCCL = -5   /* reserved for collective errors (merge driver)     */
+} smiler_status;
+
+/* Per-call counters and per-phase device times (CUDA events on the handle's
+ * stream).  Times are filled only when smiler_knn_opts.timing != 0. */
+typedef struct smiler_knn_stats {
+    int64_t candidates;   /* sum over (MQ, item query) of candidate starts t      */
+    int64_t tau_verified; /* DTWs computed to set the thresholds tau_i (a5)       */
+    int64_t survivors;    /* candidates with LB_w <= tau_i, verified by DTW (a7)  */
+    int64_t finalists;    /* verified candidates with key <= tau key (a8 input)   */
+    double dtw_cells;     /* banded-DTW cells evaluated (a5 + a7)                 */
+    double bf_cells;      /* cells a brute-force scan of every candidate needs    */
+    int64_t posting_bytes;/* window-level posting bytes written by a3, read by a4 */
+    int64_t lb_bytes;     /* LB_w bytes written by a4 and read by a6              */
+    int32_t kernel_launches;
+    int32_t mq_chunks;
+    double ns_prep, ns_window_lb, ns_group_scan, ns_tau, ns_filter, ns_verify, ns_select;
+    double ns_total;
+} smiler_knn_stats;
+
+typedef struct smiler_knn_opts {
+    int32_t no_prune; /* 1: skip thresholding, verify every candidate (GPU brute force) */
+    int32_t timing;   /* 1: record per-phase CUDA events into stats                     */
+    int32_t mq_chunk; /* master queries per internal chunk; 0 = automatic               */
+    int32_t reserved[5];
+} smiler_knn_opts;
+
+/*
+ * smiler_index_build -- upload sensor series and build the index (a1).
+ *
+ * series        n_total values of `dtype`; n_sensors series concatenated.
+ *               Each series is the indexed history C of one sensor (P:597-608,
+ *               z-normalised by the caller).
+ * sensor_offsets n_sensors+1 ascending offsets into `series` (first 0, last
+ *               n_total); NULL means one sensor of length n_total.
+ * window        omega >= 1, the disjoint/sliding window length.
+ * band          Sakoe-Chiba warping width: band >= 1 means an
+ *               absolute rho = (int)band for every item query; 0 < band < 1
+ *               means rho_i = floor(band * d_i) (R4).  band == 0 means rho = 0.
+ *               Envelopes E(C) (Def. B.1, Eq. 25, clipped per
+ *               sensor, R3) are built here for an absolute band, lazily on the
+ *               first query for a fractional band (width rho_max, R4).
+ * device        CUDA device ordinal; cuda_stream a cudaStream_t (NULL = legacy
+ *               default stream) used by every call on the handle.
+ * out           receives the handle.
+ * Errors: EINVAL (n_total < 1, bad offsets, window < 1, band < 0),
+ *         ERANGE (I16 value with |x| > 1023), ENOMEM, ECUDA.
+ */
+SMILER_API int smiler_index_build(const void *series, smiler_dtype dtype, int64_t n_total,
+                       const int64_t *sensor_offsets, int32_t n_sensors, int32_t window,
+                       float band, int32_t device, void *cuda_stream, smiler_index **out);
+
+/*
+ * smiler_index_build_shard -- one sensor, window-range shard for multi-GPU
+ * (SURVEY §8(e)).  `slice` holds global points [slice_begin, slice_begin +
+ * n_slice) of a series of n_global points; the handle owns candidate starts
+ * t in [t_begin, t_end) (global).  slice_begin must be a multiple of window
+ * (disjoint windows stay global, so every LB_w equals the unsharded value);
+ * the slice must carry a halo: slice_begin <= max(0, t_begin - rho_max) and
+ * slice_begin + n_slice >= min(n_global, t_end + D - 1 + rho_max) for every
+ * later query (checked by smiler_knn, EINVAL otherwise).  Returned ids are
+ * global t.
+ */
+SMILER_API int smiler_index_build_shard(const void *slice, smiler_dtype dtype, int64_t n_slice,
+                             int64_t slice_begin, int64_t n_global, int64_t t_begin,
+                             int64_t t_end, int32_t window, float band, int32_t device,
+                             void *cuda_stream, smiler_index **out);
+
+/*
+ * smiler_knn -- Suffix kNN Search (Def. 4.1) for a batch of master
+ * queries, through the two-level index (Sec. 4.3): window-level
+ * posting lists (a3), group-level LB_w scan (a4, Thm 4.3 / Eq. 5), per-query
+ * threshold tau_i (a5, R8), filtering (a6), banded-DTW verification (a7,
+ * Eq. 21-24) and top-k selection (a8).
+ *
+ * queries       [n_mq][D] master queries, oldest -> newest, same
+ *               dtype as the index; D = lengths[n_len-1].
+ * query_sensor  [n_mq] sensor searched by each MQ; NULL -> 0.
+ * lengths       ELV [n_len], strictly increasing, lengths[0] >= 1, each <= the
+ *               sensor's length, lengths[n_len-1] = D <= 1024, n_len <= 16.
+ *               Item query IQ_i = the last lengths[i] points of the MQ
+ *               (P:859-860).
+ * k             max(EKV), 1 <= k <= 1024; smaller k are prefixes.
+ * ids           [n_mq][n_len][k] int64: start t of C_{t,d_i} (R2) within the
+ *               sensor (global t for shards).
+ * dists         [n_mq][n_len][k] int32 (I16) or float (F32): DTW with
+ *               dist(a,b) = (a-b)^2 (R1).
+ *               Rows are sorted by (dist, t) (R11); padding is id -1 with
+ *               dist INT32_MAX / +inf (R12).
+ * stats         may be NULL.
+ * Results are exactly the brute-force kNN (filtering never dismisses a true
+ * neighbour: Thm 4.1/4.3 with tau_i >= the k-th distance, R8, R16).
+ * Errors: EINVAL, ENOMEM, ECUDA.
+ */
+SMILER_API int smiler_knn(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+               int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
+               void *dists, smiler_knn_stats *stats);
+
+/* smiler_knn with options (opts may be NULL = defaults). */
+SMILER_API int smiler_knn_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                  int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
+                  void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts);
+
+/*
+ * smiler_merge_topk -- final selection over G per-shard top-k lists (a9,
+ * SURVEY §8(e)); called after an all-gather of the shards' (ids, dists).
+ * ids_in [G][rows][k] int64, dists_in [G][rows][k] int32/float (dtype);
+ * writes the k smallest by (dist, id) of each row to ids_out/dists_out
+ * [rows][k], padding as smiler_knn.  Each candidate must appear in at most
+ * one shard (ownership partition), so the merge is exact.  Runs on `device`
+ * and `cuda_stream`.
+ */
+SMILER_API int smiler_merge_topk(const int64_t *ids_in, const void *dists_in, smiler_dtype dtype,
+                      int32_t G, int32_t rows, int32_t k, int64_t *ids_out, void *dists_out,
+                      int32_t device, void *cuda_stream);
+
+/* ---- Per-step entry points used by the parity tests (same kernels) ------ */
+
+/* Envelope U, L (Eq. 25, clipped, R3) of one sensor with width rho, as built
+ * by the a1 kernel.  U, L: [sensor length] of the index dtype. */
+SMILER_API int smiler_index_envelope(smiler_index *idx, int32_t sensor, int32_t rho, void *U, void *L);
+
+/* Steps a2-a4 only: for each MQ, the window-level posting lists (P_EQ, P_EC)
+ * (may be NULL) as [n_mq][D-window+1][n_dw][2] int32/float (n_dw = floor(N/w)
+ * of the MQ's sensor; all MQs must search sensors of equal length), and LB_w
+ * per candidate as [n_mq][n_len][N] int32/float indexed by t (entries with
+ * t > N - d_i are unspecified).  Envelope width rho_max as in smiler_knn. */
+SMILER_API int smiler_lower_bounds(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                        int32_t n_mq, const int32_t *lengths, int32_t n_len, void *postings,
+                        void *lbw);
+
+/* Step a7 only: banded DTW (Eq. 21-24) of item query q[0..d) against
+ * C_{t,d} of `sensor` for each t in ts[0..n_t), warping width rho.  dists:
+ * [n_t] int32/float.  Every t must satisfy 0 <= t <= N-d. */
+SMILER_API int smiler_dtw(smiler_index *idx, int32_t sensor, const void *q, int32_t d, int32_t rho,
+               const int64_t *ts, int64_t n_t, void *dists);
+
+/* Release the handle and all its device memory.  NULL-safe. */
+SMILER_API void smiler_free(smiler_index *idx);
+
+/* Thread-local message for the last non-OK status ("" if none). */
+SMILER_API const char *smiler_last_error(void);
+
+/* SMILER_ABI_VERSION of the loaded library. */
+SMILER_API int32_t smiler_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SMILER_H */

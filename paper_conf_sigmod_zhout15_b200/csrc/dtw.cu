@@ -1,0 +1,229 @@
+// dtw.cu -- step a7 (and the DTWs of a5): banded DTW verification.
+//
+// Recurrence: Eq. 21-24, dist(a,b) = (a-b)^2 (R1).
+// The paper's Alg. 2 keeps a compressed 2 x (2rho+2) matrix in
+// shared memory per thread.  Here the band lives in REGISTERS: one thread per
+// candidate, the 2rho+1 band cells of the current row are a statically indexed
+// register array updated in place, rows are the candidate's points c_j and the
+// band runs over the item query's points q_i (so q is warp-uniform and c is one
+// value per row).  Candidate points are staged 32 rows at a time through
+// shared memory as [row][lane] (conflict-free, coalesced loads); the query is
+// staged once per task in shared memory and read R rows at a time into
+// registers.  Per cell: FADD, FMNMX3, FFMA (f32) or IADD, VIMNMX3, IMAD (int).
+// No tensor cores: DTW is a min-plus recurrence, not a contraction.
+//
+// Band coordinates: row j (1..d) = candidate point c_j, slot u in [0, 2rho]
+// = query point i = j + u - rho.  Predecessors of (i, j):
+//   (i-1, j)   -> same row, slot u-1      (computed just before)
+//   (i-1, j-1) -> previous row, slot u
+//   (i, j-1)   -> previous row, slot u+1
+// Row 0 is g(0,0) = 0 at slot rho and inf elsewhere (Eq. 22); cells with
+// i < 1 or i > d are inf (Eq. 22/23).  For f32 those cells get a query value
+// of +inf, which makes every such cell +inf without a mask; for int32 the
+// first and last rho rows run a masked variant.
+#include <type_traits>
+#include <utility>
+
+#include "internal.h"
+
+namespace smiler {
+
+constexpr int kDtwThreads = 256;
+constexpr int kDtwWarps = kDtwThreads / 32;
+constexpr int kRows = 4;                       // rows per register block
+
+// Per-warp query staging length (values): d + W + kRows, rounded up to 4.
+__host__ __device__ inline int dtw_qstage(int d, int rho) { return (d + 2 * rho + 1 + kRows + 3) & ~3; }
+
+template <typename V> __device__ __forceinline__ V vmin3(V a, V b, V c);
+template <> __device__ __forceinline__ float vmin3(float a, float b, float c) {
+    return fminf(fminf(a, b), c);
+}
+template <> __device__ __forceinline__ int32_t vmin3(int32_t a, int32_t b, int32_t c) {
+    return min(min(a, b), c);
+}
+__device__ __forceinline__ float cell(float q, float c, float m) {
+    float diff = q - c;
+    return fmaf(diff, diff, m);  // R16: pinned
+}
+__device__ __forceinline__ int32_t cell(int32_t q, int32_t c, int32_t m) {
+    int32_t diff = q - c;
+    return diff * diff + m;
+}
+template <typename V> __device__ __forceinline__ uint32_t vbits(V v);
+template <> __device__ __forceinline__ uint32_t vbits(float v) { return __float_as_uint(v); }
+template <> __device__ __forceinline__ uint32_t vbits(int32_t v) { return (uint32_t)v; }
+
+// One DP row (row index j, 1-based) over the band; qrow[u] = q_{j+u-rho}.
+template <typename V, int RHO, bool MASK>
+__device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V cj, int j, int d,
+                                       const V INF) {
+    constexpr int W = 2 * RHO + 1;
+    V left = INF;
+#pragma unroll
+    for (int u = 0; u < W; u++) {
+        V up = (u + 1 < W) ? band[u + 1] : INF;
+        V m = vmin3<V>(left, band[u], up);
+        V nv = cell(qrow[u], cj, m);
+        if (MASK) {
+            int i = j + u - RHO;
+            nv = (i >= 1 && i <= d) ? nv : INF;
+        }
+        band[u] = nv;
+        left = nv;
+    }
+}
+
+template <typename S, int RHO>
+__global__ void __launch_bounds__(kDtwThreads) dtw_kernel(const DtwParams<S> p) {
+    using V = typename Tr<S>::V;
+    constexpr int W = 2 * RHO + 1;
+    constexpr bool IS_F = std::is_same<S, float>::value;
+    const V INF = Tr<S>::inf();
+    extern __shared__ __align__(16) unsigned char dtw_smem[];
+    const int lane = threadIdx.x & 31;
+    const int wib = threadIdx.x >> 5;
+    const int qs = dtw_qstage(p.d, RHO);
+    V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (qs + 32 * 33);
+    V (*s_c)[33] = reinterpret_cast<V (*)[33]>(sq + qs);
+    const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nw = (gridDim.x * blockDim.x) >> 5;
+    const int total = p.task_off[p.n_mq];
+    const int d = p.d;
+    int cur_mq = -1;
+
+    for (int task = gw; task < total; task += nw) {
+        // segment lookup: largest mq with task_off[mq] <= task
+        int lo = 0, hi = p.n_mq;
+        while (hi - lo > 1) {
+            int mid = (lo + hi) >> 1;
+            if (p.task_off[mid] <= task) lo = mid; else hi = mid;
+        }
+        const int mq = lo;
+        const int chunk = task - p.task_off[mq];
+        const MQMeta m = p.meta[mq];
+        const int seg = mq * p.n_len + p.li;
+        int cnt;
+        int64_t lbase;
+        if (p.mode == 0) {
+            cnt = p.LT;
+            lbase = (int64_t)seg * p.LT;
+        } else {
+            cnt = p.counts[seg];
+            lbase = m.seg_off + (int64_t)p.li * m.n;
+        }
+        const int idx = chunk * 32 + lane;
+        const int t = idx < cnt ? p.list[lbase + idx] : -1;
+
+        if (mq != cur_mq) {  // stage IQ_li of this MQ: sq[x] = q_{x-rho+1}
+            __syncwarp();
+            const V *q = p.qv + (int64_t)mq * p.D + (p.D - d);
+            for (int x = lane; x < d + W + kRows; x += 32) {
+                int i = x - RHO + 1;
+                V v = IS_F ? INF : (V)0;
+                if (i >= 1 && i <= d) v = q[i - 1];
+                sq[x] = v;
+            }
+            cur_mq = mq;
+            __syncwarp();
+        }
+
+        V band[W];
+#pragma unroll
+        for (int u = 0; u < W; u++) band[u] = (u == RHO) ? (V)0 : INF;
+
+        const S *cs = p.series + m.series_off;
+        for (int j0 = 0; j0 < d; j0 += 32) {
+            __syncwarp();
+            const bool in_row = (j0 + lane) < d;
+#pragma unroll 4
+            for (int l = 0; l < 32; l++) {
+                int tl = __shfl_sync(0xffffffffu, t, l);
+                V v = (V)0;
+                if (tl >= 0 && in_row) v = (V)cs[tl + j0 + lane];
+                s_c[lane][l] = v;
+            }
+            __syncwarp();
+            const int jn = min(32, d - j0);
+            int r = 0;
+            for (; r + kRows <= jn; r += kRows) {
+                const int j = j0 + r + 1;
+                V qr[W + kRows - 1];
+#pragma unroll
+                for (int x = 0; x < W + kRows - 1; x++) qr[x] = sq[j - 1 + x];
+                const bool fast = IS_F || (j - RHO >= 1 && j + kRows - 1 + RHO <= d);
+                if (fast) {
+#pragma unroll
+                    for (int rr = 0; rr < kRows; rr++)
+                        dp_row<V, RHO, false>(band, qr + rr, s_c[r + rr][lane], j + rr, d, INF);
+                } else {
+#pragma unroll
+                    for (int rr = 0; rr < kRows; rr++)
+                        dp_row<V, RHO, true>(band, qr + rr, s_c[r + rr][lane], j + rr, d, INF);
+                }
+            }
+            for (; r < jn; r++) {
+                const int j = j0 + r + 1;
+                V qr[W];
+#pragma unroll
+                for (int x = 0; x < W; x++) qr[x] = sq[j - 1 + x];
+                dp_row<V, RHO, !IS_F>(band, qr, s_c[r][lane], j, d, INF);
+            }
+        }
+        const V dist = band[RHO];
+        const uint64_t key = t >= 0 ? (((uint64_t)vbits<V>(dist) << 32) | (uint32_t)t) : kKeyMax;
+        if (p.mode == 0) {
+            if (idx < cnt) p.keys_out[lbase + idx] = key;
+        } else {
+            const bool fin = t >= 0 && key <= p.tau_key[seg];
+            const unsigned bal = __ballot_sync(0xffffffffu, fin);
+            if (bal) {
+                int base = 0;
+                if (lane == 0) base = atomicAdd(&p.fin_count[seg], __popc(bal));
+                base = __shfl_sync(0xffffffffu, base, 0);
+                if (fin) p.fin[m.seg_off + (int64_t)p.li * m.n + base + __popc(bal & ((1u << lane) - 1))] = key;
+            }
+        }
+    }
+}
+
+template <typename S, int RHO>
+static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
+    using V = typename Tr<S>::V;
+    size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + 32 * 33) * sizeof(V);
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(dtw_kernel<S, RHO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + 32 * 33) * sizeof(V)));
+        attr = true;
+    }
+    static int occ = 0, sms = 0;
+    if (!occ) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &occ, dtw_kernel<S, RHO>, kDtwThreads,
+            (size_t)kDtwWarps * (dtw_qstage(256, RHO) + 32 * 33) * sizeof(V));
+        if (occ < 1) occ = 1;
+    }
+    if (grid <= 0) grid = sms * occ;
+    dtw_kernel<S, RHO><<<grid, kDtwThreads, smem, st>>>(p);
+}
+
+template <typename S, int... Rs>
+static bool dispatch(int rho, const DtwParams<S> &p, int grid, cudaStream_t st,
+                     std::integer_sequence<int, Rs...>) {
+    bool done = false;
+    ((rho == Rs ? (launch_one<S, Rs>(p, grid, st), done = true) : false), ...);
+    return done;
+}
+
+template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st) {
+    dispatch<S>(rho, p, grid, st, std::make_integer_sequence<int, kMaxRhoFast + 1>{});
+}
+
+template void launch_dtw<int16_t>(int, const DtwParams<int16_t> &, int, cudaStream_t);
+template void launch_dtw<float>(int, const DtwParams<float> &, int, cudaStream_t);
+
+}  // namespace smiler

@@ -1,0 +1,79 @@
+// internal.h -- device-side data structures shared by the kernels of
+// libsmiler.so (not part of the C ABI; see include/smiler.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/smiler.h"
+
+namespace smiler {
+
+constexpr int kMaxLen = 16;      // max item queries per master query
+constexpr int kMaxD = 1024;      // max master-query length
+constexpr int kMaxK = 1024;      // max k
+constexpr int kMaxWindow = 64;   // max omega
+constexpr int kMaxRhoFast = 32;  // rho handled by the register-band DTW kernels
+constexpr int kSortCap = 4096;   // keys sorted in shared memory by one CTA
+constexpr uint64_t kKeyMax = ~0ull;
+
+// Value type of the arithmetic for a storage type (R16, R17).
+template <typename S> struct Tr;
+template <> struct Tr<int16_t> {
+    using V = int32_t;
+    using V2 = int2;
+    using V4 = int4;
+    static __device__ __forceinline__ V inf() { return 0x3FFFFFFF; }
+};
+template <> struct Tr<float> {
+    using V = float;
+    using V2 = float2;
+    using V4 = float4;
+    static __device__ __forceinline__ V inf() { return __int_as_float(0x7f800000); }
+};
+
+// Per master query (chunk-relative), built on the host.
+struct MQMeta {
+    int64_t series_off;  // element offset of the sensor's series in the device copy
+    int64_t n;           // sensor (slice) length N
+    int64_t origin;      // global id of local t = 0
+    int64_t t_lo, t_hi;  // owned candidate starts, local coordinates
+    int64_t n_dw;        // floor(N / w) disjoint windows
+    int64_t post_off;    // offset (in pairs) of this MQ's posting lists
+    int64_t seg_off;     // offset of this MQ's per-candidate segments; (mq,i) at seg_off + i*n
+    int32_t nblk;        // group-scan CTAs for this MQ
+    int32_t sensor;
+};
+
+// Parameters common to one smiler_knn chunk.
+struct QParams {
+    int D, w, n_len, k, rho_env, E, LT, n_mq;
+    int len[kMaxLen];
+    int rho[kMaxLen];
+};
+
+// Work list of one DTW launch (one item-query index `li`, all MQs of a chunk).
+template <typename S> struct DtwParams {
+    const S *series;
+    const MQMeta *meta;
+    const typename Tr<S>::V *qv;  // [n_mq][D] master queries in the arithmetic type
+    int D, n_len, li, d, n_mq;
+    int mode;                     // 0 = tau list -> keys_out; 1 = survivors -> finalists
+    const int32_t *list;          // candidate t values
+    int LT;                       // tau mode: list stride per segment
+    const int32_t *counts;        // survivors mode: per-segment counts
+    const int32_t *task_off;      // [n_mq + 1] prefix of warp tasks
+    uint64_t *keys_out;           // tau mode
+    const uint64_t *tau_key;      // survivors mode: per-segment key threshold
+    uint64_t *fin;                // survivors mode: finalist keys (segment layout)
+    int32_t *fin_count;
+};
+
+template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st);
+
+// DTW cells of one banded d x d matrix (|i-j| <= rho).
+inline int64_t dtw_cells(int d, int rho) {
+    if (rho > d - 1) rho = d - 1;
+    return (int64_t)d * (2 * rho + 1) - (int64_t)rho * (rho + 1);
+}
+
+}  // namespace smiler

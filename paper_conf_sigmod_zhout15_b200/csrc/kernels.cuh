@@ -1,0 +1,640 @@
+// kernels.cuh -- steps a1-a6, a8, a9 of the Search Step.
+// Included once, by smiler.cu.  DTW (a5/a7) is in dtw.cu.
+#pragma once
+#include <stdint.h>
+
+#include <type_traits>
+
+#include "internal.h"
+
+namespace smiler {
+
+// ---------------------------------------------------------------------------
+// Small device helpers
+// ---------------------------------------------------------------------------
+template <typename V> __device__ __forceinline__ uint32_t key_bits(V v);
+template <> __device__ __forceinline__ uint32_t key_bits(float v) { return __float_as_uint(v); }
+template <> __device__ __forceinline__ uint32_t key_bits(int32_t v) { return (uint32_t)v; }
+
+// e(v; U, L) of Eq. 26 accumulated: (v - clamp(v, L, U))^2.
+__device__ __forceinline__ void lb_term(float v, float U, float L, float &acc) {
+    float dd = v - fminf(fmaxf(v, L), U);
+    acc = fmaf(dd, dd, acc);
+}
+__device__ __forceinline__ void lb_term(int32_t v, int32_t U, int32_t L, int32_t &acc) {
+    int32_t dd = v - min(max(v, L), U);
+    acc += dd * dd;
+}
+__device__ __forceinline__ float vmax(float a, float b) { return fmaxf(a, b); }
+__device__ __forceinline__ int32_t vmax(int32_t a, int32_t b) { return max(a, b); }
+
+__device__ __forceinline__ uint64_t warp_min_u64(uint64_t v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        uint64_t x = __shfl_xor_sync(0xffffffffu, v, o);
+        v = x < v ? x : v;
+    }
+    return v;
+}
+
+// Block-wide min of a uint64 (blockDim.x multiple of 32, <= 1024).
+__device__ __forceinline__ uint64_t block_min_u64(uint64_t v, uint64_t *s_red) {
+    v = warp_min_u64(v);
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    __syncthreads();
+    if (lane == 0) s_red[wid] = v;
+    __syncthreads();
+    if (wid == 0) {
+        uint64_t x = lane < nw ? s_red[lane] : kKeyMax;
+        x = warp_min_u64(x);
+        if (lane == 0) s_red[0] = x;
+    }
+    __syncthreads();
+    return s_red[0];
+}
+
+// Exclusive block scan of int (returns exclusive prefix; *total gets the sum).
+__device__ __forceinline__ int block_excl_scan(int v, int *s_scan, int *total) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    __syncthreads();
+    if (lane == 31) s_scan[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+        int w = lane < nw ? s_scan[lane] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            int y = __shfl_up_sync(0xffffffffu, w, o);
+            if (lane >= o) w += y;
+        }
+        if (lane < nw) s_scan[lane] = w;  // inclusive warp totals
+    }
+    __syncthreads();
+    const int before = wid > 0 ? s_scan[wid - 1] : 0;
+    *total = s_scan[nw - 1];
+    return before + x - v;
+}
+
+// Bitonic sort of n (power of two) uint64 keys in shared memory, ascending.
+__device__ void bitonic_sort_smem(uint64_t *s, int n) {
+    for (int size = 2; size <= n; size <<= 1) {
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            __syncthreads();
+            for (int i = threadIdx.x; i < (n >> 1); i += blockDim.x) {
+                int lo = 2 * i - (i & (stride - 1));
+                int hi = lo + stride;
+                bool asc = ((lo & size) == 0);
+                uint64_t a = s[lo], b = s[hi];
+                if ((a > b) == asc) {
+                    s[lo] = b;
+                    s[hi] = a;
+                }
+            }
+        }
+    }
+    __syncthreads();
+}
+
+// k-th smallest (1-based) of keys[0..n) (global memory), keys unique except
+// kKeyMax padding; returns kKeyMax if fewer than k keys are < kKeyMax.
+// MSB radix select, 8 bits per pass, one CTA.  s_hist: 256 ints.
+__device__ uint64_t block_radix_kth(const uint64_t *keys, int64_t n, int k, int *s_hist,
+                                    uint64_t *s_bcast) {
+    uint64_t prefix = 0, mask = 0;
+    int krem = k;
+    for (int shift = 56; shift >= 0; shift -= 8) {
+        for (int i = threadIdx.x; i < 256; i += blockDim.x) s_hist[i] = 0;
+        __syncthreads();
+        for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
+            uint64_t x = keys[i];
+            if (x != kKeyMax && (x & mask) == prefix) atomicAdd(&s_hist[(x >> shift) & 255], 1);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int acc = 0, dsel = -1;
+            for (int dg = 0; dg < 256; dg++) {
+                if (acc + s_hist[dg] >= krem) {
+                    dsel = dg;
+                    break;
+                }
+                acc += s_hist[dg];
+            }
+            if (dsel < 0) {
+                s_bcast[0] = kKeyMax;  // fewer than k keys
+            } else {
+                s_bcast[0] = prefix | ((uint64_t)dsel << shift);
+                s_bcast[1] = (uint64_t)(krem - acc);
+            }
+        }
+        __syncthreads();
+        if (s_bcast[0] == kKeyMax) return kKeyMax;
+        prefix = s_bcast[0];
+        krem = (int)s_bcast[1];
+        mask |= (uint64_t)255 << shift;
+        __syncthreads();
+    }
+    return prefix;
+}
+
+// ---------------------------------------------------------------------------
+// a1: envelope E(C) = (U, L), Def. B.1 / Eq. 25, clipped to the
+// sensor (R3).  grid (tiles, sensors); each CTA stages tile + 2 rho halo of
+// one sensor in shared memory.
+// ---------------------------------------------------------------------------
+constexpr int kEnvTile = 2048;
+
+template <typename S>
+__global__ void __launch_bounds__(256) envelope_kernel(const S *series, const int64_t *soff,
+                                                      const int64_t *slen, int rho, S *U, S *L) {
+    extern __shared__ __align__(16) unsigned char env_smem[];
+    S *tile = reinterpret_cast<S *>(env_smem);
+    const int s = blockIdx.y;
+    const int64_t n = slen[s];
+    const int64_t x0 = (int64_t)blockIdx.x * kEnvTile;
+    if (x0 >= n) return;
+    const S *c = series + soff[s];
+    const int span = kEnvTile + 2 * rho;
+    for (int i = threadIdx.x; i < span; i += blockDim.x) {
+        int64_t x = x0 - rho + i;
+        tile[i] = (x >= 0 && x < n) ? c[x] : (S)0;
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < kEnvTile; i += blockDim.x) {
+        int64_t x = x0 + i;
+        if (x >= n) break;
+        int64_t lo = x - rho < 0 ? 0 : x - rho;
+        int64_t hi = x + rho > n - 1 ? n - 1 : x + rho;
+        S mx = tile[lo - (x0 - rho)], mn = mx;
+        for (int64_t y = lo + 1; y <= hi; y++) {
+            S v = tile[y - (x0 - rho)];
+            mx = v > mx ? v : mx;
+            mn = v < mn ? v : mn;
+        }
+        U[soff[s] + x] = mx;
+        L[soff[s] + x] = mn;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a2: query prep.  One CTA per MQ: MQ values in the arithmetic type (qv) and
+// the table {q, U(Q), L(Q), 0} with the MQ envelope of width rho_env clipped
+// to the MQ (R3, R4, R20).
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D, int rho,
+                                                        typename Tr<S>::V *qv,
+                                                        typename Tr<S>::V4 *qtab) {
+    using V = typename Tr<S>::V;
+    using V4 = typename Tr<S>::V4;
+    __shared__ V s[kMaxD];
+    const int mq = blockIdx.x;
+    for (int p = threadIdx.x; p < D; p += blockDim.x) {
+        V v = (V)queries[(int64_t)mq * D + p];
+        s[p] = v;
+        qv[(int64_t)mq * D + p] = v;
+    }
+    __syncthreads();
+    for (int p = threadIdx.x; p < D; p += blockDim.x) {
+        int lo = p - rho < 0 ? 0 : p - rho;
+        int hi = p + rho > D - 1 ? D - 1 : p + rho;
+        V mx = s[lo], mn = s[lo];
+        for (int y = lo + 1; y <= hi; y++) {
+            mx = s[y] > mx ? s[y] : mx;
+            mn = s[y] < mn ? s[y] : mn;
+        }
+        V4 e;
+        e.x = s[p];
+        e.y = mx;
+        e.z = mn;
+        e.w = (V)0;
+        qtab[(int64_t)mq * D + p] = e;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3: window-level index (Sec. 4.3.1; Fig. 4-5).  For every sliding
+// window SW_b = MQ[D-w-b .. D-b) (R19) and disjoint window DW_r = c[rw..rw+w):
+//   P_EQ[b][r] = sum_j e(c[rw+j]; U(Q), L(Q) at D-w-b+j)    (LB_keogh(E(SW), DW))
+//   P_EC[b][r] = sum_j e(MQ[D-w-b+j]; U(C), L(C) at rw+j)   (LB_keogh(E(DW), SW))
+// One thread per DW r holds its w points and envelope in registers; the MQ
+// table sits in shared memory and is read as warp-uniform 16-byte broadcasts.
+// Output layout post[mq][b][r] = {P_EQ, P_EC}: coalesced over r.
+// ALU-bound: 8 ALU ops per (b, r, j) (clamp = 2 MNMX, sub, FMA/IMAD, twice).
+// WT = w at compile time (0 = runtime w, reading the DW from global memory).
+// ---------------------------------------------------------------------------
+template <typename S, int WT>
+__global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
+                                                       const MQMeta *meta,
+                                                       const typename Tr<S>::V4 *qtab, int D,
+                                                       int w, typename Tr<S>::V2 *post) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    using V4 = typename Tr<S>::V4;
+    extern __shared__ __align__(16) unsigned char wl_smem[];
+    V4 *sq = reinterpret_cast<V4 *>(wl_smem);
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int64_t)blockIdx.x * blockDim.x >= m.n_dw) return;
+    for (int p = threadIdx.x; p < D; p += blockDim.x) sq[p] = qtab[(int64_t)mq * D + p];
+    __syncthreads();
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= m.n_dw) return;
+    const int n_sw = D - w + 1;
+    V2 *out = post + m.post_off + r;
+    const int64_t base = m.series_off + r * w;
+    if constexpr (WT > 0) {
+        V c[WT], U[WT], L[WT];
+#pragma unroll
+        for (int j = 0; j < WT; j++) {
+            c[j] = (V)series[base + j];
+            U[j] = (V)UC[base + j];
+            L[j] = (V)LC[base + j];
+        }
+        for (int b = 0; b < n_sw; b++) {
+            const V4 *qq = sq + (D - WT - b);
+            V eq = (V)0, ec = (V)0;
+#pragma unroll
+            for (int j = 0; j < WT; j++) {
+                const V4 Q = qq[j];
+                lb_term(c[j], Q.y, Q.z, eq);
+                lb_term(Q.x, U[j], L[j], ec);
+            }
+            V2 o;
+            o.x = eq;
+            o.y = ec;
+            out[(int64_t)b * m.n_dw] = o;
+        }
+    } else {
+        for (int b = 0; b < n_sw; b++) {
+            const V4 *qq = sq + (D - w - b);
+            V eq = (V)0, ec = (V)0;
+            for (int j = 0; j < w; j++) {
+                const V4 Q = qq[j];
+                lb_term((V)series[base + j], Q.y, Q.z, eq);
+                lb_term(Q.x, (V)UC[base + j], (V)LC[base + j], ec);
+            }
+            V2 o;
+            o.x = eq;
+            o.y = ec;
+            out[(int64_t)b * m.n_dw] = o;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a4: group-level index scan ("LB scan"), Sec. 4.3.2 / Alg. 1 (P:1373-1419,
+// P:4061-4090) with the garbles fixed as reading R5, and Remark 2:
+// every posting element is read once and its running sums serve all item
+// queries.  Thread <-> rightmost disjoint window r (r = -1 .. n_dw-1), CTA <->
+// RT consecutive r.  For each CSG_b (b < w):
+//   S_EQ, S_EC += post[b + j w][r - j]              (j = 0, 1, ...)
+//   m = j + 1; for every IQ_i with m_i(b) = floor((d_i - b)/w) = m:
+//     LB_w(IQ_i, C_t) = max(S_EQ, S_EC),  t = (r - j) w - (d_i - b) % w  (Eq. 4/5)
+// The right end e = t + d_i = (r+1) w + b is the same for every IQ, so the CTA
+// buffers LB_w in shared memory at slot (r - R0) w + b (padded to w+1) and
+// writes each IQ's contiguous t range coalesced.  Slots never written (no full
+// DW, m = 0) hold LB_w = 0 (R6).  The CTA also emits, per IQ, the E candidates
+// with the smallest (LB_w, t) of its tile: the tau set of step a5.
+// Reads all posting lists once (HBM-bound); writes LB_w [mq][i][t].
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void group_scan_kernel(const typename Tr<S>::V2 *post, const MQMeta *meta,
+                                  const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    extern __shared__ __align__(16) unsigned char gs_smem[];
+    __shared__ uint64_t s_red[32];
+    const int RT = blockDim.x;
+    const int w = P.w, nl = P.n_len;
+    const int stride = RT * (w + 1);
+    V *tile = reinterpret_cast<V *>(gs_smem);
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) return;
+    for (int x = threadIdx.x; x < nl * stride; x += RT) tile[x] = (V)0;
+    __syncthreads();
+    const int64_t R0 = (int64_t)blockIdx.x * RT - 1;
+    const int64_t r = R0 + threadIdx.x;
+    const int n_sw = P.D - w + 1;
+    if (r >= 0 && r < m.n_dw) {
+        const V2 *pp = post + m.post_off;
+        for (int b = 0; b < w && b < n_sw; b++) {
+            const int jmax = (n_sw - 1 - b) / w + 1;
+            int ii = 0;
+            while (ii < nl && P.len[ii] - b < w) ii++;  // IQs with m_i(b) = 0 keep LB_w = 0
+            V se = (V)0, sc = (V)0;
+            const int jlim = (int)min((int64_t)jmax, r + 1);
+#pragma unroll 4
+            for (int j = 0; j < jlim; j++) {
+                if (ii >= nl) break;
+                const V2 pv = pp[(int64_t)(b + j * w) * m.n_dw + (r - j)];
+                se += pv.x;
+                sc += pv.y;
+                while (ii < nl && (P.len[ii] - b) / w == j + 1) {
+                    tile[ii * stride + threadIdx.x * (w + 1) + b] = vmax(se, sc);
+                    ii++;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    // write LB_w of the tile, per IQ, coalesced over t
+    const int64_t e0 = (R0 + 1) * w;
+    for (int i = 0; i < nl; i++) {
+        const int d = P.len[i];
+        const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
+        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        V *out = lb + m.seg_off + (int64_t)i * m.n;
+        for (int s = threadIdx.x; s < RT * w; s += RT) {
+            const int64_t t = e0 + s - d;
+            if (t >= tmin && t < tend) out[t] = tile[i * stride + (s / w) * (w + 1) + (s % w)];
+        }
+    }
+    // tau set: E smallest (LB_w, t) of the tile per IQ
+    if (P.E > 0) {
+        for (int i = 0; i < nl; i++) {
+            const int d = P.len[i];
+            const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
+            const int64_t tend = min(m.t_hi, m.n - d + 1);
+            V *row = tile + i * stride + threadIdx.x * (w + 1);
+            int32_t *dst = tauc + (int64_t)(mq * nl + i) * P.LT + (int64_t)blockIdx.x * P.E;
+            for (int e = 0; e < P.E; e++) {
+                uint64_t best = kKeyMax;
+                int bb = -1;
+                for (int b = 0; b < w; b++) {
+                    const int64_t t = e0 + (int64_t)threadIdx.x * w + b - d;
+                    const uint32_t kb = key_bits(row[b]);
+                    if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
+                        uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
+                        if (key < best) {
+                            best = key;
+                            bb = b;
+                        }
+                    }
+                }
+                const uint64_t win = block_min_u64(best, s_red);
+                if (win != kKeyMax && best == win) {
+                    // mark taken (bits 0xFFFFFFFF are neither a valid int32 >= 0 nor a float >= 0)
+                    if constexpr (sizeof(V) == 4) {
+                        uint32_t allones = 0xFFFFFFFFu;
+                        row[bb] = *reinterpret_cast<V *>(&allones);
+                    }
+                }
+                if (threadIdx.x == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+                __syncthreads();
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a5 (second half): tau_i = k-th smallest (DTW, t) key of the verified tau set
+// (an upper bound on the k-th NN distance: k candidates lie at or below it;
+// reading R8).  One CTA per segment (mq, i).  thr = the LB_w admission bound:
+// int: dist; f32: dist * (1 + 2^-10) rounded up (R16 rounding slack).
+// no candidates enough -> key max / thr = +inf (no pruning).
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, int LT, int k,
+                                                        uint64_t *tau_key, uint32_t *thr) {
+    using V = typename Tr<S>::V;
+    __shared__ int s_hist[256];
+    __shared__ uint64_t s_b[2];
+    const int seg = blockIdx.x;
+    const uint64_t kth = block_radix_kth(tauk + (int64_t)seg * LT, LT, k, s_hist, s_b);
+    if (threadIdx.x == 0) {
+        tau_key[seg] = kth;
+        if (kth == kKeyMax) {
+            thr[seg] = sizeof(V) == 4 && std::is_same<V, float>::value ? 0x7f800000u : 0x7FFFFFFFu;
+        } else {
+            uint32_t db = (uint32_t)(kth >> 32);
+            if constexpr (std::is_same<V, float>::value) {
+                float tf = __uint_as_float(db);
+                thr[seg] = __float_as_uint(__fmul_ru(tf, 1.0f + 1.0f / 1024.0f));
+            } else {
+                thr[seg] = db;
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a6: filtering: keep t with LB_w(t) <= thr_i (ties survive).
+// Two-phase filter-then-verify keeps warps homogeneous.
+// grid (tiles, segments); block-aggregated compaction, one atomic per CTA.
+// ---------------------------------------------------------------------------
+constexpr int kFiltThreads = 256;
+constexpr int kFiltItems = 8;
+
+template <typename S>
+__global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<S>::V *lb,
+                                                             const MQMeta *meta, const QParams P,
+                                                             const uint32_t *thr, int32_t *surv,
+                                                             int32_t *surv_count) {
+    using V = typename Tr<S>::V;
+    __shared__ int s_scan[32];
+    __shared__ int s_base;
+    const int seg = blockIdx.y;
+    const int mq = seg / P.n_len, i = seg % P.n_len;
+    const MQMeta m = meta[mq];
+    const int d = P.len[i];
+    const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t te = min(m.t_hi, m.n - d + 1);
+    const int64_t t0 = tb + (int64_t)blockIdx.x * kFiltThreads * kFiltItems;
+    if (t0 >= te) return;
+    const uint32_t th = thr[seg];
+    const V *src = lb + m.seg_off + (int64_t)i * m.n;
+    uint32_t flags = 0;
+#pragma unroll
+    for (int it = 0; it < kFiltItems; it++) {
+        const int64_t t = t0 + (int64_t)it * kFiltThreads + threadIdx.x;
+        if (t < te) {
+            bool keep;
+            if constexpr (std::is_same<V, float>::value)
+                keep = src[t] <= __uint_as_float(th);
+            else
+                keep = src[t] <= (int32_t)th;
+            flags |= (uint32_t)keep << it;
+        }
+    }
+    int total;
+    const int pos = block_excl_scan(__popc(flags), s_scan, &total);
+    if (threadIdx.x == 0) s_base = total ? atomicAdd(&surv_count[seg], total) : 0;
+    __syncthreads();
+    int o = s_base + pos;
+    int32_t *dst = surv + m.seg_off + (int64_t)i * m.n;
+#pragma unroll
+    for (int it = 0; it < kFiltItems; it++)
+        if (flags >> it & 1) dst[o++] = (int32_t)(t0 + (int64_t)it * kFiltThreads + threadIdx.x);
+}
+
+// no-prune mode: every owned candidate of every segment is a survivor.
+__global__ void all_candidates_kernel(const MQMeta *meta, const QParams P, int32_t *surv,
+                                      int32_t *surv_count) {
+    const int seg = blockIdx.y;
+    const int mq = seg / P.n_len, i = seg % P.n_len;
+    const MQMeta m = meta[mq];
+    const int d = P.len[i];
+    const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t te = min(m.t_hi, m.n - d + 1);
+    const int64_t nc = te > tb ? te - tb : 0;
+    int32_t *dst = surv + m.seg_off + (int64_t)i * m.n;
+    for (int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < nc;
+         x += (int64_t)gridDim.x * blockDim.x)
+        dst[x] = (int32_t)(tb + x);
+    if (blockIdx.x == 0 && threadIdx.x == 0) surv_count[seg] = (int32_t)nc;
+}
+
+// Warp-task prefix for one item-query index li: task_off[mq] = sum over earlier
+// MQs of ceil(count/32).  Single CTA.
+__global__ void __launch_bounds__(1024) task_prefix_kernel(const int32_t *counts, int static_count,
+                                                          int n_mq, int n_len, int li,
+                                                          int32_t *task_off) {
+    __shared__ int s_scan[32];
+    __shared__ int s_carry;
+    if (threadIdx.x == 0) s_carry = 0;
+    __syncthreads();
+    for (int base = 0; base < n_mq; base += blockDim.x) {
+        const int mq = base + threadIdx.x;
+        int c = 0;
+        if (mq < n_mq) c = static_count >= 0 ? static_count : counts[mq * n_len + li];
+        const int tasks = (c + 31) >> 5;
+        int total;
+        const int ex = block_excl_scan(tasks, s_scan, &total);
+        if (mq < n_mq) task_off[mq] = s_carry + ex;
+        __syncthreads();
+        if (threadIdx.x == 0) s_carry += total;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) task_off[n_mq] = s_carry;
+}
+
+// ---------------------------------------------------------------------------
+// a8: selection: the k smallest (DTW, t) keys of each segment,
+// sorted ascending; all k are returned (not only the k-th).  One CTA per
+// segment.  <= kSortCap finalists: bitonic sort in shared memory; otherwise
+// radix-select the k-th key first and sort the k keys at or below it.
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void __launch_bounds__(512) topk_kernel(const uint64_t *fin, const int32_t *fin_count,
+                                                  const MQMeta *meta, const QParams P,
+                                                  int64_t *out_ids, typename Tr<S>::V *out_d) {
+    using V = typename Tr<S>::V;
+    __shared__ uint64_t s_keys[kSortCap];
+    __shared__ int s_hist[256];
+    __shared__ uint64_t s_b[2];
+    __shared__ int s_cnt;
+    const int seg = blockIdx.x;
+    const int mq = seg / P.n_len, i = seg % P.n_len;
+    const MQMeta m = meta[mq];
+    const int k = P.k;
+    const int cnt = fin_count[seg];
+    const uint64_t *src = fin + m.seg_off + (int64_t)i * m.n;
+    int nsort;
+    if (cnt <= kSortCap) {
+        nsort = 1;
+        while (nsort < cnt || nsort < k) nsort <<= 1;
+        for (int x = threadIdx.x; x < nsort; x += blockDim.x) s_keys[x] = x < cnt ? src[x] : kKeyMax;
+    } else {
+        const uint64_t kth = block_radix_kth(src, cnt, k, s_hist, s_b);
+        if (threadIdx.x == 0) s_cnt = 0;
+        nsort = 1;
+        while (nsort < k) nsort <<= 1;
+        for (int x = threadIdx.x; x < nsort; x += blockDim.x) s_keys[x] = kKeyMax;
+        __syncthreads();
+        for (int x = threadIdx.x; x < cnt; x += blockDim.x) {
+            uint64_t v = src[x];
+            if (v <= kth) {
+                int pos = atomicAdd(&s_cnt, 1);
+                if (pos < nsort) s_keys[pos] = v;
+            }
+        }
+    }
+    bitonic_sort_smem(s_keys, nsort);
+    const V INF = Tr<S>::inf();
+    for (int j = threadIdx.x; j < k; j += blockDim.x) {
+        const uint64_t key = s_keys[j];
+        const int64_t o = (int64_t)seg * k + j;
+        if (key == kKeyMax) {
+            out_ids[o] = -1;
+            if constexpr (std::is_same<V, float>::value) out_d[o] = INF;
+            else out_d[o] = (V)0x7FFFFFFF;
+        } else {
+            out_ids[o] = (int64_t)(uint32_t)key + m.origin;
+            const uint32_t db = (uint32_t)(key >> 32);
+            if constexpr (std::is_same<V, float>::value) out_d[o] = __uint_as_float(db);
+            else out_d[o] = (int32_t)db;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a9: merge of G per-shard top-k lists.  One CTA per row.
+// Key = (dist bits << 32) | id (ids < 2^32); padding (id -1) -> key max.
+// ---------------------------------------------------------------------------
+template <typename V>
+__global__ void __launch_bounds__(512) merge_topk_kernel(const int64_t *ids_in, const V *d_in,
+                                                        int G, int rows, int k, int64_t *ids_out,
+                                                        V *d_out, V pad) {
+    __shared__ uint64_t s_keys[kSortCap];
+    const int row = blockIdx.x;
+    const int n = G * k;
+    int nsort = 1;
+    while (nsort < n) nsort <<= 1;
+    for (int x = threadIdx.x; x < nsort; x += blockDim.x) {
+        uint64_t key = kKeyMax;
+        if (x < n) {
+            const int g = x / k, j = x % k;
+            const int64_t o = ((int64_t)g * rows + row) * k + j;
+            const int64_t id = ids_in[o];
+            if (id >= 0) key = ((uint64_t)key_bits(d_in[o]) << 32) | (uint32_t)id;
+        }
+        s_keys[x] = key;
+    }
+    bitonic_sort_smem(s_keys, nsort);
+    for (int j = threadIdx.x; j < k; j += blockDim.x) {
+        const uint64_t key = s_keys[j];
+        const int64_t o = (int64_t)row * k + j;
+        if (key == kKeyMax) {
+            ids_out[o] = -1;
+            d_out[o] = pad;
+        } else {
+            ids_out[o] = (int64_t)(uint32_t)key;
+            const uint32_t db = (uint32_t)(key >> 32);
+            d_out[o] = *reinterpret_cast<const V *>(&db);
+        }
+    }
+}
+
+// Stats: acc[0] += finalists, acc[1 + i] += survivors of item query i.
+__global__ void accum_counts_kernel(const int32_t *scount, const int32_t *fcount, int nseg, int n_len,
+                                    unsigned long long *acc) {
+    for (int s = threadIdx.x; s < nseg; s += blockDim.x) {
+        atomicAdd(&acc[0], (unsigned long long)fcount[s]);
+        atomicAdd(&acc[1 + s % n_len], (unsigned long long)scount[s]);
+    }
+}
+
+// int16 range check for the I16 dtype (R17): counts |x| > 1023.
+__global__ void range_check_kernel(const int16_t *x, int64_t n, int *bad) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        if (x[i] > 1023 || x[i] < -1023) atomicAdd(bad, 1);
+}
+
+// Gather DTW keys of smiler_dtw's candidate list into distances.
+template <typename V>
+__global__ void keys_to_dists_kernel(const uint64_t *keys, int64_t n, V *out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t db = (uint32_t)(keys[i] >> 32);
+        out[i] = *reinterpret_cast<const V *>(&db);
+    }
+}
+
+}  // namespace smiler

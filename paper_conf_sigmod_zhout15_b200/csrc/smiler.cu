@@ -1,0 +1,948 @@
+// smiler.cu -- host orchestration and C ABI of libsmiler.so (include/smiler.h).
+//
+// Per smiler_knn chunk of master queries, on the handle's stream and without
+// any host synchronisation inside the pipeline:
+//   a2 query_prep -> a3 window_lb -> a4 group_scan (+ tau set)
+//   -> a5 DTW(tau set) + tau_select -> a6 filter -> a7 DTW(survivors)
+//   -> a8 topk -> copy out
+// Data-dependent sizes (survivors, finalists) stay on the device; buffers are
+// sized for the worst case (every candidate) and kernels read the counts.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <map>
+#include <string>
+#include <type_traits>
+#include <vector>
+
+#include "internal.h"
+#include "kernels.cuh"
+
+using namespace smiler;
+
+// ---------------------------------------------------------------------------
+// errors
+// ---------------------------------------------------------------------------
+static thread_local std::string g_err;
+
+static int fail(int code, const char *fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CU(call)                                                                           \
+    do {                                                                                   \
+        cudaError_t e_ = (call);                                                           \
+        if (e_ != cudaSuccess) {                                                           \
+            if (e_ == cudaErrorMemoryAllocation)                                           \
+                return fail(SMILER_ENOMEM, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), \
+                            __FILE__, __LINE__);                                           \
+            return fail(SMILER_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_),     \
+                        __FILE__, __LINE__);                                               \
+        }                                                                                  \
+    } while (0)
+
+#define CHECK_LAUNCH() CU(cudaGetLastError())
+
+#define TRY(x)                      \
+    do {                            \
+        int r_ = (x);               \
+        if (r_ != SMILER_OK) return r_; \
+    } while (0)
+
+static bool is_device_ptr(const void *p) {
+    if (!p) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// ---------------------------------------------------------------------------
+// handle
+// ---------------------------------------------------------------------------
+struct DevBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+    int ensure(size_t bytes) {
+        if (bytes <= cap) return SMILER_OK;
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+        size_t want = bytes + bytes / 8 + 256;
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            return fail(SMILER_ENOMEM, "cudaMalloc(%zu): %s", want, cudaGetErrorString(e));
+        }
+        cap = want;
+        return SMILER_OK;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+    }
+    template <typename T> T *as() const { return reinterpret_cast<T *>(p); }
+};
+
+struct SensorInfo {
+    int64_t off;     // device element offset (aligned)
+    int64_t n;       // length
+    int64_t origin;  // global id of local t = 0
+    int64_t t_lo, t_hi;
+    int64_t n_global;  // shard: the full series length; else n
+    int64_t slice_begin;
+};
+
+struct smiler_index {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    smiler_dtype dtype = SMILER_I16;
+    int window = 1;
+    float band = 0.f;
+    bool shard = false;
+    std::vector<SensorInfo> sensors;
+    int64_t dev_elems = 0;
+    void *d_series = nullptr;
+    int64_t *d_soff = nullptr, *d_slen = nullptr;
+    std::map<int, std::pair<void *, void *>> env;  // rho -> (U, L)
+    int num_sms = 148;
+    // workspace
+    DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, tauk, taukey, thr, scount, fcount,
+        taskoff, out_ids, out_d, tmp;
+    std::vector<cudaEvent_t> events;
+};
+
+static size_t esize(smiler_dtype t) { return t == SMILER_I16 ? 2 : 4; }
+
+static int set_device(smiler_index *idx) {
+    CU(cudaSetDevice(idx->device));
+    return SMILER_OK;
+}
+
+static int rho_for(float band, int d) {
+    if (band >= 1.0f) return (int)band;
+    if (band <= 0.0f) return 0;
+    return (int)floorf(band * (float)d);
+}
+
+// a1: envelope of every sensor with width rho, cached per rho.
+static int ensure_envelope(smiler_index *idx, int rho, void **U, void **L) {
+    auto it = idx->env.find(rho);
+    if (it != idx->env.end()) {
+        *U = it->second.first;
+        *L = it->second.second;
+        return SMILER_OK;
+    }
+    const size_t bytes = (size_t)idx->dev_elems * esize(idx->dtype);
+    void *u = nullptr, *l = nullptr;
+    CU(cudaMalloc(&u, bytes));
+    cudaError_t e = cudaMalloc(&l, bytes);
+    if (e != cudaSuccess) {
+        cudaFree(u);
+        return fail(SMILER_ENOMEM, "envelope alloc: %s", cudaGetErrorString(e));
+    }
+    int64_t nmax = 0;
+    for (auto &s : idx->sensors) nmax = std::max(nmax, s.n);
+    dim3 grid((unsigned)((nmax + kEnvTile - 1) / kEnvTile), (unsigned)idx->sensors.size());
+    size_t smem = (size_t)(kEnvTile + 2 * rho) * esize(idx->dtype);
+    if (idx->dtype == SMILER_I16) {
+        if (smem > 48 * 1024)
+            cudaFuncSetAttribute(envelope_kernel<int16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        envelope_kernel<int16_t><<<grid, 256, smem, idx->stream>>>(
+            (const int16_t *)idx->d_series, idx->d_soff, idx->d_slen, rho, (int16_t *)u, (int16_t *)l);
+    } else {
+        if (smem > 48 * 1024)
+            cudaFuncSetAttribute(envelope_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        envelope_kernel<float><<<grid, 256, smem, idx->stream>>>(
+            (const float *)idx->d_series, idx->d_soff, idx->d_slen, rho, (float *)u, (float *)l);
+    }
+    CHECK_LAUNCH();
+    idx->env[rho] = {u, l};
+    *U = u;
+    *L = l;
+    return SMILER_OK;
+}
+
+static int upload_series(smiler_index *idx, const void *series, const int64_t *offs, int ns) {
+    const size_t es = esize(idx->dtype);
+    const int64_t align = 64;
+    int64_t total = 0;
+    std::vector<int64_t> dev_off(ns);
+    for (int s = 0; s < ns; s++) {
+        dev_off[s] = total;
+        total += (offs[s + 1] - offs[s] + align - 1) / align * align;
+    }
+    total += align;
+    idx->dev_elems = total;
+    CU(cudaMalloc(&idx->d_series, (size_t)total * es));
+    CU(cudaMemsetAsync(idx->d_series, 0, (size_t)total * es, idx->stream));
+    const bool dev = is_device_ptr(series);
+    for (int s = 0; s < ns; s++) {
+        const int64_t n = offs[s + 1] - offs[s];
+        CU(cudaMemcpyAsync((char *)idx->d_series + dev_off[s] * es,
+                           (const char *)series + offs[s] * es, (size_t)n * es,
+                           dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, idx->stream));
+        idx->sensors[s].off = dev_off[s];
+    }
+    std::vector<int64_t> so(ns), sl(ns);
+    for (int s = 0; s < ns; s++) {
+        so[s] = idx->sensors[s].off;
+        sl[s] = idx->sensors[s].n;
+    }
+    CU(cudaMalloc(&idx->d_soff, sizeof(int64_t) * ns));
+    CU(cudaMalloc(&idx->d_slen, sizeof(int64_t) * ns));
+    CU(cudaMemcpyAsync(idx->d_soff, so.data(), sizeof(int64_t) * ns, cudaMemcpyHostToDevice, idx->stream));
+    CU(cudaMemcpyAsync(idx->d_slen, sl.data(), sizeof(int64_t) * ns, cudaMemcpyHostToDevice, idx->stream));
+    if (idx->dtype == SMILER_I16) {
+        int *bad = nullptr;
+        CU(cudaMalloc(&bad, sizeof(int)));
+        CU(cudaMemsetAsync(bad, 0, sizeof(int), idx->stream));
+        range_check_kernel<<<idx->num_sms * 4, 256, 0, idx->stream>>>((const int16_t *)idx->d_series,
+                                                                      total, bad);
+        int hb = 0;
+        cudaMemcpyAsync(&hb, bad, sizeof(int), cudaMemcpyDeviceToHost, idx->stream);
+        cudaError_t e = cudaStreamSynchronize(idx->stream);
+        cudaFree(bad);
+        if (e != cudaSuccess) return fail(SMILER_ECUDA, "range check: %s", cudaGetErrorString(e));
+        if (hb) return fail(SMILER_ERANGE, "%d I16 values outside [-1023, 1023] (R17)", hb);
+    }
+    return SMILER_OK;
+}
+
+static void destroy(smiler_index *idx) {
+    if (!idx) return;
+    cudaSetDevice(idx->device);
+    if (idx->stream) cudaStreamSynchronize(idx->stream);
+    if (idx->d_series) cudaFree(idx->d_series);
+    if (idx->d_soff) cudaFree(idx->d_soff);
+    if (idx->d_slen) cudaFree(idx->d_slen);
+    for (auto &kv : idx->env) {
+        cudaFree(kv.second.first);
+        cudaFree(kv.second.second);
+    }
+    DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
+                      &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->tauk,
+                      &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
+                      &idx->out_ids, &idx->out_d,  &idx->tmp};
+    for (DevBuf *b : bufs) b->release();
+    for (auto ev : idx->events) cudaEventDestroy(ev);
+    delete idx;
+}
+
+static int common_build(smiler_index *idx, int32_t device, void *stream) {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return fail(SMILER_ECUDA, "no CUDA device available (%s); there is no CPU fallback",
+                    cudaGetErrorString(e));
+    }
+    if (device < 0 || device >= ndev) return fail(SMILER_EINVAL, "device %d out of range [0,%d)", device, ndev);
+    idx->device = device;
+    idx->stream = (cudaStream_t)stream;
+    CU(cudaSetDevice(device));
+    CU(cudaDeviceGetAttribute(&idx->num_sms, cudaDevAttrMultiProcessorCount, device));
+    return SMILER_OK;
+}
+
+extern "C" int smiler_index_build(const void *series, smiler_dtype dtype, int64_t n_total,
+                                  const int64_t *sensor_offsets, int32_t n_sensors, int32_t window,
+                                  float band, int32_t device, void *cuda_stream, smiler_index **out) {
+    if (!out) return fail(SMILER_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!series) return fail(SMILER_EINVAL, "series is NULL");
+    if (dtype != SMILER_I16 && dtype != SMILER_F32) return fail(SMILER_EINVAL, "bad dtype %d", (int)dtype);
+    if (n_total < 1) return fail(SMILER_EINVAL, "n_total must be >= 1");
+    if (window < 1 || window > kMaxWindow) return fail(SMILER_EINVAL, "window must be in [1, %d]", kMaxWindow);
+    if (!(band >= 0.f) || !isfinite(band)) return fail(SMILER_EINVAL, "band must be finite and >= 0");
+    std::vector<int64_t> offs;
+    if (sensor_offsets) {
+        if (n_sensors < 1) return fail(SMILER_EINVAL, "n_sensors must be >= 1");
+        std::vector<int64_t> h(n_sensors + 1);
+        if (is_device_ptr(sensor_offsets)) {
+            if (cudaMemcpy(h.data(), sensor_offsets, sizeof(int64_t) * (n_sensors + 1),
+                           cudaMemcpyDeviceToHost) != cudaSuccess)
+                return fail(SMILER_ECUDA, "reading sensor_offsets");
+        } else {
+            memcpy(h.data(), sensor_offsets, sizeof(int64_t) * (n_sensors + 1));
+        }
+        if (h[0] != 0 || h[n_sensors] != n_total) return fail(SMILER_EINVAL, "sensor_offsets must start at 0 and end at n_total");
+        for (int s = 0; s < n_sensors; s++)
+            if (h[s + 1] <= h[s]) return fail(SMILER_EINVAL, "sensor %d is empty or offsets not ascending", s);
+        offs = h;
+    } else {
+        n_sensors = 1;
+        offs = {0, n_total};
+    }
+    smiler_index *idx = new smiler_index();
+    int rc = common_build(idx, device, cuda_stream);
+    if (rc) {
+        delete idx;
+        return rc;
+    }
+    idx->dtype = dtype;
+    idx->window = window;
+    idx->band = band;
+    idx->sensors.resize(n_sensors);
+    for (int s = 0; s < n_sensors; s++) {
+        SensorInfo &si = idx->sensors[s];
+        si.n = offs[s + 1] - offs[s];
+        si.origin = 0;
+        si.t_lo = 0;
+        si.t_hi = si.n;
+        si.n_global = si.n;
+        si.slice_begin = 0;
+    }
+    rc = upload_series(idx, series, offs.data(), n_sensors);
+    if (rc == SMILER_OK && band >= 1.0f) {
+        void *U, *L;
+        rc = ensure_envelope(idx, rho_for(band, 1), &U, &L);
+    }
+    if (rc == SMILER_OK) {
+        cudaError_t e = cudaStreamSynchronize(idx->stream);
+        if (e != cudaSuccess) rc = fail(SMILER_ECUDA, "index build: %s", cudaGetErrorString(e));
+    }
+    if (rc) {
+        destroy(idx);
+        return rc;
+    }
+    *out = idx;
+    return SMILER_OK;
+}
+
+extern "C" int smiler_index_build_shard(const void *slice, smiler_dtype dtype, int64_t n_slice,
+                                        int64_t slice_begin, int64_t n_global, int64_t t_begin,
+                                        int64_t t_end, int32_t window, float band, int32_t device,
+                                        void *cuda_stream, smiler_index **out) {
+    if (!out) return fail(SMILER_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (window < 1 || window > kMaxWindow) return fail(SMILER_EINVAL, "window must be in [1, %d]", kMaxWindow);
+    if (n_slice < 1 || slice_begin < 0 || slice_begin + n_slice > n_global)
+        return fail(SMILER_EINVAL, "slice [%lld, +%lld) outside the series of %lld points",
+                    (long long)slice_begin, (long long)n_slice, (long long)n_global);
+    if (slice_begin % window) return fail(SMILER_EINVAL, "slice_begin must be a multiple of window");
+    if (t_begin < slice_begin || t_end < t_begin || t_end > slice_begin + n_slice)
+        return fail(SMILER_EINVAL, "owned range [%lld, %lld) not inside the slice", (long long)t_begin,
+                    (long long)t_end);
+    if (n_global - 1 > (int64_t)INT32_MAX) return fail(SMILER_EINVAL, "series longer than 2^31 points");
+    int64_t offs[2] = {0, n_slice};
+    smiler_index *idx = nullptr;
+    int rc = smiler_index_build(slice, dtype, n_slice, offs, 1, window, band, device, cuda_stream, &idx);
+    if (rc) return rc;
+    idx->shard = true;
+    SensorInfo &si = idx->sensors[0];
+    si.origin = slice_begin;
+    si.t_lo = t_begin - slice_begin;
+    si.t_hi = t_end - slice_begin;
+    si.n_global = n_global;
+    si.slice_begin = slice_begin;
+    *out = idx;
+    return SMILER_OK;
+}
+
+extern "C" void smiler_free(smiler_index *idx) { destroy(idx); }
+
+extern "C" const char *smiler_last_error(void) { return g_err.c_str(); }
+
+extern "C" int32_t smiler_abi_version(void) { return SMILER_ABI_VERSION; }
+
+// ---------------------------------------------------------------------------
+// smiler_knn
+// ---------------------------------------------------------------------------
+struct Plan {
+    int D, n_len, k, w, rho_env;
+    std::vector<int> len, rho;
+    int RT;
+};
+
+static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len, int k, Plan &pl) {
+    if (n_len < 1 || n_len > kMaxLen) return fail(SMILER_EINVAL, "n_len must be in [1, %d]", kMaxLen);
+    if (k < 1 || k > kMaxK) return fail(SMILER_EINVAL, "k must be in [1, %d]", kMaxK);
+    pl.len.assign(lengths_h, lengths_h + n_len);
+    for (int i = 0; i < n_len; i++) {
+        if (pl.len[i] < 1) return fail(SMILER_EINVAL, "lengths[%d] < 1", i);
+        if (i && pl.len[i] <= pl.len[i - 1]) return fail(SMILER_EINVAL, "lengths must be strictly increasing");
+    }
+    pl.D = pl.len[n_len - 1];
+    if (pl.D > kMaxD) return fail(SMILER_EINVAL, "D = %d exceeds %d", pl.D, kMaxD);
+    pl.w = idx->window;
+    if (pl.w > pl.D) return fail(SMILER_EINVAL, "window %d longer than D = %d", pl.w, pl.D);
+    pl.n_len = n_len;
+    pl.k = k;
+    pl.rho.resize(n_len);
+    pl.rho_env = 0;
+    for (int i = 0; i < n_len; i++) {
+        int r = rho_for(idx->band, pl.len[i]);
+        pl.rho_env = std::max(pl.rho_env, r);  // R4: envelopes use rho_max
+        pl.rho[i] = std::min(r, pl.len[i] - 1);  // rho >= d-1 is unconstrained DTW
+        if (pl.rho[i] > kMaxRhoFast)
+            return fail(SMILER_EINVAL, "warping width %d for d=%d exceeds the supported %d", r, pl.len[i],
+                        kMaxRhoFast);
+    }
+    const size_t vs = 4;
+    pl.RT = 128;
+    while (pl.RT > 32 && (size_t)n_len * pl.RT * (pl.w + 1) * vs > 96 * 1024) pl.RT >>= 1;
+    return SMILER_OK;
+}
+
+template <typename S>
+static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int mode,
+                        const int32_t *list, int LT, const int32_t *counts, int32_t *task_off,
+                        uint64_t *keys_out, const uint64_t *tau_key, uint64_t *fin,
+                        int32_t *fin_count, const MQMeta *d_meta, const typename Tr<S>::V *qv,
+                        int D) {
+    task_prefix_kernel<<<1, 1024, 0, idx->stream>>>(counts, mode == 0 ? LT : -1, n_mq, pl.n_len, li,
+                                                    task_off);
+    CHECK_LAUNCH();
+    DtwParams<S> p;
+    p.series = (const S *)idx->d_series;
+    p.meta = d_meta;
+    p.qv = qv;
+    p.D = D;
+    p.n_len = pl.n_len;
+    p.li = li;
+    p.d = pl.len[li];
+    p.n_mq = n_mq;
+    p.mode = mode;
+    p.list = list;
+    p.LT = LT;
+    p.counts = counts;
+    p.task_off = task_off;
+    p.keys_out = keys_out;
+    p.tau_key = tau_key;
+    p.fin = fin;
+    p.fin_count = fin_count;
+    launch_dtw<S>(pl.rho[li], p, 0, idx->stream);
+    CHECK_LAUNCH();
+    return SMILER_OK;
+}
+
+struct PhaseTimer {
+    smiler_index *idx;
+    bool on;
+    std::vector<std::pair<int, int>> marks;  // (phase, event index)
+    int next = 0;
+    int mark(int phase) {
+        if (!on) return SMILER_OK;
+        if (next >= (int)idx->events.size()) {
+            cudaEvent_t ev;
+            CU(cudaEventCreate(&ev));
+            idx->events.push_back(ev);
+        }
+        CU(cudaEventRecord(idx->events[next], idx->stream));
+        marks.push_back({phase, next});
+        next++;
+        return SMILER_OK;
+    }
+};
+
+template <typename S>
+static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query_sensor_in,
+                    int32_t n_mq, const int32_t *lengths_in, int32_t n_len, int32_t k, int64_t *ids,
+                    void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts,
+                    bool lb_only, void *post_out, void *lb_out) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    using V4 = typename Tr<S>::V4;
+    smiler_knn_opts o;
+    memset(&o, 0, sizeof(o));
+    if (opts) o = *opts;
+    if (!queries) return fail(SMILER_EINVAL, "queries is NULL");
+    if (n_mq < 1) return fail(SMILER_EINVAL, "n_mq must be >= 1");
+    if (!lengths_in) return fail(SMILER_EINVAL, "lengths is NULL");
+    if (!lb_only && (!ids || !dists)) return fail(SMILER_EINVAL, "ids/dists is NULL");
+    TRY(set_device(idx));
+    std::vector<int32_t> lens_h(n_len > 0 ? n_len : 1);
+    if (n_len < 1 || n_len > kMaxLen) return fail(SMILER_EINVAL, "n_len must be in [1, %d]", kMaxLen);
+    if (is_device_ptr(lengths_in)) CU(cudaMemcpy(lens_h.data(), lengths_in, 4 * n_len, cudaMemcpyDeviceToHost));
+    else memcpy(lens_h.data(), lengths_in, 4 * n_len);
+    Plan pl;
+    TRY(validate_query(idx, lens_h.data(), n_len, lb_only ? 1 : k, pl));
+    const int D = pl.D, w = pl.w, nl = pl.n_len;
+    std::vector<int32_t> qsens(n_mq, 0);
+    if (query_sensor_in) {
+        if (is_device_ptr(query_sensor_in)) CU(cudaMemcpy(qsens.data(), query_sensor_in, 4 * (size_t)n_mq, cudaMemcpyDeviceToHost));
+        else memcpy(qsens.data(), query_sensor_in, 4 * (size_t)n_mq);
+    }
+    for (int j = 0; j < n_mq; j++) {
+        if (qsens[j] < 0 || qsens[j] >= (int)idx->sensors.size())
+            return fail(SMILER_EINVAL, "query_sensor[%d] = %d out of range", j, qsens[j]);
+        const SensorInfo &si = idx->sensors[qsens[j]];
+        if (!idx->shard && pl.D > si.n)
+            return fail(SMILER_EINVAL, "D = %d longer than sensor %d (%lld points)", pl.D, qsens[j], (long long)si.n);
+        if (idx->shard) {
+            const int64_t need_lo = std::max<int64_t>(0, si.t_lo + si.slice_begin - pl.rho_env);
+            const int64_t need_hi = std::min<int64_t>(si.n_global, si.t_hi + si.slice_begin + pl.D - 1 + pl.rho_env);
+            if (si.slice_begin > need_lo || si.slice_begin + si.n < need_hi)
+                return fail(SMILER_EINVAL, "shard halo too small: need [%lld, %lld), have [%lld, %lld)",
+                            (long long)need_lo, (long long)need_hi, (long long)si.slice_begin,
+                            (long long)(si.slice_begin + si.n));
+        }
+    }
+    if (lb_only) {
+        for (int j = 1; j < n_mq; j++)
+            if (idx->sensors[qsens[j]].n != idx->sensors[qsens[0]].n)
+                return fail(SMILER_EINVAL, "smiler_lower_bounds needs sensors of equal length");
+    }
+    void *dUC, *dLC;
+    TRY(ensure_envelope(idx, pl.rho_env, &dUC, &dLC));
+
+    const size_t es = sizeof(S);
+    const bool q_dev = is_device_ptr(queries);
+    const bool out_dev = lb_only ? (is_device_ptr(lb_out) || (post_out && is_device_ptr(post_out)))
+                                 : (is_device_ptr(ids) && is_device_ptr(dists));
+    if (!lb_only && (is_device_ptr(ids) != is_device_ptr(dists)))
+        return fail(SMILER_EINVAL, "ids and dists must both be host or both be device buffers");
+
+    // ---- per-MQ sizes and chunking -------------------------------------
+    const int n_sw = D - w + 1;
+    auto mq_bytes = [&](int j) -> size_t {
+        const SensorInfo &si = idx->sensors[qsens[j]];
+        const size_t ndw = (size_t)(si.n / w);
+        return (size_t)n_sw * ndw * 8 + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
+    };
+    size_t budget = (size_t)24 << 30;
+    {
+        size_t fr = 0, tot = 0;
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) budget = std::min(budget, fr / 2);
+        cudaGetLastError();
+    }
+    int chunk_max = o.mq_chunk > 0 ? o.mq_chunk : 65535;
+    chunk_max = std::min(chunk_max, 65535);
+
+    if (stats) {
+        memset(stats, 0, sizeof(*stats));
+        TRY(idx->tmp.ensure(8 * (kMaxLen + 1)));
+        CU(cudaMemsetAsync(idx->tmp.p, 0, 8 * (kMaxLen + 1), idx->stream));
+    }
+    PhaseTimer tm{idx, stats != nullptr && o.timing != 0};
+    int launches = 0;
+    int64_t tau_slots_total = 0;
+    double cells_acc = 0, bf_cells = 0;
+    int64_t cand_total = 0, surv_total = 0, fin_total = 0, post_bytes = 0, lb_bytes = 0;
+    int n_chunks = 0;
+
+    for (int c0 = 0; c0 < n_mq;) {
+        // choose the chunk
+        size_t acc = 0;
+        int c1 = c0;
+        while (c1 < n_mq && c1 - c0 < chunk_max) {
+            size_t b = mq_bytes(c1);
+            if (c1 > c0 && acc + b > budget) break;
+            acc += b;
+            c1++;
+        }
+        const int B = c1 - c0;
+        n_chunks++;
+        // ---- metadata ------------------------------------------------------
+        std::vector<MQMeta> meta(B);
+        int64_t post_tot = 0, seg_tot = 0;
+        int nblk_min = INT32_MAX, nblk_max = 0;
+        for (int j = 0; j < B; j++) {
+            const SensorInfo &si = idx->sensors[qsens[c0 + j]];
+            MQMeta &m = meta[j];
+            m.series_off = si.off;
+            m.n = si.n;
+            m.origin = si.origin;
+            m.t_lo = si.t_lo;
+            m.t_hi = si.t_hi;
+            m.n_dw = si.n / w;
+            m.post_off = post_tot;
+            m.seg_off = seg_tot;
+            m.nblk = (int)(si.n / ((int64_t)pl.RT * w) + 1);
+            m.sensor = qsens[c0 + j];
+            post_tot += (int64_t)n_sw * m.n_dw;
+            seg_tot += (int64_t)nl * si.n;
+            nblk_min = std::min(nblk_min, m.nblk);
+            nblk_max = std::max(nblk_max, m.nblk);
+            for (int i = 0; i < nl; i++) {
+                const int64_t tb = std::max<int64_t>(0, si.t_lo);
+                const int64_t te = std::min<int64_t>(si.t_hi, si.n - pl.len[i] + 1);
+                const int64_t nc = te > tb ? te - tb : 0;
+                cand_total += nc;
+                bf_cells += (double)nc * (double)dtw_cells(pl.len[i], pl.rho[i]);
+            }
+        }
+        int E = 0;
+        if (!lb_only && !o.no_prune) E = std::min(8, std::max(1, (2 * pl.k + nblk_min - 1) / nblk_min));
+        const int LT = std::max(1, nblk_max * E);
+        QParams P;
+        memset(&P, 0, sizeof(P));
+        P.D = D;
+        P.w = w;
+        P.n_len = nl;
+        P.k = pl.k;
+        P.rho_env = pl.rho_env;
+        P.E = E;
+        P.LT = LT;
+        P.n_mq = B;
+        for (int i = 0; i < nl; i++) {
+            P.len[i] = pl.len[i];
+            P.rho[i] = pl.rho[i];
+        }
+        const int nseg = B * nl;
+        TRY(idx->meta.ensure(sizeof(MQMeta) * B));
+        TRY(idx->queries.ensure(es * (size_t)B * D));
+        TRY(idx->qv.ensure(sizeof(V) * (size_t)B * D));
+        TRY(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
+        TRY(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
+        TRY(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
+        if (!lb_only) {
+            TRY(idx->surv.ensure(4 * (size_t)seg_tot));
+            TRY(idx->fin.ensure(8 * (size_t)seg_tot));
+            TRY(idx->tauc.ensure(4 * (size_t)nseg * LT));
+            TRY(idx->tauk.ensure(8 * (size_t)nseg * LT));
+            TRY(idx->taukey.ensure(8 * (size_t)nseg));
+            TRY(idx->thr.ensure(4 * (size_t)nseg));
+            TRY(idx->scount.ensure(4 * (size_t)nseg));
+            TRY(idx->fcount.ensure(4 * (size_t)nseg));
+            TRY(idx->taskoff.ensure(4 * (size_t)(B + 1) * nl * 2));
+            TRY(idx->out_ids.ensure(8 * (size_t)nseg * pl.k));
+            TRY(idx->out_d.ensure(4 * (size_t)nseg * pl.k));
+        }
+        MQMeta *d_meta = idx->meta.as<MQMeta>();
+        CU(cudaMemcpyAsync(d_meta, meta.data(), sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
+        CU(cudaMemcpyAsync(idx->queries.p, (const char *)queries + (size_t)c0 * D * es, es * (size_t)B * D,
+                           q_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, idx->stream));
+        TRY(tm.mark(0));
+        // ---- a2 ----------------------------------------------------------
+        query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env,
+                                                         idx->qv.as<V>(), idx->qtab.as<V4>());
+        CHECK_LAUNCH();
+        launches++;
+        TRY(tm.mark(1));
+        // ---- a3 ----------------------------------------------------------
+        {
+            int64_t ndw_max = 0;
+            for (auto &m : meta) ndw_max = std::max(ndw_max, m.n_dw);
+            if (ndw_max > 0) {
+                dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
+                size_t smem = sizeof(V4) * D;
+                auto go = [&](auto kern) {
+                    if (smem > 48 * 1024)
+                        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                    kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
+                                                           (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
+                                                           w, idx->post.as<V2>());
+                };
+                switch (w) {
+                    case 4: go(window_lb_kernel<S, 4>); break;
+                    case 8: go(window_lb_kernel<S, 8>); break;
+                    case 16: go(window_lb_kernel<S, 16>); break;
+                    case 32: go(window_lb_kernel<S, 32>); break;
+                    default: go(window_lb_kernel<S, 0>); break;
+                }
+                CHECK_LAUNCH();
+                launches++;
+            }
+        }
+        post_bytes += post_tot * 8;
+        TRY(tm.mark(2));
+        // ---- a4 ----------------------------------------------------------
+        {
+            dim3 grid((unsigned)nblk_max, (unsigned)B);
+            size_t smem = (size_t)nl * pl.RT * (w + 1) * sizeof(V);
+            if (smem > 48 * 1024)
+                cudaFuncSetAttribute(group_scan_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            group_scan_kernel<S><<<grid, pl.RT, smem, idx->stream>>>(idx->post.as<V2>(), d_meta, P,
+                                                                     idx->lb.as<V>(), idx->tauc.as<int32_t>());
+            CHECK_LAUNCH();
+            launches++;
+        }
+        lb_bytes += 2 * seg_tot * 4;
+        TRY(tm.mark(3));
+        if (lb_only) {
+            // copy LB_w [n_mq][n_len][N] and postings out
+            const size_t lbb = sizeof(V) * (size_t)seg_tot;
+            const int64_t lb_off = (int64_t)meta[0].n * nl * c0;
+            CU(cudaMemcpyAsync((char *)lb_out + lb_off * sizeof(V), idx->lb.p, lbb,
+                               out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
+            if (post_out) {
+                const int64_t po = (int64_t)n_sw * meta[0].n_dw * c0;
+                CU(cudaMemcpyAsync((char *)post_out + po * sizeof(V2), idx->post.p, sizeof(V2) * (size_t)post_tot,
+                                   out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
+            }
+            c0 = c1;
+            continue;
+        }
+        int32_t *scount = idx->scount.as<int32_t>();
+        int32_t *fcount = idx->fcount.as<int32_t>();
+        uint64_t *taukey = idx->taukey.as<uint64_t>();
+        uint32_t *thr = idx->thr.as<uint32_t>();
+        CU(cudaMemsetAsync(scount, 0, 4 * (size_t)nseg, idx->stream));
+        CU(cudaMemsetAsync(fcount, 0, 4 * (size_t)nseg, idx->stream));
+        int32_t *taskoff = idx->taskoff.as<int32_t>();
+        // ---- a5: tau ------------------------------------------------------
+        if (!o.no_prune) {
+            for (int i = 0; i < nl; i++) {
+                TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
+                                    taskoff + (size_t)i * (B + 1), idx->tauk.as<uint64_t>(), nullptr,
+                                    nullptr, nullptr, d_meta, idx->qv.as<V>(), D));
+                launches += 2;
+                tau_slots_total += (int64_t)B * LT;
+                cells_acc += (double)B * LT * (double)dtw_cells(pl.len[i], pl.rho[i]);
+            }
+            tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
+            CHECK_LAUNCH();
+            launches++;
+        } else {
+            CU(cudaMemsetAsync(taukey, 0xFF, 8 * (size_t)nseg, idx->stream));
+        }
+        TRY(tm.mark(4));
+        // ---- a6 ----------------------------------------------------------
+        {
+            int64_t nmax = 0;
+            for (auto &m : meta) nmax = std::max(nmax, m.n);
+            if (!o.no_prune) {
+                dim3 grid((unsigned)((nmax + kFiltThreads * kFiltItems - 1) / (kFiltThreads * kFiltItems)),
+                          (unsigned)nseg);
+                filter_kernel<S><<<grid, kFiltThreads, 0, idx->stream>>>(idx->lb.as<V>(), d_meta, P, thr,
+                                                                         idx->surv.as<int32_t>(), scount);
+            } else {
+                dim3 grid((unsigned)std::min<int64_t>((nmax + 255) / 256, 1024), (unsigned)nseg);
+                all_candidates_kernel<<<grid, 256, 0, idx->stream>>>(d_meta, P, idx->surv.as<int32_t>(), scount);
+            }
+            CHECK_LAUNCH();
+            launches++;
+        }
+        TRY(tm.mark(5));
+        // ---- a7 ----------------------------------------------------------
+        int32_t *taskoff2 = taskoff + (size_t)nl * (B + 1);
+        for (int i = 0; i < nl; i++) {
+            TRY(run_dtw_list<S>(idx, pl, i, B, 1, idx->surv.as<int32_t>(), 0, scount,
+                                taskoff2 + (size_t)i * (B + 1), nullptr, taukey, idx->fin.as<uint64_t>(),
+                                fcount, d_meta, idx->qv.as<V>(), D));
+            launches += 2;
+        }
+        TRY(tm.mark(6));
+        // ---- a8 ----------------------------------------------------------
+        topk_kernel<S><<<nseg, 512, 0, idx->stream>>>(idx->fin.as<uint64_t>(), fcount, d_meta, P,
+                                                      idx->out_ids.as<int64_t>(), idx->out_d.as<V>());
+        CHECK_LAUNCH();
+        launches++;
+        TRY(tm.mark(7));
+        const size_t ob = (size_t)nseg * pl.k;
+        CU(cudaMemcpyAsync(ids + (size_t)c0 * nl * pl.k, idx->out_ids.p, 8 * ob,
+                           out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
+        CU(cudaMemcpyAsync((char *)dists + (size_t)c0 * nl * pl.k * 4, idx->out_d.p, 4 * ob,
+                           out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
+        if (stats) {
+            accum_counts_kernel<<<1, 256, 0, idx->stream>>>(scount, fcount, nseg, nl,
+                                                            idx->tmp.as<unsigned long long>());
+            CHECK_LAUNCH();
+        }
+        c0 = c1;
+    }
+    unsigned long long acc_h[kMaxLen + 1] = {0};
+    if (stats && !lb_only)
+        CU(cudaMemcpyAsync(acc_h, idx->tmp.p, 8 * (kMaxLen + 1), cudaMemcpyDeviceToHost, idx->stream));
+    if (!out_dev || stats) CU(cudaStreamSynchronize(idx->stream));
+    CHECK_LAUNCH();
+    if (stats) {
+        fin_total = (int64_t)acc_h[0];
+        for (int i = 0; i < nl; i++) {
+            surv_total += (int64_t)acc_h[1 + i];
+            cells_acc += (double)acc_h[1 + i] * (double)dtw_cells(pl.len[i], pl.rho[i]);
+        }
+        stats->candidates = cand_total;
+        stats->tau_verified = tau_slots_total;
+        stats->survivors = surv_total;
+        stats->finalists = fin_total;
+        stats->dtw_cells = cells_acc;
+        stats->bf_cells = bf_cells;
+        stats->posting_bytes = post_bytes;
+        stats->lb_bytes = lb_bytes;
+        stats->kernel_launches = launches;
+        stats->mq_chunks = n_chunks;
+        if (tm.on) {
+            double *slots[8] = {nullptr, &stats->ns_prep, &stats->ns_window_lb, &stats->ns_group_scan,
+                                &stats->ns_tau, &stats->ns_filter, &stats->ns_verify, &stats->ns_select};
+            for (size_t x = 1; x < tm.marks.size(); x++) {
+                int ph = tm.marks[x].first;
+                if (ph == 0) continue;
+                float ms = 0;
+                CU(cudaEventElapsedTime(&ms, idx->events[tm.marks[x - 1].second], idx->events[tm.marks[x].second]));
+                *slots[ph] += ms * 1e6;
+                stats->ns_total += ms * 1e6;
+            }
+        }
+    }
+    return SMILER_OK;
+}
+
+extern "C" int smiler_knn_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                             int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
+                             void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (idx->dtype == SMILER_I16)
+        return knn_impl<int16_t>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats,
+                                 opts, false, nullptr, nullptr);
+    return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, opts,
+                           false, nullptr, nullptr);
+}
+
+extern "C" int smiler_knn(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                          int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
+                          void *dists, smiler_knn_stats *stats) {
+    return smiler_knn_ex(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, nullptr);
+}
+
+extern "C" int smiler_lower_bounds(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                   int32_t n_mq, const int32_t *lengths, int32_t n_len, void *postings,
+                                   void *lbw) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!lbw) return fail(SMILER_EINVAL, "lbw is NULL");
+    smiler_knn_opts o;
+    memset(&o, 0, sizeof(o));
+    if (idx->dtype == SMILER_I16)
+        return knn_impl<int16_t>(idx, queries, query_sensor, n_mq, lengths, n_len, 1, nullptr, nullptr,
+                                 nullptr, &o, true, postings, lbw);
+    return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, 1, nullptr, nullptr, nullptr,
+                           &o, true, postings, lbw);
+}
+
+extern "C" int smiler_index_envelope(smiler_index *idx, int32_t sensor, int32_t rho, void *U, void *L) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!U || !L) return fail(SMILER_EINVAL, "U/L is NULL");
+    if (sensor < 0 || sensor >= (int)idx->sensors.size()) return fail(SMILER_EINVAL, "bad sensor %d", sensor);
+    if (rho < 0) return fail(SMILER_EINVAL, "rho < 0");
+    TRY(set_device(idx));
+    void *dU, *dL;
+    TRY(ensure_envelope(idx, rho, &dU, &dL));
+    const SensorInfo &si = idx->sensors[sensor];
+    const size_t es = esize(idx->dtype);
+    CU(cudaMemcpyAsync(U, (char *)dU + si.off * es, si.n * es, cudaMemcpyDefault, idx->stream));
+    CU(cudaMemcpyAsync(L, (char *)dL + si.off * es, si.n * es, cudaMemcpyDefault, idx->stream));
+    CU(cudaStreamSynchronize(idx->stream));
+    return SMILER_OK;
+}
+
+template <typename S>
+static int dtw_impl(smiler_index *idx, int32_t sensor, const void *q, int32_t d, int32_t rho,
+                    const int64_t *ts, int64_t n_t, void *dists) {
+    using V = typename Tr<S>::V;
+    const SensorInfo &si = idx->sensors[sensor];
+    if (d < 1 || d > kMaxD || d > si.n) return fail(SMILER_EINVAL, "bad d = %d", d);
+    if (rho < 0) return fail(SMILER_EINVAL, "rho < 0");
+    rho = std::min(rho, d - 1);
+    if (rho > kMaxRhoFast) return fail(SMILER_EINVAL, "rho %d exceeds %d", rho, kMaxRhoFast);
+    if (n_t < 1 || n_t > INT32_MAX / 2) return fail(SMILER_EINVAL, "bad n_t");
+    std::vector<int64_t> th(n_t);
+    if (is_device_ptr(ts)) CU(cudaMemcpy(th.data(), ts, 8 * n_t, cudaMemcpyDeviceToHost));
+    else memcpy(th.data(), ts, 8 * n_t);
+    std::vector<int32_t> t32(n_t);
+    for (int64_t x = 0; x < n_t; x++) {
+        if (th[x] < 0 || th[x] > si.n - d) return fail(SMILER_EINVAL, "ts[%lld] = %lld out of range", (long long)x, (long long)th[x]);
+        t32[x] = (int32_t)th[x];
+    }
+    MQMeta m;
+    memset(&m, 0, sizeof(m));
+    m.series_off = si.off;
+    m.n = si.n;
+    m.t_hi = si.n;
+    TRY(idx->meta.ensure(sizeof(MQMeta)));
+    TRY(idx->queries.ensure(sizeof(S) * d));
+    TRY(idx->qv.ensure(sizeof(V) * d));
+    TRY(idx->qtab.ensure(sizeof(typename Tr<S>::V4) * d));
+    TRY(idx->tauc.ensure(4 * (size_t)n_t));
+    TRY(idx->tauk.ensure(8 * (size_t)n_t));
+    TRY(idx->taskoff.ensure(8));
+    TRY(idx->out_d.ensure(4 * (size_t)n_t));
+    CU(cudaMemcpyAsync(idx->meta.p, &m, sizeof(m), cudaMemcpyHostToDevice, idx->stream));
+    CU(cudaMemcpyAsync(idx->queries.p, q, sizeof(S) * d, cudaMemcpyDefault, idx->stream));
+    CU(cudaMemcpyAsync(idx->tauc.p, t32.data(), 4 * n_t, cudaMemcpyHostToDevice, idx->stream));
+    query_prep_kernel<S><<<1, 256, 0, idx->stream>>>(idx->queries.as<S>(), d, 0, idx->qv.as<V>(),
+                                                     idx->qtab.as<typename Tr<S>::V4>());
+    CHECK_LAUNCH();
+    Plan pl;
+    pl.n_len = 1;
+    pl.len = {d};
+    pl.rho = {rho};
+    TRY(run_dtw_list<S>(idx, pl, 0, 1, 0, idx->tauc.as<int32_t>(), (int)n_t, nullptr, idx->taskoff.as<int32_t>(),
+                        idx->tauk.as<uint64_t>(), nullptr, nullptr, nullptr, idx->meta.as<MQMeta>(),
+                        idx->qv.as<V>(), d));
+    keys_to_dists_kernel<V><<<std::max<int64_t>(1, std::min<int64_t>((n_t + 255) / 256, 4096)), 256, 0,
+                             idx->stream>>>(idx->tauk.as<uint64_t>(), n_t, idx->out_d.as<V>());
+    CHECK_LAUNCH();
+    CU(cudaMemcpyAsync(dists, idx->out_d.p, 4 * n_t, cudaMemcpyDefault, idx->stream));
+    CU(cudaStreamSynchronize(idx->stream));
+    return SMILER_OK;
+}
+
+extern "C" int smiler_dtw(smiler_index *idx, int32_t sensor, const void *q, int32_t d, int32_t rho,
+                          const int64_t *ts, int64_t n_t, void *dists) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!q || !ts || !dists) return fail(SMILER_EINVAL, "NULL argument");
+    if (sensor < 0 || sensor >= (int)idx->sensors.size()) return fail(SMILER_EINVAL, "bad sensor %d", sensor);
+    TRY(set_device(idx));
+    if (idx->dtype == SMILER_I16) return dtw_impl<int16_t>(idx, sensor, q, d, rho, ts, n_t, dists);
+    return dtw_impl<float>(idx, sensor, q, d, rho, ts, n_t, dists);
+}
+
+extern "C" int smiler_merge_topk(const int64_t *ids_in, const void *dists_in, smiler_dtype dtype, int32_t G,
+                                 int32_t rows, int32_t k, int64_t *ids_out, void *dists_out, int32_t device,
+                                 void *cuda_stream) {
+    if (!ids_in || !dists_in || !ids_out || !dists_out) return fail(SMILER_EINVAL, "NULL argument");
+    if (G < 1 || rows < 1 || k < 1 || k > kMaxK || (int64_t)G * k > kSortCap)
+        return fail(SMILER_EINVAL, "need G >= 1, rows >= 1, 1 <= k <= %d, G*k <= %d", kMaxK, kSortCap);
+    if (dtype != SMILER_I16 && dtype != SMILER_F32) return fail(SMILER_EINVAL, "bad dtype");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return fail(SMILER_ECUDA, "no CUDA device available; there is no CPU fallback");
+    }
+    CU(cudaSetDevice(device));
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    const size_t nin = (size_t)G * rows * k, nout = (size_t)rows * k;
+    const bool in_dev = is_device_ptr(ids_in) && is_device_ptr(dists_in);
+    const bool out_dev = is_device_ptr(ids_out) && is_device_ptr(dists_out);
+    void *buf = nullptr;
+    const size_t need = (in_dev ? 0 : nin * 12) + (out_dev ? 0 : nout * 12);
+    if (need) CU(cudaMalloc(&buf, need));
+    const int64_t *di = ids_in;
+    const void *dd = dists_in;
+    char *cur = (char *)buf;
+    if (!in_dev) {
+        CU(cudaMemcpyAsync(cur, ids_in, nin * 8, cudaMemcpyHostToDevice, st));
+        CU(cudaMemcpyAsync(cur + nin * 8, dists_in, nin * 4, cudaMemcpyHostToDevice, st));
+        di = (const int64_t *)cur;
+        dd = cur + nin * 8;
+        cur += nin * 12;
+    }
+    int64_t *io = ids_out;
+    void *doo = dists_out;
+    if (!out_dev) {
+        io = (int64_t *)cur;
+        doo = cur + nout * 8;
+    }
+    if (dtype == SMILER_I16)
+        merge_topk_kernel<int32_t><<<rows, 512, 0, st>>>(di, (const int32_t *)dd, G, rows, k, io,
+                                                         (int32_t *)doo, 0x7FFFFFFF);
+    else
+        merge_topk_kernel<float><<<rows, 512, 0, st>>>(di, (const float *)dd, G, rows, k, io, (float *)doo,
+                                                       INFINITY);
+    CHECK_LAUNCH();
+    if (!out_dev) {
+        CU(cudaMemcpyAsync(ids_out, io, nout * 8, cudaMemcpyDeviceToHost, st));
+        CU(cudaMemcpyAsync(dists_out, doo, nout * 4, cudaMemcpyDeviceToHost, st));
+    }
+    if (need) {
+        CU(cudaStreamSynchronize(st));
+        cudaFree(buf);
+    }
+    return SMILER_OK;
+}

@@ -1,0 +1,265 @@
+"""Thin ctypes binding of libsmiler.so (include/smiler.h).
+
+Argument marshalling only: every step of the Search Step runs in the library's
+CUDA kernels.  Buffers may be numpy arrays (host) or torch tensors (host or
+CUDA); their raw pointers are passed straight to the C ABI.  There is no CPU
+fallback: if libsmiler.so is missing or has no usable CUDA device the calls
+raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Any, Optional, Sequence, Tuple
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsmiler.so")
+
+SMILER_I16 = 0
+SMILER_F32 = 1
+STATUS = {0: "OK", -1: "EINVAL", -2: "ERANGE", -3: "ENOMEM", -4: "ECUDA", -5: "ENCCL"}
+
+
+class SmilerError(RuntimeError):
+    def __init__(self, fn: str, code: int, msg: str):
+        super().__init__("%s -> %s: %s" % (fn, STATUS.get(code, code), msg))
+        self.code = code
+
+
+class KnnStats(ctypes.Structure):
+    _fields_ = [("candidates", ctypes.c_int64), ("tau_verified", ctypes.c_int64),
+                ("survivors", ctypes.c_int64), ("finalists", ctypes.c_int64),
+                ("dtw_cells", ctypes.c_double), ("bf_cells", ctypes.c_double),
+                ("posting_bytes", ctypes.c_int64), ("lb_bytes", ctypes.c_int64),
+                ("kernel_launches", ctypes.c_int32), ("mq_chunks", ctypes.c_int32),
+                ("ns_prep", ctypes.c_double), ("ns_window_lb", ctypes.c_double),
+                ("ns_group_scan", ctypes.c_double), ("ns_tau", ctypes.c_double),
+                ("ns_filter", ctypes.c_double), ("ns_verify", ctypes.c_double),
+                ("ns_select", ctypes.c_double), ("ns_total", ctypes.c_double)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class KnnOpts(ctypes.Structure):
+    _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
+                ("mq_chunk", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libsmiler.so (raises if it has not been built: no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError("libsmiler.so not built (run python -m paper_conf_sigmod_zhout15_b200.build); "
+                              "there is no CPU fallback")
+        L = ctypes.CDLL(LIB_PATH)
+        P, i32, i64, f32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_float
+        L.smiler_index_build.argtypes = [P, i32, i64, P, i32, i32, f32, i32, P, ctypes.POINTER(P)]
+        L.smiler_index_build_shard.argtypes = [P, i32, i64, i64, i64, i64, i64, i32, f32, i32, P,
+                                               ctypes.POINTER(P)]
+        L.smiler_knn.argtypes = [P, P, P, i32, P, i32, i32, P, P, P]
+        L.smiler_knn_ex.argtypes = [P, P, P, i32, P, i32, i32, P, P, P, P]
+        L.smiler_merge_topk.argtypes = [P, P, i32, i32, i32, i32, P, P, i32, P]
+        L.smiler_index_envelope.argtypes = [P, i32, i32, P, P]
+        L.smiler_lower_bounds.argtypes = [P, P, P, i32, P, i32, P, P]
+        L.smiler_dtw.argtypes = [P, i32, P, i32, i32, P, i64, P]
+        L.smiler_free.argtypes = [P]
+        L.smiler_free.restype = None
+        L.smiler_last_error.restype = ctypes.c_char_p
+        L.smiler_abi_version.restype = i32
+        for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex",
+                  "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_dtw"):
+            getattr(L, f).restype = i32
+        _lib = L
+    return _lib
+
+
+def _check(fn: str, rc: int):
+    if rc != 0:
+        raise SmilerError(fn, rc, lib().smiler_last_error().decode())
+
+
+def _ptr(x: Any) -> Optional[int]:
+    if x is None:
+        return None
+    if isinstance(x, np.ndarray):
+        assert x.flags["C_CONTIGUOUS"], "arrays must be C-contiguous"
+        return x.ctypes.data
+    if hasattr(x, "data_ptr"):
+        assert x.is_contiguous(), "tensors must be contiguous"
+        return x.data_ptr()
+    raise TypeError(type(x))
+
+
+def _dtype_code(x: Any) -> int:
+    name = str(x.dtype)
+    if "int16" in name:
+        return SMILER_I16
+    if "float32" in name:
+        return SMILER_F32
+    raise TypeError("series dtype must be int16 or float32, got %s" % name)
+
+
+def _stream_ptr(stream) -> Optional[int]:
+    if stream is None:
+        return None
+    return int(getattr(stream, "cuda_stream", stream))
+
+
+# ---------------------------------------------------------------------------
+# The ABI calls, same names as include/smiler.h
+# ---------------------------------------------------------------------------
+def smiler_index_build(series, sensor_offsets=None, window: int = 16, band: float = 8.0,
+                       device: int = 0, stream=None) -> int:
+    h = ctypes.c_void_p()
+    offs = None
+    ns = 1
+    if sensor_offsets is not None:
+        offs = np.ascontiguousarray(sensor_offsets, dtype=np.int64)
+        ns = len(offs) - 1
+    n_total = int(series.shape[0]) if hasattr(series, "shape") else len(series)
+    _check("smiler_index_build",
+           lib().smiler_index_build(_ptr(series), _dtype_code(series), n_total, _ptr(offs), ns, window,
+                                    float(band), device, _stream_ptr(stream), ctypes.byref(h)))
+    return h.value
+
+
+def smiler_index_build_shard(slice_, slice_begin: int, n_global: int, t_begin: int, t_end: int,
+                             window: int, band: float, device: int = 0, stream=None) -> int:
+    h = ctypes.c_void_p()
+    _check("smiler_index_build_shard",
+           lib().smiler_index_build_shard(_ptr(slice_), _dtype_code(slice_), int(slice_.shape[0]),
+                                          slice_begin, n_global, t_begin, t_end, window, float(band),
+                                          device, _stream_ptr(stream), ctypes.byref(h)))
+    return h.value
+
+
+def smiler_knn(handle: int, queries, query_sensor, lengths, k: int, ids, dists,
+               stats: Optional[KnnStats] = None, opts: Optional[KnnOpts] = None) -> None:
+    """Fills ids [n_mq, n_len, k] int64 and dists [n_mq, n_len, k] int32/float32
+    (host numpy or device tensors, caller-allocated)."""
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    qs = None if query_sensor is None else (
+        query_sensor if hasattr(query_sensor, "data_ptr") else np.ascontiguousarray(query_sensor, np.int32))
+    n_mq = int(queries.shape[0])
+    _check("smiler_knn",
+           lib().smiler_knn_ex(handle, _ptr(queries), _ptr(qs), n_mq, _ptr(lens), len(lens), k, _ptr(ids),
+                               _ptr(dists), ctypes.byref(stats) if stats is not None else None,
+                               ctypes.byref(opts) if opts is not None else None))
+
+
+def smiler_merge_topk(ids_in, dists_in, G: int, rows: int, k: int, ids_out, dists_out,
+                      device: int = 0, stream=None) -> None:
+    _check("smiler_merge_topk",
+           lib().smiler_merge_topk(_ptr(ids_in), _ptr(dists_in), _dtype_code_dist(dists_in), G, rows, k,
+                                   _ptr(ids_out), _ptr(dists_out), device, _stream_ptr(stream)))
+
+
+def _dtype_code_dist(x) -> int:
+    name = str(x.dtype)
+    if "int32" in name:
+        return SMILER_I16
+    if "float32" in name:
+        return SMILER_F32
+    raise TypeError("dists dtype must be int32 or float32, got %s" % name)
+
+
+def smiler_index_envelope(handle: int, sensor: int, rho: int, U, L) -> None:
+    _check("smiler_index_envelope", lib().smiler_index_envelope(handle, sensor, rho, _ptr(U), _ptr(L)))
+
+
+def smiler_lower_bounds(handle: int, queries, query_sensor, lengths, postings, lbw) -> None:
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    qs = None if query_sensor is None else np.ascontiguousarray(query_sensor, np.int32)
+    _check("smiler_lower_bounds",
+           lib().smiler_lower_bounds(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens),
+                                     len(lens), _ptr(postings), _ptr(lbw)))
+
+
+def smiler_dtw(handle: int, sensor: int, q, rho: int, ts, dists) -> None:
+    tsa = np.ascontiguousarray(ts, dtype=np.int64) if not hasattr(ts, "data_ptr") else ts
+    _check("smiler_dtw", lib().smiler_dtw(handle, sensor, _ptr(q), int(q.shape[0]), rho, _ptr(tsa),
+                                          int(tsa.shape[0]), _ptr(dists)))
+
+
+def smiler_free(handle: Optional[int]) -> None:
+    lib().smiler_free(handle)
+
+
+def smiler_abi_version() -> int:
+    return int(lib().smiler_abi_version())
+
+
+# ---------------------------------------------------------------------------
+# Convenience wrapper (host numpy in, host numpy out)
+# ---------------------------------------------------------------------------
+class Index:
+    """RAII-style owner of one smiler_index handle."""
+
+    def __init__(self, series, sensor_offsets=None, window: int = 16, band: float = 8.0,
+                 device: int = 0, stream=None, _handle: Optional[int] = None):
+        self.dtype = _dtype_code(series)
+        self.handle = _handle if _handle is not None else smiler_index_build(
+            series, sensor_offsets, window, band, device, stream)
+
+    @classmethod
+    def shard(cls, slice_, slice_begin, n_global, t_begin, t_end, window, band, device=0, stream=None):
+        h = smiler_index_build_shard(slice_, slice_begin, n_global, t_begin, t_end, window, band, device,
+                                     stream)
+        return cls(slice_, _handle=h)
+
+    def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
+            no_prune: bool = False, timing: bool = False, mq_chunk: int = 0):
+        n_mq = queries.shape[0]
+        ids = np.empty((n_mq, len(lengths), k), np.int64)
+        dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
+        st = KnnStats() if stats else None
+        op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk)
+        smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
+        if stats:
+            return ids, dists, st.as_dict()
+        return ids, dists
+
+    def envelope(self, sensor: int, rho: int, n: int):
+        dt = np.int16 if self.dtype == SMILER_I16 else np.float32
+        U = np.empty(n, dt)
+        L = np.empty(n, dt)
+        smiler_index_envelope(self.handle, sensor, rho, U, L)
+        return U, L
+
+    def lower_bounds(self, queries, lengths, n: int, window: int, query_sensor=None):
+        n_mq, D = queries.shape
+        vt = np.int32 if self.dtype == SMILER_I16 else np.float32
+        post = np.empty((n_mq, D - window + 1, n // window, 2), vt)
+        lbw = np.empty((n_mq, len(lengths), n), vt)
+        smiler_lower_bounds(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, post, lbw)
+        return post, lbw
+
+    def dtw(self, sensor: int, q, rho: int, ts):
+        vt = np.int32 if self.dtype == SMILER_I16 else np.float32
+        out = np.empty(len(ts), vt)
+        smiler_dtw(self.handle, sensor, np.ascontiguousarray(q), rho, ts, out)
+        return out
+
+    def close(self):
+        if self.handle:
+            smiler_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

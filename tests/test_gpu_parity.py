@@ -1,0 +1,348 @@
+"""Parity of the CUDA path (through the C ABI) with the oracle (-m gpu).
+
+i16: ids and dists bit-exact.  f32: ids and dists bit-exact against the oracle
+run in the kernel's precision (R16 pinned fma; the kNN decision is taken in the
+same precision on both sides), and dists within relative 1e-5 of the fp64
+oracle (BASELINE.json north_star tolerance) with id sets equal up to ties
+within that tolerance.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+THREADS = os.cpu_count() or 8
+
+
+@pytest.fixture(scope="module")
+def pkg():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sigmod_zhout15_b200 import build
+    build.build()
+    import paper_conf_sigmod_zhout15_b200 as p
+    return p
+
+
+def gpu_knn(pkg, wl, **kw):
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        return idx.knn(wl.queries, wl.lengths, wl.k, wl.query_sensor, **kw)
+
+
+def assert_f64_tolerance(ids, dists, oid, od):
+    """dists within rel 1e-5 of fp64; ids equal except ties within that tolerance."""
+    fin = np.isfinite(od)
+    assert (np.isfinite(dists) == fin).all()
+    assert np.allclose(dists[fin], od[fin], rtol=1e-5, atol=0)
+    for row in np.ndindex(ids.shape[:-1]):
+        a, b = ids[row], oid[row]
+        if (a == b).all():
+            continue
+        # differing positions must be near-ties of the oracle distances
+        for j in np.nonzero(a != b)[0]:
+            dj = od[row][j]
+            close = np.abs(od[row] - dj) <= 1e-5 * max(dj, 1e-30)
+            assert close.sum() >= 2 or j == len(a) - 1, (row, j)
+
+
+def check_workload(pkg, orc, wl, mq_subset=None, **kw):
+    ids, dists = gpu_knn(pkg, wl, **kw)
+    sel = list(range(wl.n_mq)) if mq_subset is None else list(mq_subset)
+    if wl.dtype == "i16":
+        oid, od = orc.knn(wl, mq_subset=sel, threads=THREADS)
+        np.testing.assert_array_equal(ids[sel], oid)
+        np.testing.assert_array_equal(dists[sel].astype(np.int64), od)
+    else:
+        oid32, od32 = orc.knn(wl, mode="f32", mq_subset=sel, threads=THREADS)
+        np.testing.assert_array_equal(ids[sel], oid32)
+        np.testing.assert_array_equal(dists[sel], od32)
+        oid64, od64 = orc.knn(wl, mode="f64", mq_subset=sel, threads=THREADS)
+        assert_f64_tolerance(ids[sel], dists[sel], oid64, od64)
+    # rows sorted by (dist, t), no duplicate t
+    for row in np.ndindex(ids.shape[:-1]):
+        r = [(d, t) for d, t in zip(dists[row].tolist(), ids[row].tolist()) if t >= 0]
+        assert r == sorted(r) and len({t for _, t in r}) == len(r)
+    return ids, dists
+
+
+# ---------------------------------------------------------------------------
+# a1 envelope, a3 postings, a4 LB_w
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("rho", [0, 1, 4, 25])
+def test_envelope_bit_exact(pkg, orc, dtype, rho):
+    wl = synth.make_workload("C3", dtype, n=5003, n_sensors=3)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        for s in range(3):
+            x = wl.sensor_slice(s)
+            U, L = idx.envelope(s, rho, len(x))
+            oU, oL = orc.envelope(x, rho)
+            np.testing.assert_array_equal(U.astype(oU.dtype), oU)
+            np.testing.assert_array_equal(L.astype(oL.dtype), oL)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("cfg,n,lengths,window,band", [
+    ("C2", 9001, [16, 32, 64, 128], 8, 0.1),
+    ("C3", 7013, [32, 64, 96], 16, 8.0),
+    ("C5", 4099, [16, 32, 64, 128], 8, 0.2),
+    ("C1", 1000, [8, 24], 16, 3.0),          # d < 2w-1: candidates with no full DW (R6)
+    ("C1", 777, [5, 13, 40], 5, 2.0),         # odd window, generic-w kernel
+])
+def test_postings_and_lbw(pkg, orc, dtype, cfg, n, lengths, window, band):
+    wl = synth.make_workload(cfg, dtype, n=n, n_sensors=1, mq_per_sensor=3, lengths=lengths,
+                             window=window, band=band)
+    rhos = wl.rhos()
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        post, lbw = idx.lower_bounds(wl.queries, wl.lengths, n, window)
+    for j in range(wl.n_mq):
+        res, (UC, LC, UQ, LQ, rho_env) = orc.mq_lower_bounds(wl.series, wl.queries[j], wl.lengths, rhos,
+                                                             window)
+        PE, PC = orc.postings(wl.series, UC, LC, wl.queries[j], UQ, LQ, window)
+        for i, d in enumerate(wl.lengths):
+            got = lbw[j, i, :n - d + 1]
+            exp = res[i]["w"]
+            if dtype == "i16":
+                np.testing.assert_array_equal(got.astype(np.int64), exp)
+            else:
+                np.testing.assert_allclose(got, exp, rtol=2e-5, atol=1e-6)
+        if dtype == "i16":
+            np.testing.assert_array_equal(post[j, :, :, 0].astype(np.int64), PE)
+            np.testing.assert_array_equal(post[j, :, :, 1].astype(np.int64), PC)
+        else:
+            np.testing.assert_allclose(post[j, :, :, 0], PE, rtol=2e-5, atol=1e-6)
+            np.testing.assert_allclose(post[j, :, :, 1], PC, rtol=2e-5, atol=1e-6)
+
+
+# ---------------------------------------------------------------------------
+# a7 banded DTW
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("d,rho", [(1, 0), (2, 1), (7, 3), (16, 1), (32, 4), (33, 8), (64, 6), (96, 8),
+                                   (128, 12), (128, 25), (100, 32), (20, 32), (300, 30), (1024, 5)])
+def test_dtw_kernel(pkg, orc, dtype, d, rho):
+    wl = synth.make_workload("C2", dtype, n=3000, mq_per_sensor=1, lengths=[max(d, 1)], window=1, band=1.0)
+    rng = np.random.default_rng(d * 100 + rho)
+    ts = rng.integers(0, 3000 - d + 1, size=203)   # several warps and a ragged tail
+    q = wl.queries[0]
+    with pkg.Index(wl.series, None, 1, 1.0) as idx:
+        got = idx.dtw(0, q, rho, ts)
+    r = min(rho, d - 1)
+    if dtype == "i16":
+        exp = orc.dtw_list(wl.series, q, r, ts)
+        np.testing.assert_array_equal(got.astype(np.int64), exp)
+    else:
+        e32, e64 = orc.dtw_list(wl.series, q, r, ts)
+        np.testing.assert_array_equal(got, e32)
+        np.testing.assert_allclose(got, e64, rtol=1e-5, atol=0)
+
+
+# ---------------------------------------------------------------------------
+# end-to-end kNN, configs C1..C5 at oracle sizes
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_golden_appendix_a_gpu(pkg, orc, dtype):
+    import json
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "appendix_a.json")))
+    C = np.array(g["C"], np.int16)
+    MQ = np.array([g["MQ"]], np.int16)
+    if dtype == "f32":   # P13: dyadic scaling keeps every f32 op exact
+        C = (C / 8.0).astype(np.float32)
+        MQ = (MQ / 8.0).astype(np.float32)
+    with pkg.Index(C, None, g["w"], float(g["rho"])) as idx:
+        ids, dists = idx.knn(MQ, g["lengths"], g["k"])
+        post, lbw = idx.lower_bounds(MQ, g["lengths"], len(C), g["w"])
+    scale = 64.0 if dtype == "f32" else 1.0
+    for li, iq in enumerate(g["IQ"]):
+        assert ids[0, li].tolist() == iq["knn_ids"]
+        assert (dists[0, li] * scale).tolist() == iq["knn_dists"]
+        assert (lbw[0, li, :len(iq["t"])] * scale).tolist() == iq["LB_w"]
+    assert (post[0, :, :, 0] * scale).tolist() == g["P_EQ"]
+    assert (post[0, :, :, 1] * scale).tolist() == g["P_EC"]
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c1_full(pkg, orc, dtype):
+    wl = synth.make_workload("C1", dtype)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c2_reduced(pkg, orc, dtype):
+    wl = synth.make_workload("C2", dtype, n=20011, mq_per_sensor=4)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c3_reduced(pkg, orc, dtype):
+    wl = synth.make_workload("C3", dtype, n=15007, n_sensors=6)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c4_reduced(pkg, orc, dtype):
+    wl = synth.make_workload("C4", dtype, n=60013, mq_per_sensor=2)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c5_reduced(pkg, orc, dtype):
+    wl = synth.make_workload("C5", dtype, n=12001, n_sensors=4, mq_per_sensor=2, consecutive=True)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_pruned_equals_no_prune(pkg, dtype):
+    wl = synth.make_workload("C5", dtype, n=30011, n_sensors=3, mq_per_sensor=3)
+    a = gpu_knn(pkg, wl)
+    b = gpu_knn(pkg, wl, no_prune=True)
+    np.testing.assert_array_equal(a[0], b[0])
+    np.testing.assert_array_equal(a[1], b[1])
+
+
+# ---------------------------------------------------------------------------
+# edge cases
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_edges_padding_and_small_series(pkg, orc, dtype):
+    # fewer candidates than k (R12), D == N for the longest item query
+    wl = synth.make_workload("C1", dtype, n=40, lengths=[8, 16, 40], k=30, window=4, band=3.0)
+    ids, dists = check_workload(pkg, orc, wl)
+    assert (ids[0, 2, 1:] == -1).all() and ids[0, 2, 0] == 0
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("band", [0.0, 40.0, 0.5])
+def test_edges_band_extremes(pkg, orc, dtype, band):
+    wl = synth.make_workload("C1", dtype, n=900, lengths=[6, 16, 31], k=5, window=3, band=band)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_edges_k1_single_length(pkg, orc, dtype):
+    wl = synth.make_workload("C3", dtype, n=5000, n_sensors=2, lengths=[64], k=1, window=16)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_edges_uneven_sensors(pkg, orc, dtype):
+    parts = [synth.quantise(synth.sensor_series(9, s, n, 200, 144), dtype) for s, n in
+             enumerate((3001, 517, 4099))]
+    series = np.concatenate([p[:n] for p, n in zip(parts, (3001, 517, 4099))])
+    offs = np.array([0, 3001, 3518, 7617], np.int64)
+    qs = np.stack([parts[s][n + 3:n + 3 + 64] for s, n in ((0, 3001), (1, 517), (2, 4099), (1, 517))])
+    wl = synth.Workload("uneven", dtype, series, offs, np.ascontiguousarray(qs),
+                        np.array([0, 1, 2, 1], np.int32), [16, 40, 64], 9, 8, 5.0)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_edges_constant_series_ties(pkg, dtype):
+    """All distances tie: the lowest t wins (R11); also drives the >4096-finalist
+    radix-select path of a8 in no-prune mode."""
+    n = 9000
+    series = np.full(n, 5, np.int16) if dtype == "i16" else np.full(n, 0.625, np.float32)
+    q = np.full((1, 32), 3, np.int16) if dtype == "i16" else np.full((1, 32), 0.375, np.float32)
+    for no_prune in (False, True):
+        with pkg.Index(series, None, 8, 2.0) as idx:
+            ids, dists = idx.knn(q, [16, 32], 7, no_prune=no_prune)
+        for li, d in enumerate((16, 32)):
+            assert ids[0, li].tolist() == list(range(7))
+            exp = d * 4 if dtype == "i16" else d * 0.0625
+            assert (dists[0, li] == exp).all()
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_shards_merge_equals_unsharded(pkg, orc, dtype):
+    """C4's window-range sharding: G logical shards with halos,
+    merged by smiler_merge_topk, equal the unsharded result and the oracle."""
+    wl = synth.make_workload("C4", dtype, n=40009, mq_per_sensor=2)
+    full_ids, full_d = check_workload(pkg, orc, wl)
+    N, D, w = len(wl.series), wl.D, wl.window
+    rho_env = max(wl.rhos())
+    for G in (2, 3, 4, 8):
+        bounds = [((N * g) // G) // w * w for g in range(G)] + [N]
+        outs_i, outs_d = [], []
+        for g in range(G):
+            t0, t1 = bounds[g], bounds[g + 1]
+            s0 = max(0, t0 - rho_env) // w * w
+            s1 = min(N, t1 + D - 1 + rho_env)
+            sl = np.ascontiguousarray(wl.series[s0:s1])
+            with pkg.Index.shard(sl, s0, N, t0, t1, w, wl.band) as idx:
+                i_, d_ = idx.knn(wl.queries, wl.lengths, wl.k)
+            outs_i.append(i_)
+            outs_d.append(d_)
+        I = np.ascontiguousarray(np.stack(outs_i))
+        Dd = np.ascontiguousarray(np.stack(outs_d))
+        rows = wl.n_mq * len(wl.lengths)
+        mi = np.empty((rows, wl.k), np.int64)
+        md = np.empty((rows, wl.k), Dd.dtype)
+        pkg.smiler_merge_topk(I, Dd, G, rows, wl.k, mi, md)
+        np.testing.assert_array_equal(mi.reshape(full_ids.shape), full_ids)
+        np.testing.assert_array_equal(md.reshape(full_d.shape), full_d)
+
+
+def test_errors_on_gpu(pkg):
+    x = np.zeros(100, np.int16)
+    x[5] = 2000
+    with pytest.raises(pkg.SmilerError) as ei:
+        pkg.Index(x, None, 8, 2.0)
+    assert ei.value.code == -2
+    y = np.zeros(100, np.int16)
+    with pkg.Index(y, None, 8, 2.0) as idx:
+        with pytest.raises(pkg.SmilerError) as ei:
+            idx.knn(np.zeros((1, 32), np.int16), [32, 16], 3)
+        assert ei.value.code == -1
+        with pytest.raises(pkg.SmilerError):
+            idx.knn(np.zeros((1, 200), np.int16), [200], 3)   # D > N
+        ids, d = idx.knn(np.zeros((1, 32), np.int16), [16, 32], 3)   # handle still usable
+        assert ids[0, 0].tolist() == [0, 1, 2]
+
+
+def test_repeated_calls_deterministic(pkg):
+    wl = synth.make_workload("C5", "f32", n=20000, n_sensors=2, mq_per_sensor=4)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        a = idx.knn(wl.queries, wl.lengths, wl.k, wl.query_sensor)
+        b = idx.knn(wl.queries, wl.lengths, wl.k, wl.query_sensor, mq_chunk=3)
+    np.testing.assert_array_equal(a[0], b[0])
+    np.testing.assert_array_equal(a[1], b[1])
+
+
+# ---------------------------------------------------------------------------
+# full size (BASELINE configs[1], the bench workload), sampled against the oracle
+# ---------------------------------------------------------------------------
+@pytest.mark.slow
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c2_full_size_sampled(pkg, orc, dtype):
+    wl = synth.make_workload("C2", dtype, mq_per_sensor=8)
+    rhos = wl.rhos()
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        ids, dists, st = idx.knn(wl.queries, wl.lengths, wl.k, stats=True)
+        bi, bd = idx.knn(wl.queries[:2], wl.lengths, wl.k, no_prune=True)
+        np.testing.assert_array_equal(ids[:2], bi)     # pruning exact at full size
+        np.testing.assert_array_equal(dists[:2], bd)
+        rng = np.random.default_rng(5)
+        for j in range(wl.n_mq):
+            for i, d in enumerate(wl.lengths):
+                q = wl.queries[j, wl.D - d:]
+                # every returned distance is the oracle's DTW of that candidate
+                ex = orc.dtw_list(wl.series, q, rhos[i], ids[j, i])
+                if dtype == "f32":
+                    ex = ex[0]
+                np.testing.assert_array_equal(dists[j, i].astype(ex.dtype), ex)
+                # random candidates: GPU DTW == oracle, and none beats the k-th result
+                ts = rng.integers(0, len(wl.series) - d + 1, size=64)
+                g = idx.dtw(0, q, rhos[i], ts)
+                e2 = orc.dtw_list(wl.series, q, rhos[i], ts)
+                if dtype == "f32":
+                    e2 = e2[0]
+                np.testing.assert_array_equal(g.astype(e2.dtype), e2)
+                kth = (dists[j, i, -1], ids[j, i, -1])
+                for t, v in zip(ts.tolist(), g.tolist()):
+                    assert (v, t) >= kth or t in ids[j, i]
+    assert st["survivors"] < st["candidates"]
