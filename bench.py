@@ -193,6 +193,9 @@ def main():
     ap.add_argument("--oracle-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--two-level", action="store_true", help="time the paper's two-level path (a3 -> HBM -> a4)")
+    ap.add_argument("--two-level-steps", type=int, default=3,
+                    help="extra steps of the two-level path for the LB-scan (a4) HBM figure; 0 = skip")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -246,7 +249,7 @@ def main():
     ids = torch.empty((wl.n_mq, n_len, k), dtype=torch.int64, device=dev)
     dd = torch.empty((wl.n_mq, n_len, k), dtype=torch.int32 if args.dtype == "i16" else torch.float32, device=dev)
     st = pkg.KnnStats()
-    op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0)
+    op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=int(args.two_level))
 
     def step(stats=None):
         pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, stats, op if stats is not None else None)
@@ -326,50 +329,89 @@ def main():
             dist.destroy_process_group()
         return
 
-    # ---- roofline of the dominant kernel --------------------------------------
+    # ---- secondary: the paper's two-level path (postings in HBM), for a4's HBM figure
+    two = None
+    if args.two_level_steps > 0 and not args.two_level:
+        op2 = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=1)
+        st2 = pkg.KnnStats()
+        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, st2, op2)
+        ph2 = {f: 0.0 for f in phase}
+        acc2 = {f: 0 for f in acc}
+        for _ in range(args.two_level_steps):
+            pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, st2, op2)
+            for f in ph2:
+                ph2[f] += getattr(st2, f)
+            for f in acc2:
+                acc2[f] += getattr(st2, f)
+        torch.cuda.synchronize(dev)
+        two = (ph2, acc2, args.two_level_steps)
+
+    # ---- rooflines ---------------------------------------------------------------
     peaks, peak_kind = load_peaks()
     alu = load_alu_peaks()
     steps = args.steps
-    chunks = max(1, acc["mq_chunks"])
-    ph_ms = {k_[3:]: v_ / 1e6 / steps for k_, v_ in phase.items()}
-    n_mq = wl.n_mq
-    lb_write = acc["lb_bytes"] / 2 / steps
-    scan_bytes = acc["posting_bytes"] / steps + lb_write           # a4 reads postings, writes LB_w
-    scan_s = phase["ns_group_scan"] / 1e9 / steps
-    scan_gbs = scan_bytes / scan_s / 1e9 if scan_s > 0 else 0.0
-    win_s = phase["ns_window_lb"] / 1e9 / steps
-    n_sw = wl.D - wl.window + 1
-    win_terms = n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window * wl.window
-                           for s in wl.query_sensor.tolist()) / 1.0
-    ver_s = phase["ns_verify"] / 1e9 / steps
-    tau_s = phase["ns_tau"] / 1e9 / steps
-    cells_s = acc["dtw_cells"] / steps / (ver_s + tau_s) if ver_s + tau_s > 0 else 0.0
     sm_mhz = ck.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    kernels = {
-        "group_scan_a4": {"bound": "hbm", "achieved": scan_gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                          "frac": scan_gbs / peaks["hbm_gbs"], "ms": scan_s * 1e3,
-                          "bytes_per_launch": scan_bytes / chunks},
-    }
     if alu:
         term_peak = alu["lbterm_per_clk_sm"] * alu["sms"] * sm_mhz * 1e6
         cell_peak = alu["dtw_cell_f32_per_clk_sm" if args.dtype == "f32" else "dtw_cell_i32_per_clk_sm"] * \
             alu["sms"] * sm_mhz * 1e6
+        alu_src = "profiles/alu_peaks.json (alu_bench) x median SM clock under load"
     else:
         term_peak = 148 * 16 * sm_mhz * 1e6
         cell_peak = 148 * 42.7 * sm_mhz * 1e6
-    win_rate = win_terms / win_s if win_s > 0 else 0.0
-    kernels["window_lb_a3"] = {"bound": "alu", "achieved": win_rate / 1e12, "peak": term_peak / 1e12,
-                               "unit": "T (SW,DW,j) term-pairs/s", "frac": win_rate / term_peak, "ms": win_s * 1e3}
-    kernels["dtw_verify_a7"] = {"bound": "alu", "achieved": cells_s / 1e12, "peak": cell_peak / 1e12,
-                                "unit": "T DTW cells/s", "frac": cells_s / cell_peak, "ms": (ver_s + tau_s) * 1e3}
-    dom = max(("group_scan_a4", scan_s), ("window_lb_a3", win_s), ("dtw_verify_a7", ver_s + tau_s),
-              key=lambda x: x[1])[0]
+        alu_src = "issue-rate estimate (no alu_peaks.json) x median SM clock"
+    n_sw = wl.D - wl.window + 1
+    # algorithmic work: (SW, DW, j) term pairs = n_sw * n_dw * w per MQ
+    win_terms = n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window * wl.window
+                           for s in wl.query_sensor.tolist())
+    post_bytes_step = 8 * n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window
+                                     for s in wl.query_sensor.tolist())
+    lb_bytes_step = 4 * n_len * sum(int(wl.offsets[s + 1] - wl.offsets[s]) for s in wl.query_sensor.tolist())
+
+    def rooflines(ph, ac, nsteps, fused):
+        ks = {}
+        win_s = ph["ns_window_lb"] / 1e9 / nsteps
+        if win_s > 0:
+            rate = win_terms / win_s
+            ks["lb_fused" if fused else "window_lb_a3"] = {
+                "bound": "alu", "achieved": rate / 1e12, "peak": term_peak / 1e12,
+                "unit": "T term-pairs/s", "frac": rate / term_peak, "ms": win_s * 1e3,
+                "algorithmic_per_launch": "%d (SW,DW,j) term pairs x MQs in the chunk" % (win_terms // wl.n_mq)}
+        gs_s = ph["ns_group_scan"] / 1e9 / nsteps
+        if not fused and gs_s > 0:
+            byts = post_bytes_step + lb_bytes_step
+            gbs = byts / gs_s / 1e9
+            ks["group_scan_a4"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                                   "frac": gbs / peaks["hbm_gbs"], "ms": gs_s * 1e3,
+                                   "algorithmic_bytes_per_step": byts}
+        v_s = (ph["ns_verify"] + ph["ns_tau"]) / 1e9 / nsteps
+        if v_s > 0:
+            cr = ac["dtw_cells"] / nsteps / v_s
+            ks["dtw_verify_a7"] = {"bound": "alu", "achieved": cr / 1e12, "peak": cell_peak / 1e12,
+                                   "unit": "T DTW cells/s", "frac": cr / cell_peak, "ms": v_s * 1e3}
+        f_s = ph["ns_filter"] / 1e9 / nsteps
+        if f_s > 0:
+            gbs = lb_bytes_step / f_s / 1e9
+            ks["filter_a6"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                               "frac": gbs / peaks["hbm_gbs"], "ms": f_s * 1e3}
+        return ks
+
+    fused_main = not args.two_level and wl.window in (4, 8, 16)
+    kernels = rooflines(phase, acc, steps, fused_main)
+    ph_ms = {k_[3:]: v_ / 1e6 / steps for k_, v_ in phase.items()}
+    dom = max(kernels.items(), key=lambda kv: kv[1]["ms"])[0]
     rf = dict(kernels[dom])
     rf["kernel"] = dom
     rf["traffic"] = None
-    rf["peak_source"] = ("MEASURED_PEAKS.json hbm_gbs (%s)" % peak_kind if rf["bound"] == "hbm"
-                         else ("profiles/alu_peaks.json x median SM clock" if alu else
-                               "guide unit counts x median SM clock (no alu_peaks.json)"))
+    rf["peak_source"] = ("MEASURED_PEAKS.json hbm_gbs (%s)" % peak_kind if rf["bound"] == "hbm" else alu_src)
+    two_level = None
+    if two is not None:
+        ph2, acc2, n2 = two
+        k2 = rooflines(ph2, acc2, n2, False)
+        two_level = {"ms_per_step": ph2["ns_total"] / 1e6 / n2,
+                     "value": wl.n_mq / (ph2["ns_total"] / 1e9 / n2),
+                     "phase_ms_per_step": {k_[3:]: v_ / 1e6 / n2 for k_, v_ in ph2.items()}, "kernels": k2}
+    scan = (two_level or {}).get("kernels", {}).get("group_scan_a4") or kernels.get("group_scan_a4")
 
     cpu = None
     if world == 1 and not args.no_cpu:
@@ -389,9 +431,11 @@ def main():
         "dtw_cells_per_s": acc["dtw_cells"] / steps / (ms_max / 1000.0 / steps) * world,
         "bf_equiv_cells_per_s": acc["bf_cells"] / steps / (ms_max / 1000.0 / steps) * world,
         "survivor_frac": acc["survivors"] / max(1, acc["candidates"]),
-        "lb_scan_gbs": scan_gbs, "lb_scan_frac_of_hbm": scan_gbs / peaks["hbm_gbs"],
+        "lb_scan_gbs": scan["achieved"] if scan else None,
+        "lb_scan_frac_of_hbm": scan["frac"] if scan else None,
+        "lb_path": "fused a3+a4 (posting rows on chip)" if fused_main else "two-level (postings in HBM)",
         "phase_ms_per_step": ph_ms,
-        "roofline": rf, "kernels": kernels,
+        "roofline": rf, "kernels": kernels, "two_level": two_level,
         "gpu_launches": int(acc["kernel_launches"]),
         "clocks": ck,
         "cpu_baseline": cpu,

@@ -76,7 +76,10 @@ typedef struct smiler_knn_opts {
     int32_t no_prune; /* 1: skip thresholding, verify every candidate (GPU brute force) */
     int32_t timing;   /* 1: record per-phase CUDA events into stats                     */
     int32_t mq_chunk; /* master queries per internal chunk; 0 = automatic               */
-    int32_t reserved[5];
+    int32_t two_level;/* 1: materialise the window-level posting lists in HBM (a3) and
+                         scan them (a4), as the paper's two-level index; 0: automatic
+                         (fused a3+a4 with posting rows kept on chip when w is 4/8/16) */
+    int32_t reserved[4];
 } smiler_knn_opts;
 
 /*

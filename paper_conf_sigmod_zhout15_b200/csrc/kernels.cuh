@@ -216,181 +216,7 @@ __global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D
     }
 }
 
-// ---------------------------------------------------------------------------
-// a3: window-level index (Sec. 4.3.1; Fig. 4-5).  For every sliding
-// window SW_b = MQ[D-w-b .. D-b) (R19) and disjoint window DW_r = c[rw..rw+w):
-//   P_EQ[b][r] = sum_j e(c[rw+j]; U(Q), L(Q) at D-w-b+j)    (LB_keogh(E(SW), DW))
-//   P_EC[b][r] = sum_j e(MQ[D-w-b+j]; U(C), L(C) at rw+j)   (LB_keogh(E(DW), SW))
-// One thread per DW r holds its w points and envelope in registers; the MQ
-// table sits in shared memory and is read as warp-uniform 16-byte broadcasts.
-// Output layout post[mq][b][r] = {P_EQ, P_EC}: coalesced over r.
-// ALU-bound: 8 ALU ops per (b, r, j) (clamp = 2 MNMX, sub, FMA/IMAD, twice).
-// WT = w at compile time (0 = runtime w, reading the DW from global memory).
-// ---------------------------------------------------------------------------
-template <typename S, int WT>
-__global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
-                                                       const MQMeta *meta,
-                                                       const typename Tr<S>::V4 *qtab, int D,
-                                                       int w, typename Tr<S>::V2 *post) {
-    using V = typename Tr<S>::V;
-    using V2 = typename Tr<S>::V2;
-    using V4 = typename Tr<S>::V4;
-    extern __shared__ __align__(16) unsigned char wl_smem[];
-    V4 *sq = reinterpret_cast<V4 *>(wl_smem);
-    const int mq = blockIdx.y;
-    const MQMeta m = meta[mq];
-    if ((int64_t)blockIdx.x * blockDim.x >= m.n_dw) return;
-    for (int p = threadIdx.x; p < D; p += blockDim.x) sq[p] = qtab[(int64_t)mq * D + p];
-    __syncthreads();
-    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= m.n_dw) return;
-    const int n_sw = D - w + 1;
-    V2 *out = post + m.post_off + r;
-    const int64_t base = m.series_off + r * w;
-    if constexpr (WT > 0) {
-        V c[WT], U[WT], L[WT];
-#pragma unroll
-        for (int j = 0; j < WT; j++) {
-            c[j] = (V)series[base + j];
-            U[j] = (V)UC[base + j];
-            L[j] = (V)LC[base + j];
-        }
-        for (int b = 0; b < n_sw; b++) {
-            const V4 *qq = sq + (D - WT - b);
-            V eq = (V)0, ec = (V)0;
-#pragma unroll
-            for (int j = 0; j < WT; j++) {
-                const V4 Q = qq[j];
-                lb_term(c[j], Q.y, Q.z, eq);
-                lb_term(Q.x, U[j], L[j], ec);
-            }
-            V2 o;
-            o.x = eq;
-            o.y = ec;
-            out[(int64_t)b * m.n_dw] = o;
-        }
-    } else {
-        for (int b = 0; b < n_sw; b++) {
-            const V4 *qq = sq + (D - w - b);
-            V eq = (V)0, ec = (V)0;
-            for (int j = 0; j < w; j++) {
-                const V4 Q = qq[j];
-                lb_term((V)series[base + j], Q.y, Q.z, eq);
-                lb_term(Q.x, (V)UC[base + j], (V)LC[base + j], ec);
-            }
-            V2 o;
-            o.x = eq;
-            o.y = ec;
-            out[(int64_t)b * m.n_dw] = o;
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// a4: group-level index scan ("LB scan"), Sec. 4.3.2 / Alg. 1 (P:1373-1419,
-// P:4061-4090) with the garbles fixed as reading R5, and Remark 2:
-// every posting element is read once and its running sums serve all item
-// queries.  Thread <-> rightmost disjoint window r (r = -1 .. n_dw-1), CTA <->
-// RT consecutive r.  For each CSG_b (b < w):
-//   S_EQ, S_EC += post[b + j w][r - j]              (j = 0, 1, ...)
-//   m = j + 1; for every IQ_i with m_i(b) = floor((d_i - b)/w) = m:
-//     LB_w(IQ_i, C_t) = max(S_EQ, S_EC),  t = (r - j) w - (d_i - b) % w  (Eq. 4/5)
-// The right end e = t + d_i = (r+1) w + b is the same for every IQ, so the CTA
-// buffers LB_w in shared memory at slot (r - R0) w + b (padded to w+1) and
-// writes each IQ's contiguous t range coalesced.  Slots never written (no full
-// DW, m = 0) hold LB_w = 0 (R6).  The CTA also emits, per IQ, the E candidates
-// with the smallest (LB_w, t) of its tile: the tau set of step a5.
-// Reads all posting lists once (HBM-bound); writes LB_w [mq][i][t].
-// ---------------------------------------------------------------------------
-template <typename S>
-__global__ void group_scan_kernel(const typename Tr<S>::V2 *post, const MQMeta *meta,
-                                  const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
-    using V = typename Tr<S>::V;
-    using V2 = typename Tr<S>::V2;
-    extern __shared__ __align__(16) unsigned char gs_smem[];
-    __shared__ uint64_t s_red[32];
-    const int RT = blockDim.x;
-    const int w = P.w, nl = P.n_len;
-    const int stride = RT * (w + 1);
-    V *tile = reinterpret_cast<V *>(gs_smem);
-    const int mq = blockIdx.y;
-    const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) return;
-    for (int x = threadIdx.x; x < nl * stride; x += RT) tile[x] = (V)0;
-    __syncthreads();
-    const int64_t R0 = (int64_t)blockIdx.x * RT - 1;
-    const int64_t r = R0 + threadIdx.x;
-    const int n_sw = P.D - w + 1;
-    if (r >= 0 && r < m.n_dw) {
-        const V2 *pp = post + m.post_off;
-        for (int b = 0; b < w && b < n_sw; b++) {
-            const int jmax = (n_sw - 1 - b) / w + 1;
-            int ii = 0;
-            while (ii < nl && P.len[ii] - b < w) ii++;  // IQs with m_i(b) = 0 keep LB_w = 0
-            V se = (V)0, sc = (V)0;
-            const int jlim = (int)min((int64_t)jmax, r + 1);
-#pragma unroll 4
-            for (int j = 0; j < jlim; j++) {
-                if (ii >= nl) break;
-                const V2 pv = pp[(int64_t)(b + j * w) * m.n_dw + (r - j)];
-                se += pv.x;
-                sc += pv.y;
-                while (ii < nl && (P.len[ii] - b) / w == j + 1) {
-                    tile[ii * stride + threadIdx.x * (w + 1) + b] = vmax(se, sc);
-                    ii++;
-                }
-            }
-        }
-    }
-    __syncthreads();
-    // write LB_w of the tile, per IQ, coalesced over t
-    const int64_t e0 = (R0 + 1) * w;
-    for (int i = 0; i < nl; i++) {
-        const int d = P.len[i];
-        const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
-        const int64_t tend = min(m.t_hi, m.n - d + 1);
-        V *out = lb + m.seg_off + (int64_t)i * m.n;
-        for (int s = threadIdx.x; s < RT * w; s += RT) {
-            const int64_t t = e0 + s - d;
-            if (t >= tmin && t < tend) out[t] = tile[i * stride + (s / w) * (w + 1) + (s % w)];
-        }
-    }
-    // tau set: E smallest (LB_w, t) of the tile per IQ
-    if (P.E > 0) {
-        for (int i = 0; i < nl; i++) {
-            const int d = P.len[i];
-            const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
-            const int64_t tend = min(m.t_hi, m.n - d + 1);
-            V *row = tile + i * stride + threadIdx.x * (w + 1);
-            int32_t *dst = tauc + (int64_t)(mq * nl + i) * P.LT + (int64_t)blockIdx.x * P.E;
-            for (int e = 0; e < P.E; e++) {
-                uint64_t best = kKeyMax;
-                int bb = -1;
-                for (int b = 0; b < w; b++) {
-                    const int64_t t = e0 + (int64_t)threadIdx.x * w + b - d;
-                    const uint32_t kb = key_bits(row[b]);
-                    if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
-                        uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
-                        if (key < best) {
-                            best = key;
-                            bb = b;
-                        }
-                    }
-                }
-                const uint64_t win = block_min_u64(best, s_red);
-                if (win != kKeyMax && best == win) {
-                    // mark taken (bits 0xFFFFFFFF are neither a valid int32 >= 0 nor a float >= 0)
-                    if constexpr (sizeof(V) == 4) {
-                        uint32_t allones = 0xFFFFFFFFu;
-                        row[bb] = *reinterpret_cast<V *>(&allones);
-                    }
-                }
-                if (threadIdx.x == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
-                __syncthreads();
-            }
-        }
-    }
-}
+#include "lb.cuh"
 
 // ---------------------------------------------------------------------------
 // a5 (second half): tau_i = k-th smallest (DTW, t) key of the verified tau set

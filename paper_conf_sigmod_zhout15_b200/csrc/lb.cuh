@@ -1,0 +1,342 @@
+// lb.cuh -- steps a3/a4 of the Search Step: the SMiLer Index lower bounds.
+// Included by kernels.cuh.
+//
+// Notation (Sec. 4.3): w = omega, n_sw = D - w + 1 sliding windows
+// SW_b = MQ[D-w-b .. D-b) (R19), n_dw = floor(N/w) disjoint windows
+// DW_r = c[rw .. rw+w).  Posting element (window level):
+//   P_EQ[b][r] = sum_j e(c[rw+j]; U(Q), L(Q) at D-w-b+j)
+//   P_EC[b][r] = sum_j e(MQ[D-w-b+j]; U(C), L(C) at rw+j)
+// Group level (Alg. 1, garbles fixed per R5; Thm 4.3 / Eq. 5):
+//   for CSG_b (b < w) and rightmost DW r, the running sums over j of
+//   P[b + j w][r - j] give LB_w(IQ_i, C_t) = max(S_EQ, S_EC) as soon as
+//   j + 1 = m_i(b) = floor((d_i - b)/w), at t = (r - j) w - (d_i - b) % w (Eq. 4).
+// Both the right end e = t + d_i = (r+1) w + b and the tile slot
+// (r - Rb) w + b are independent of i, so one CTA buffers the LB_w of a run
+// of consecutive r in shared memory and writes each IQ's t range coalesced.
+//
+// Three kernels:
+//   window_lb_kernel  (a3) posting lists -> HBM          [two-level path]
+//   group_scan_kernel (a4) HBM posting lists -> LB_w     [two-level path, HBM-bound]
+//   lb_fused_kernel   (a3+a4) one CSG row of posting lists at a time lives in
+//                     shared memory; nothing but LB_w goes to HBM [one-shot path]
+#pragma once
+// (included inside namespace smiler by kernels.cuh)
+
+// emission table: em[j*w + b] = lo | hi << 8, the IQ range [lo, hi) with
+// m_i(b) == j + 1 (contiguous in i because d_i increases).
+__device__ __forceinline__ void build_emit_table(uint16_t *em, int mmax, int w, const QParams &P) {
+    for (int x = threadIdx.x; x < mmax * w; x += blockDim.x) {
+        const int j = x / w, b = x % w;
+        int lo = 0, hi = 0;
+        while (lo < P.n_len && P.len[lo] - b < (j + 1) * w) lo++;
+        hi = lo;
+        while (hi < P.n_len && P.len[hi] - b < (j + 2) * w) hi++;
+        em[x] = (uint16_t)(lo | (hi << 8));
+    }
+}
+
+// Write a CTA's LB_w tile (slot s <-> e = e0 + s, padded to w+1 per row) to
+// lb[mq][i][t] and emit the tau set (E smallest (LB_w, t) per IQ) of the tile.
+template <typename V, int W>
+__device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, const QParams &P, V *lb,
+                                 int32_t *tauc, int mq, uint64_t *s_red) {
+    const int w = W > 0 ? W : P.w;
+    const int nl = P.n_len;
+    const int stride = RT * (w + 1);
+    const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
+    for (int i = 0; i < nl; i++) {
+        const int d = P.len[i];
+        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        V *out = lb + m.seg_off + (int64_t)i * m.n;
+        const V *row = tile + i * stride;
+        for (int s = threadIdx.x; s < RT * w; s += blockDim.x) {
+            const int64_t t = e0 + s - d;
+            if (t >= tmin && t < tend) out[t] = row[(s / w) * (w + 1) + (s % w)];
+        }
+    }
+    if (P.E <= 0) return;
+    for (int i = 0; i < nl; i++) {
+        const int d = P.len[i];
+        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        V *row = tile + i * stride;
+        int32_t *dst = tauc + (int64_t)(mq * nl + i) * P.LT + (int64_t)blockIdx.x * P.E;
+        for (int e = 0; e < P.E; e++) {
+            uint64_t best = kKeyMax;
+            int bs = -1;
+            for (int s = threadIdx.x; s < RT * w; s += blockDim.x) {
+                const int64_t t = e0 + s - d;
+                const int slot = (s / w) * (w + 1) + (s % w);
+                const uint32_t kb = key_bits(row[slot]);
+                if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
+                    const uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
+                    if (key < best) {
+                        best = key;
+                        bs = slot;
+                    }
+                }
+            }
+            const uint64_t win = block_min_u64(best, s_red);
+            if (win != kKeyMax && best == win) {  // unique: keys carry t
+                uint32_t allones = 0xFFFFFFFFu;   // "taken": not a valid LB >= 0
+                row[bs] = *reinterpret_cast<V *>(&allones);
+            }
+            if (threadIdx.x == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+            __syncthreads();
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3: window-level posting lists.  Thread <-> DW r (its w points and envelope
+// in registers).  The b loop runs in chunks of BC sliding windows; consecutive
+// SWs overlap in w-1 positions, so one chunk needs w+BC-1 MQ positions
+// {q, U(Q), L(Q)} loaded once into registers (no shared-memory load per term).
+// 8 ALU ops per (b, r, j) term pair.  Output post[mq][b][r] = {P_EQ, P_EC}.
+// ---------------------------------------------------------------------------
+template <typename S, int W>
+__global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
+                                                       const MQMeta *meta,
+                                                       const typename Tr<S>::V4 *qtab, int D,
+                                                       int w_rt, typename Tr<S>::V2 *post) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    using V4 = typename Tr<S>::V4;
+    extern __shared__ __align__(16) unsigned char wl_smem[];
+    V4 *sq = reinterpret_cast<V4 *>(wl_smem);
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int64_t)blockIdx.x * blockDim.x >= m.n_dw) return;
+    for (int p = threadIdx.x; p < D; p += blockDim.x) sq[p] = qtab[(int64_t)mq * D + p];
+    __syncthreads();
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= m.n_dw) return;
+    V2 *out = post + m.post_off + r;
+    if constexpr (W > 0) {
+        constexpr int BC = W < 8 ? W : 8;
+        const int n_sw = D - W + 1;
+        const int64_t base = m.series_off + r * W;
+        V c[W], U[W], L[W];
+#pragma unroll
+        for (int j = 0; j < W; j++) {
+            c[j] = (V)series[base + j];
+            U[j] = (V)UC[base + j];
+            L[j] = (V)LC[base + j];
+        }
+        for (int b0 = 0; b0 < n_sw; b0 += BC) {
+            // positions D-W-b0-(BC-1) .. D-b0-1 cover SW_{b0} .. SW_{b0+BC-1}
+            const int pb = D - W - b0 - (BC - 1);
+            V4 win[W + BC - 1];
+#pragma unroll
+            for (int k = 0; k < W + BC - 1; k++) win[k] = sq[max(pb + k, 0)];
+#pragma unroll
+            for (int bb = 0; bb < BC; bb++) {
+                const int b = b0 + bb;
+                if (b < n_sw) {
+                    V eq = (V)0, ec = (V)0;
+#pragma unroll
+                    for (int j = 0; j < W; j++) {
+                        const V4 Q = win[BC - 1 - bb + j];
+                        lb_term(c[j], Q.y, Q.z, eq);
+                        lb_term(Q.x, U[j], L[j], ec);
+                    }
+                    V2 o;
+                    o.x = eq;
+                    o.y = ec;
+                    out[(int64_t)b * m.n_dw] = o;
+                }
+            }
+        }
+    } else {
+        const int w = w_rt;
+        const int n_sw = D - w + 1;
+        const int64_t base = m.series_off + r * w;
+        for (int b = 0; b < n_sw; b++) {
+            const V4 *qq = sq + (D - w - b);
+            V eq = (V)0, ec = (V)0;
+            for (int j = 0; j < w; j++) {
+                const V4 Q = qq[j];
+                lb_term((V)series[base + j], Q.y, Q.z, eq);
+                lb_term(Q.x, (V)UC[base + j], (V)LC[base + j], ec);
+            }
+            V2 o;
+            o.x = eq;
+            o.y = ec;
+            out[(int64_t)b * m.n_dw] = o;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a4: group-level scan over the posting lists in HBM (HBM-bound).  Thread <->
+// rightmost DW r (r = Rb .. Rb+RT-1, Rb = blockIdx.x*RT - 1).  For each CSG_b,
+// posting pairs are fetched 8 at a time ahead of the running sums (8 loads of
+// 8 B in flight per thread); emission follows the per-CTA table em.
+// smem: em [mmax*w] u16 | tile [n_len][RT*(w+1)] V.
+// ---------------------------------------------------------------------------
+template <typename S, int W>
+__global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V2 *post,
+                                                        const MQMeta *meta, const QParams P,
+                                                        typename Tr<S>::V *lb, int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    extern __shared__ __align__(16) unsigned char gs_smem[];
+    __shared__ uint64_t s_red[32];
+    const int w = W > 0 ? W : P.w;
+    const int RT = blockDim.x;
+    const int nl = P.n_len;
+    const int n_sw = P.D - w + 1;
+    const int mmax = P.D / w;
+    const int stride = RT * (w + 1);
+    uint16_t *em = reinterpret_cast<uint16_t *>(gs_smem);
+    V *tile = reinterpret_cast<V *>(gs_smem + ((mmax * w * 2 + 15) & ~15));
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) return;
+    build_emit_table(em, mmax, w, P);
+    for (int x = threadIdx.x; x < nl * stride; x += RT) tile[x] = (V)0;
+    __syncthreads();
+    const int64_t Rb = (int64_t)blockIdx.x * RT - 1;
+    const int64_t r = Rb + threadIdx.x;
+    if (r >= 0 && r < m.n_dw) {
+        const V2 *pp = post + m.post_off + r;
+        V *trow = tile + threadIdx.x * (w + 1);
+        for (int b = 0; b < w && b < n_sw; b++) {
+            const int jmax = (n_sw - 1 - b) / w + 1;
+            const int jlim = (int)min((int64_t)jmax, r + 1);
+            V se = (V)0, sc = (V)0;
+            for (int j0 = 0; j0 < jlim; j0 += 8) {
+                V2 pv[8];
+#pragma unroll
+                for (int u = 0; u < 8; u++) {
+                    const int j = j0 + u;
+                    if (j < jlim) pv[u] = pp[(int64_t)(b + j * w) * m.n_dw - j];
+                }
+#pragma unroll
+                for (int u = 0; u < 8; u++) {
+                    const int j = j0 + u;
+                    if (j < jlim) {
+                        se += pv[u].x;
+                        sc += pv[u].y;
+                        const int rng = em[j * w + b];
+                        const V lbv = vmax(se, sc);
+                        for (int i = rng & 255; i < (rng >> 8); i++) trow[i * stride + b] = lbv;
+                    }
+                }
+            }
+        }
+    }
+    __syncthreads();
+    lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * w, m, P, lb, tauc, mq, s_red);
+}
+
+// ---------------------------------------------------------------------------
+// a3+a4 fused (one-shot batches).  NT threads own NT consecutive DWs r' =
+// Rb - HALO + x (HALO = mmax - 1 DWs of left halo); the RT = NT - HALO right
+// threads own the tile's rightmost DWs r.  For each CSG row j:
+//   phase A: every thread computes P[b + j w][r'] for all b < w into smem Ps
+//            (sliding MQ window in registers, as in a3);
+//   phase B: tile threads add Ps[b][x - j] = P[b + j w][r - j] to S_b and
+//            emit LB_w for the IQs with m_i(b) = j + 1.
+// The ALU work equals a3's plus HALO/NT; HBM traffic is only the series
+// (read once) and LB_w.  smem: em | sq [D] V4 | Ps [w][NT] V2 | tile.
+// ---------------------------------------------------------------------------
+constexpr int kFusedThreads = 256;
+
+template <typename S, int W>
+__global__ void __launch_bounds__(kFusedThreads) lb_fused_kernel(const S *series, const S *UC, const S *LC,
+                                                                const MQMeta *meta,
+                                                                const typename Tr<S>::V4 *qtab,
+                                                                const QParams P, typename Tr<S>::V *lb,
+                                                                int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    using V4 = typename Tr<S>::V4;
+    constexpr int NT = kFusedThreads;
+    constexpr int BC = W < 8 ? W : 8;
+    extern __shared__ __align__(16) unsigned char fz_smem[];
+    __shared__ uint64_t s_red[32];
+    const int D = P.D;
+    const int nl = P.n_len;
+    const int n_sw = D - W + 1;
+    const int mmax = D / W;
+    const int HALO = mmax - 1;
+    const int RT = NT - HALO;
+    const int stride = RT * (W + 1);
+    uint16_t *em = reinterpret_cast<uint16_t *>(fz_smem);
+    V4 *sq = reinterpret_cast<V4 *>(fz_smem + ((mmax * W * 2 + 15) & ~15));
+    V2 *Ps = reinterpret_cast<V2 *>(sq + D);
+    V *tile = reinterpret_cast<V *>(Ps + W * NT);
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) return;
+    build_emit_table(em, mmax, W, P);
+    for (int p = threadIdx.x; p < D; p += NT) sq[p] = qtab[(int64_t)mq * D + p];
+    for (int x = threadIdx.x; x < nl * stride; x += NT) tile[x] = (V)0;
+    const int x = threadIdx.x;
+    const int64_t Rb = (int64_t)blockIdx.x * RT - 1;
+    const int64_t rp = Rb - HALO + x;  // this thread's DW
+    V c[W], U[W], L[W];
+    {
+        const bool ok = rp >= 0 && rp < m.n_dw;
+        const int64_t base = m.series_off + (ok ? rp : 0) * W;
+#pragma unroll
+        for (int j = 0; j < W; j++) {
+            c[j] = ok ? (V)series[base + j] : (V)0;
+            U[j] = ok ? (V)UC[base + j] : (V)0;
+            L[j] = ok ? (V)LC[base + j] : (V)0;
+        }
+    }
+    V se[W], sc[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
+    const bool is_tile = x >= HALO;
+    V *trow = tile + (x - HALO) * (W + 1);
+    __syncthreads();
+    for (int j = 0; j < mmax; j++) {
+        // phase A: SW_{b + jW}, b in [0, W): positions D-W-b-jW .. D-b-jW-1
+#pragma unroll
+        for (int b0 = 0; b0 < W; b0 += BC) {
+            const int pb = D - W - j * W - b0 - (BC - 1);
+            V4 win[W + BC - 1];
+#pragma unroll
+            for (int k = 0; k < W + BC - 1; k++) win[k] = sq[max(pb + k, 0)];
+#pragma unroll
+            for (int bb = 0; bb < BC; bb++) {
+                const int b = b0 + bb;
+                if (b + j * W < n_sw) {
+                    V eq = (V)0, ec = (V)0;
+#pragma unroll
+                    for (int jj = 0; jj < W; jj++) {
+                        const V4 Q = win[BC - 1 - bb + jj];
+                        lb_term(c[jj], Q.y, Q.z, eq);
+                        lb_term(Q.x, U[jj], L[jj], ec);
+                    }
+                    V2 o;
+                    o.x = eq;
+                    o.y = ec;
+                    Ps[b * NT + x] = o;
+                }
+            }
+        }
+        __syncthreads();
+        // phase B: running sums along the CSG diagonals + emission
+        if (is_tile) {
+#pragma unroll
+            for (int b = 0; b < W; b++) {
+                if (b + j * W < n_sw) {
+                    const V2 pv = Ps[b * NT + x - j];
+                    se[b] += pv.x;
+                    sc[b] += pv.y;
+                    const int rng = em[j * W + b];
+                    if (rng) {
+                        const V lbv = vmax(se[b], sc[b]);
+                        for (int i = rng & 255; i < (rng >> 8); i++) trow[i * stride + b] = lbv;
+                    }
+                }
+            }
+        }
+        __syncthreads();
+    }
+    lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * W, m, P, lb, tauc, mq, s_red);
+}
+

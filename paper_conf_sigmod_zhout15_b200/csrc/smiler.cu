@@ -366,7 +366,10 @@ extern "C" int32_t smiler_abi_version(void) { return SMILER_ABI_VERSION; }
 struct Plan {
     int D, n_len, k, w, rho_env;
     std::vector<int> len, rho;
-    int RT;
+    int RT;          // group-scan CTA width (two-level path)
+    bool fused;      // a3+a4 fused kernel
+    int RTf;         // fused: tile DWs per CTA
+    size_t smem_gs, smem_fz;
 };
 
 static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len, int k, Plan &pl) {
@@ -394,8 +397,19 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
                         kMaxRhoFast);
     }
     const size_t vs = 4;
-    pl.RT = 128;
-    while (pl.RT > 32 && (size_t)n_len * pl.RT * (pl.w + 1) * vs > 96 * 1024) pl.RT >>= 1;
+    const int mmax = pl.D / pl.w;
+    const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
+    pl.RT = 256;
+    while (pl.RT > 32 && em + (size_t)n_len * pl.RT * (pl.w + 1) * vs > 160 * 1024) pl.RT >>= 1;
+    pl.smem_gs = em + (size_t)n_len * pl.RT * (pl.w + 1) * vs;
+    pl.fused = false;
+    if (pl.w == 4 || pl.w == 8 || pl.w == 16) {
+        const int halo = mmax - 1;
+        pl.RTf = kFusedThreads - halo;
+        pl.smem_fz = em + (size_t)pl.D * 16 + (size_t)pl.w * kFusedThreads * 8 +
+                     (size_t)n_len * pl.RTf * (pl.w + 1) * vs;
+        pl.fused = halo <= kFusedThreads / 4 && pl.smem_fz <= 200 * 1024;
+    }
     return SMILER_OK;
 }
 
@@ -472,6 +486,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     else memcpy(lens_h.data(), lengths_in, 4 * n_len);
     Plan pl;
     TRY(validate_query(idx, lens_h.data(), n_len, lb_only ? 1 : k, pl));
+    if (o.two_level || (lb_only && post_out)) pl.fused = false;
     const int D = pl.D, w = pl.w, nl = pl.n_len;
     std::vector<int32_t> qsens(n_mq, 0);
     if (query_sensor_in) {
@@ -513,7 +528,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     auto mq_bytes = [&](int j) -> size_t {
         const SensorInfo &si = idx->sensors[qsens[j]];
         const size_t ndw = (size_t)(si.n / w);
-        return (size_t)n_sw * ndw * 8 + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
+        return (pl.fused ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
     };
     size_t budget = (size_t)24 << 30;
     {
@@ -563,7 +578,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             m.n_dw = si.n / w;
             m.post_off = post_tot;
             m.seg_off = seg_tot;
-            m.nblk = (int)(si.n / ((int64_t)pl.RT * w) + 1);
+            m.nblk = (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
             m.sensor = qsens[c0 + j];
             post_tot += (int64_t)n_sw * m.n_dw;
             seg_tot += (int64_t)nl * si.n;
@@ -625,8 +640,26 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         CHECK_LAUNCH();
         launches++;
         TRY(tm.mark(1));
-        // ---- a3 ----------------------------------------------------------
-        {
+        if (pl.fused) {
+            // ---- a3 + a4 fused ------------------------------------------------
+            dim3 grid((unsigned)nblk_max, (unsigned)B);
+            auto go = [&](auto kern) {
+                if (pl.smem_fz > 48 * 1024)
+                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_fz);
+                kern<<<grid, kFusedThreads, pl.smem_fz, idx->stream>>>(
+                    (const S *)idx->d_series, (const S *)dUC, (const S *)dLC, d_meta, idx->qtab.as<V4>(), P,
+                    idx->lb.as<V>(), idx->tauc.as<int32_t>());
+            };
+            switch (w) {
+                case 4: go(lb_fused_kernel<S, 4>); break;
+                case 8: go(lb_fused_kernel<S, 8>); break;
+                default: go(lb_fused_kernel<S, 16>); break;
+            }
+            CHECK_LAUNCH();
+            launches++;
+            TRY(tm.mark(2));
+        } else {
+            // ---- a3 ----------------------------------------------------------
             int64_t ndw_max = 0;
             for (auto &m : meta) ndw_max = std::max(ndw_max, m.n_dw);
             if (ndw_max > 0) {
@@ -649,17 +682,23 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 CHECK_LAUNCH();
                 launches++;
             }
-        }
-        post_bytes += post_tot * 8;
-        TRY(tm.mark(2));
-        // ---- a4 ----------------------------------------------------------
-        {
+            post_bytes += post_tot * 8;
+            TRY(tm.mark(2));
+            // ---- a4 ----------------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
-            size_t smem = (size_t)nl * pl.RT * (w + 1) * sizeof(V);
-            if (smem > 48 * 1024)
-                cudaFuncSetAttribute(group_scan_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            group_scan_kernel<S><<<grid, pl.RT, smem, idx->stream>>>(idx->post.as<V2>(), d_meta, P,
-                                                                     idx->lb.as<V>(), idx->tauc.as<int32_t>());
+            auto go4 = [&](auto kern) {
+                if (pl.smem_gs > 48 * 1024)
+                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_gs);
+                kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(idx->post.as<V2>(), d_meta, P, idx->lb.as<V>(),
+                                                               idx->tauc.as<int32_t>());
+            };
+            switch (w) {
+                case 4: go4(group_scan_kernel<S, 4>); break;
+                case 8: go4(group_scan_kernel<S, 8>); break;
+                case 16: go4(group_scan_kernel<S, 16>); break;
+                case 32: go4(group_scan_kernel<S, 32>); break;
+                default: go4(group_scan_kernel<S, 0>); break;
+            }
             CHECK_LAUNCH();
             launches++;
         }

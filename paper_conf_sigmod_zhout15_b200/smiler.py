@@ -45,7 +45,8 @@ class KnnStats(ctypes.Structure):
 
 class KnnOpts(ctypes.Structure):
     _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
-                ("mq_chunk", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
+                ("mq_chunk", ctypes.c_int32), ("two_level", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 4)]
 
 
 _lib = None
@@ -215,12 +216,12 @@ class Index:
         return cls(slice_, _handle=h)
 
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
-            no_prune: bool = False, timing: bool = False, mq_chunk: int = 0):
+            no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False):
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
-        op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk)
+        op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level))
         smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()
@@ -233,10 +234,12 @@ class Index:
         smiler_index_envelope(self.handle, sensor, rho, U, L)
         return U, L
 
-    def lower_bounds(self, queries, lengths, n: int, window: int, query_sensor=None):
+    def lower_bounds(self, queries, lengths, n: int, window: int, query_sensor=None, postings: bool = True):
+        """postings=True: two-level path (posting lists materialised and returned);
+        postings=False: the fused path (returns post=None)."""
         n_mq, D = queries.shape
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32
-        post = np.empty((n_mq, D - window + 1, n // window, 2), vt)
+        post = np.empty((n_mq, D - window + 1, n // window, 2), vt) if postings else None
         lbw = np.empty((n_mq, len(lengths), n), vt)
         smiler_lower_bounds(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, post, lbw)
         return post, lbw

@@ -100,17 +100,18 @@ def test_postings_and_lbw(pkg, orc, dtype, cfg, n, lengths, window, band):
     rhos = wl.rhos()
     with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
         post, lbw = idx.lower_bounds(wl.queries, wl.lengths, n, window)
+        _, lbw_fused = idx.lower_bounds(wl.queries, wl.lengths, n, window, postings=False)
     for j in range(wl.n_mq):
         res, (UC, LC, UQ, LQ, rho_env) = orc.mq_lower_bounds(wl.series, wl.queries[j], wl.lengths, rhos,
                                                              window)
         PE, PC = orc.postings(wl.series, UC, LC, wl.queries[j], UQ, LQ, window)
         for i, d in enumerate(wl.lengths):
-            got = lbw[j, i, :n - d + 1]
             exp = res[i]["w"]
-            if dtype == "i16":
-                np.testing.assert_array_equal(got.astype(np.int64), exp)
-            else:
-                np.testing.assert_allclose(got, exp, rtol=2e-5, atol=1e-6)
+            for got in (lbw[j, i, :n - d + 1], lbw_fused[j, i, :n - d + 1]):
+                if dtype == "i16":
+                    np.testing.assert_array_equal(got.astype(np.int64), exp)
+                else:
+                    np.testing.assert_allclose(got, exp, rtol=2e-5, atol=1e-6)
         if dtype == "i16":
             np.testing.assert_array_equal(post[j, :, :, 0].astype(np.int64), PE)
             np.testing.assert_array_equal(post[j, :, :, 1].astype(np.int64), PC)
@@ -172,16 +173,18 @@ def test_c1_full(pkg, orc, dtype):
     check_workload(pkg, orc, wl)
 
 
+@pytest.mark.parametrize("two_level", [False, True])
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
-def test_c2_reduced(pkg, orc, dtype):
+def test_c2_reduced(pkg, orc, dtype, two_level):
     wl = synth.make_workload("C2", dtype, n=20011, mq_per_sensor=4)
-    check_workload(pkg, orc, wl)
+    check_workload(pkg, orc, wl, two_level=two_level)
 
 
+@pytest.mark.parametrize("two_level", [False, True])
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
-def test_c3_reduced(pkg, orc, dtype):
+def test_c3_reduced(pkg, orc, dtype, two_level):
     wl = synth.make_workload("C3", dtype, n=15007, n_sensors=6)
-    check_workload(pkg, orc, wl)
+    check_workload(pkg, orc, wl, two_level=two_level)
 
 
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
@@ -201,8 +204,10 @@ def test_pruned_equals_no_prune(pkg, dtype):
     wl = synth.make_workload("C5", dtype, n=30011, n_sensors=3, mq_per_sensor=3)
     a = gpu_knn(pkg, wl)
     b = gpu_knn(pkg, wl, no_prune=True)
-    np.testing.assert_array_equal(a[0], b[0])
-    np.testing.assert_array_equal(a[1], b[1])
+    c = gpu_knn(pkg, wl, two_level=True)
+    for x in (b, c):
+        np.testing.assert_array_equal(a[0], x[0])
+        np.testing.assert_array_equal(a[1], x[1])
 
 
 # ---------------------------------------------------------------------------
