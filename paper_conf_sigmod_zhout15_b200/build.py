@@ -20,7 +20,7 @@ LIB = os.path.join(HERE, "libsmiler.so")
 BUILD = os.path.join(HERE, "_build")
 ALU_BENCH = os.path.join(BUILD, "alu_bench")
 SOURCES = ["smiler.cu", "dtw.cu"]
-HEADERS = ["internal.h", "kernels.cuh", os.path.join("..", "..", "include", "smiler.h")]
+HEADERS = ["internal.h", "kernels.cuh", "lb.cuh", os.path.join("..", "..", "include", "smiler.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",

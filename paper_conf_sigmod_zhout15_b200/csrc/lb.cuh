@@ -37,6 +37,7 @@ __device__ __forceinline__ void build_emit_table(uint16_t *em, int mmax, int w, 
 
 // Write a CTA's LB_w tile (slot s <-> e = e0 + s, padded to w+1 per row) to
 // lb[mq][i][t] and emit the tau set (E smallest (LB_w, t) per IQ) of the tile.
+// The first selection round is folded into the write-out pass.
 template <typename V, int W>
 __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, const QParams &P, V *lb,
                                  int32_t *tauc, int mq, uint64_t *s_red) {
@@ -48,30 +49,38 @@ __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, c
         const int d = P.len[i];
         const int64_t tend = min(m.t_hi, m.n - d + 1);
         V *out = lb + m.seg_off + (int64_t)i * m.n;
-        const V *row = tile + i * stride;
+        V *row = tile + i * stride;
+        uint64_t best = kKeyMax;
+        int bs = -1;
         for (int s = threadIdx.x; s < RT * w; s += blockDim.x) {
             const int64_t t = e0 + s - d;
-            if (t >= tmin && t < tend) out[t] = row[(s / w) * (w + 1) + (s % w)];
+            const int slot = (s / w) * (w + 1) + (s % w);
+            if (t >= tmin && t < tend) {
+                const V v = row[slot];
+                out[t] = v;
+                const uint64_t key = ((uint64_t)key_bits(v) << 32) | (uint32_t)t;
+                if (key < best) {
+                    best = key;
+                    bs = slot;
+                }
+            }
         }
-    }
-    if (P.E <= 0) return;
-    for (int i = 0; i < nl; i++) {
-        const int d = P.len[i];
-        const int64_t tend = min(m.t_hi, m.n - d + 1);
-        V *row = tile + i * stride;
+        if (P.E <= 0) continue;
         int32_t *dst = tauc + (int64_t)(mq * nl + i) * P.LT + (int64_t)blockIdx.x * P.E;
         for (int e = 0; e < P.E; e++) {
-            uint64_t best = kKeyMax;
-            int bs = -1;
-            for (int s = threadIdx.x; s < RT * w; s += blockDim.x) {
-                const int64_t t = e0 + s - d;
-                const int slot = (s / w) * (w + 1) + (s % w);
-                const uint32_t kb = key_bits(row[slot]);
-                if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
-                    const uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
-                    if (key < best) {
-                        best = key;
-                        bs = slot;
+            if (e > 0) {  // later rounds rescan the thread's slots
+                best = kKeyMax;
+                bs = -1;
+                for (int s = threadIdx.x; s < RT * w; s += blockDim.x) {
+                    const int64_t t = e0 + s - d;
+                    const int slot = (s / w) * (w + 1) + (s % w);
+                    const uint32_t kb = key_bits(row[slot]);
+                    if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
+                        const uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
+                        if (key < best) {
+                            best = key;
+                            bs = slot;
+                        }
                     }
                 }
             }
@@ -82,6 +91,37 @@ __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, c
             }
             if (threadIdx.x == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
             __syncthreads();
+        }
+    }
+}
+
+// One sliding-window chunk of posting elements: SW_{b0+bb} (bb < BC) against
+// the thread's DW (c, U, L).  Window registers hold MQ positions
+// pb .. pb + W + BC - 2 (pb = D - W - b0 - (BC-1)): q, U(Q), L(Q).
+// CHECK: per-bb validity test (only for the last chunk of a CSG row).
+template <typename V, int W, int BC, bool CHECK, typename F>
+__device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], const V (&L)[W],
+                                              const V *qq, const V *uq, const V *lq, int pb, int nvalid,
+                                              F &&store) {
+    V wq[W + BC - 1], wu[W + BC - 1], wl[W + BC - 1];
+#pragma unroll
+    for (int k = 0; k < W + BC - 1; k++) {
+        const int p = max(pb + k, 0);
+        wq[k] = qq[p];
+        wu[k] = uq[p];
+        wl[k] = lq[p];
+    }
+#pragma unroll
+    for (int bb = 0; bb < BC; bb++) {
+        if (!CHECK || bb < nvalid) {
+            V eq = (V)0, ec = (V)0;
+#pragma unroll
+            for (int j = 0; j < W; j++) {
+                const int k = BC - 1 - bb + j;
+                lb_term(c[j], wu[k], wl[k], eq);
+                lb_term(wq[k], U[j], L[j], ec);
+            }
+            store(bb, eq, ec);
         }
     }
 }
@@ -100,13 +140,19 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
                                                        int w_rt, typename Tr<S>::V2 *post) {
     using V = typename Tr<S>::V;
     using V2 = typename Tr<S>::V2;
-    using V4 = typename Tr<S>::V4;
     extern __shared__ __align__(16) unsigned char wl_smem[];
-    V4 *sq = reinterpret_cast<V4 *>(wl_smem);
+    V *sqq = reinterpret_cast<V *>(wl_smem);
+    V *squ = sqq + D;
+    V *sql = squ + D;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
     if ((int64_t)blockIdx.x * blockDim.x >= m.n_dw) return;
-    for (int p = threadIdx.x; p < D; p += blockDim.x) sq[p] = qtab[(int64_t)mq * D + p];
+    for (int p = threadIdx.x; p < D; p += blockDim.x) {
+        const typename Tr<S>::V4 e = qtab[(int64_t)mq * D + p];
+        sqq[p] = e.x;
+        squ[p] = e.y;
+        sql[p] = e.z;
+    }
     __syncthreads();
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= m.n_dw) return;
@@ -115,6 +161,7 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
         constexpr int BC = W < 8 ? W : 8;
         const int n_sw = D - W + 1;
         const int64_t base = m.series_off + r * W;
+        const int64_t ndw = m.n_dw;
         V c[W], U[W], L[W];
 #pragma unroll
         for (int j = 0; j < W; j++) {
@@ -122,41 +169,37 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
             U[j] = (V)UC[base + j];
             L[j] = (V)LC[base + j];
         }
-        for (int b0 = 0; b0 < n_sw; b0 += BC) {
-            // positions D-W-b0-(BC-1) .. D-b0-1 cover SW_{b0} .. SW_{b0+BC-1}
-            const int pb = D - W - b0 - (BC - 1);
-            V4 win[W + BC - 1];
-#pragma unroll
-            for (int k = 0; k < W + BC - 1; k++) win[k] = sq[max(pb + k, 0)];
-#pragma unroll
-            for (int bb = 0; bb < BC; bb++) {
-                const int b = b0 + bb;
-                if (b < n_sw) {
-                    V eq = (V)0, ec = (V)0;
-#pragma unroll
-                    for (int j = 0; j < W; j++) {
-                        const V4 Q = win[BC - 1 - bb + j];
-                        lb_term(c[j], Q.y, Q.z, eq);
-                        lb_term(Q.x, U[j], L[j], ec);
-                    }
-                    V2 o;
-                    o.x = eq;
-                    o.y = ec;
-                    out[(int64_t)b * m.n_dw] = o;
-                }
-            }
+        int b0 = 0;
+        for (; b0 + BC <= n_sw; b0 += BC) {
+            V2 *o = out + (int64_t)b0 * ndw;
+            posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                           [&](int bb, V eq, V ec) {
+                                               V2 v;
+                                               v.x = eq;
+                                               v.y = ec;
+                                               o[bb * ndw] = v;
+                                           });
+        }
+        if (b0 < n_sw) {
+            V2 *o = out + (int64_t)b0 * ndw;
+            posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
+                                          [&](int bb, V eq, V ec) {
+                                              V2 v;
+                                              v.x = eq;
+                                              v.y = ec;
+                                              o[bb * ndw] = v;
+                                          });
         }
     } else {
         const int w = w_rt;
         const int n_sw = D - w + 1;
         const int64_t base = m.series_off + r * w;
         for (int b = 0; b < n_sw; b++) {
-            const V4 *qq = sq + (D - w - b);
+            const int p0 = D - w - b;
             V eq = (V)0, ec = (V)0;
             for (int j = 0; j < w; j++) {
-                const V4 Q = qq[j];
-                lb_term((V)series[base + j], Q.y, Q.z, eq);
-                lb_term(Q.x, (V)UC[base + j], (V)LC[base + j], ec);
+                lb_term((V)series[base + j], squ[p0 + j], sql[p0 + j], eq);
+                lb_term(sqq[p0 + j], (V)UC[base + j], (V)LC[base + j], ec);
             }
             V2 o;
             o.x = eq;
@@ -243,14 +286,13 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
 constexpr int kFusedThreads = 256;
 
 template <typename S, int W>
-__global__ void __launch_bounds__(kFusedThreads) lb_fused_kernel(const S *series, const S *UC, const S *LC,
+__global__ void __launch_bounds__(kFusedThreads, (W <= 8 ? 3 : 1)) lb_fused_kernel(const S *series, const S *UC, const S *LC,
                                                                 const MQMeta *meta,
                                                                 const typename Tr<S>::V4 *qtab,
                                                                 const QParams P, typename Tr<S>::V *lb,
                                                                 int32_t *tauc) {
     using V = typename Tr<S>::V;
     using V2 = typename Tr<S>::V2;
-    using V4 = typename Tr<S>::V4;
     constexpr int NT = kFusedThreads;
     constexpr int BC = W < 8 ? W : 8;
     extern __shared__ __align__(16) unsigned char fz_smem[];
@@ -263,14 +305,21 @@ __global__ void __launch_bounds__(kFusedThreads) lb_fused_kernel(const S *series
     const int RT = NT - HALO;
     const int stride = RT * (W + 1);
     uint16_t *em = reinterpret_cast<uint16_t *>(fz_smem);
-    V4 *sq = reinterpret_cast<V4 *>(fz_smem + ((mmax * W * 2 + 15) & ~15));
-    V2 *Ps = reinterpret_cast<V2 *>(sq + D);
-    V *tile = reinterpret_cast<V *>(Ps + W * NT);
+    V2 *Ps = reinterpret_cast<V2 *>(fz_smem + ((mmax * W * 2 + 15) & ~15));  // [2][W][NT]
+    V *sqq = reinterpret_cast<V *>(Ps + 2 * W * NT);
+    V *squ = sqq + D;
+    V *sql = squ + D;
+    V *tile = sql + D;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
     if ((int)blockIdx.x >= m.nblk) return;
     build_emit_table(em, mmax, W, P);
-    for (int p = threadIdx.x; p < D; p += NT) sq[p] = qtab[(int64_t)mq * D + p];
+    for (int p = threadIdx.x; p < D; p += NT) {
+        const typename Tr<S>::V4 e = qtab[(int64_t)mq * D + p];
+        sqq[p] = e.x;
+        squ[p] = e.y;
+        sql[p] = e.z;
+    }
     for (int x = threadIdx.x; x < nl * stride; x += NT) tile[x] = (V)0;
     const int x = threadIdx.x;
     const int64_t Rb = (int64_t)blockIdx.x * RT - 1;
@@ -293,50 +342,43 @@ __global__ void __launch_bounds__(kFusedThreads) lb_fused_kernel(const S *series
     V *trow = tile + (x - HALO) * (W + 1);
     __syncthreads();
     for (int j = 0; j < mmax; j++) {
-        // phase A: SW_{b + jW}, b in [0, W): positions D-W-b-jW .. D-b-jW-1
+        V2 *pb_ = Ps + (j & 1) * W * NT;
+        const int nrow = min(W, n_sw - j * W);  // valid SWs b + jW in this CSG row (>= 1)
+        // phase A: P[b + jW][r'] for b < nrow
 #pragma unroll
         for (int b0 = 0; b0 < W; b0 += BC) {
+            const int nv = nrow - b0;
+            auto store = [&](int bb, V eq, V ec) {
+                V2 v;
+                v.x = eq;
+                v.y = ec;
+                pb_[(b0 + bb) * NT + x] = v;
+            };
             const int pb = D - W - j * W - b0 - (BC - 1);
-            V4 win[W + BC - 1];
-#pragma unroll
-            for (int k = 0; k < W + BC - 1; k++) win[k] = sq[max(pb + k, 0)];
-#pragma unroll
-            for (int bb = 0; bb < BC; bb++) {
-                const int b = b0 + bb;
-                if (b + j * W < n_sw) {
-                    V eq = (V)0, ec = (V)0;
-#pragma unroll
-                    for (int jj = 0; jj < W; jj++) {
-                        const V4 Q = win[BC - 1 - bb + jj];
-                        lb_term(c[jj], Q.y, Q.z, eq);
-                        lb_term(Q.x, U[jj], L[jj], ec);
-                    }
-                    V2 o;
-                    o.x = eq;
-                    o.y = ec;
-                    Ps[b * NT + x] = o;
-                }
-            }
+            if (nv >= BC)
+                posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, pb, BC, store);
+            else if (nv > 0)
+                posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, pb, nv, store);
         }
         __syncthreads();
         // phase B: running sums along the CSG diagonals + emission
         if (is_tile) {
 #pragma unroll
             for (int b = 0; b < W; b++) {
-                if (b + j * W < n_sw) {
-                    const V2 pv = Ps[b * NT + x - j];
+                if (b < nrow) {
+                    const V2 pv = pb_[b * NT + x - j];
                     se[b] += pv.x;
                     sc[b] += pv.y;
                     const int rng = em[j * W + b];
-                    if (rng) {
+                    if ((rng & 255) != (rng >> 8)) {
                         const V lbv = vmax(se[b], sc[b]);
                         for (int i = rng & 255; i < (rng >> 8); i++) trow[i * stride + b] = lbv;
                     }
                 }
             }
         }
-        __syncthreads();
+        // no second barrier: the next row writes the other Ps buffer
     }
+    __syncthreads();
     lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * W, m, P, lb, tauc, mq, s_red);
 }
-

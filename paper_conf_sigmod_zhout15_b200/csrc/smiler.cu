@@ -124,7 +124,42 @@ struct smiler_index {
     DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, tauk, taukey, thr, scount, fcount,
         taskoff, out_ids, out_d, tmp;
     std::vector<cudaEvent_t> events;
+    size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
+    // pinned staging ring for per-chunk metadata (async H2D without host sync)
+    MQMeta *h_meta[2] = {nullptr, nullptr};
+    size_t h_meta_cap[2] = {0, 0};
+    cudaEvent_t meta_ev[2] = {nullptr, nullptr};
+    int meta_slot = 0;
 };
+
+// Pinned staging slot for n MQMeta; waits until the copy that last used the
+// slot has completed.
+static int meta_stage(smiler_index *idx, int n, MQMeta **out, int *slot) {
+    const int s = idx->meta_slot;
+    idx->meta_slot ^= 1;
+    if (!idx->meta_ev[s]) CU(cudaEventCreateWithFlags(&idx->meta_ev[s], cudaEventDisableTiming));
+    else CU(cudaEventSynchronize(idx->meta_ev[s]));
+    if (idx->h_meta_cap[s] < (size_t)n) {
+        if (idx->h_meta[s]) cudaFreeHost(idx->h_meta[s]);
+        idx->h_meta[s] = nullptr;
+        size_t want = (size_t)n + n / 4 + 16;
+        CU(cudaMallocHost(&idx->h_meta[s], want * sizeof(MQMeta)));
+        idx->h_meta_cap[s] = want;
+    }
+    *out = idx->h_meta[s];
+    *slot = s;
+    return SMILER_OK;
+}
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per kernel and size.
+static void set_smem(const void *kern, size_t bytes) {
+    static std::map<const void *, size_t> done;
+    if (bytes <= 48 * 1024) return;
+    auto it = done.find(kern);
+    if (it != done.end() && it->second >= bytes) return;
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    done[kern] = bytes;
+}
 
 static size_t esize(smiler_dtype t) { return t == SMILER_I16 ? 2 : 4; }
 
@@ -240,6 +275,10 @@ static void destroy(smiler_index *idx) {
                       &idx->out_ids, &idx->out_d,  &idx->tmp};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
+    for (int s = 0; s < 2; s++) {
+        if (idx->h_meta[s]) cudaFreeHost(idx->h_meta[s]);
+        if (idx->meta_ev[s]) cudaEventDestroy(idx->meta_ev[s]);
+    }
     delete idx;
 }
 
@@ -256,6 +295,9 @@ static int common_build(smiler_index *idx, int32_t device, void *stream) {
     idx->stream = (cudaStream_t)stream;
     CU(cudaSetDevice(device));
     CU(cudaDeviceGetAttribute(&idx->num_sms, cudaDevAttrMultiProcessorCount, device));
+    size_t fr = 0, tot = 0;
+    if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) idx->budget = std::min(idx->budget, fr / 2);
+    cudaGetLastError();
     return SMILER_OK;
 }
 
@@ -406,7 +448,7 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
     if (pl.w == 4 || pl.w == 8 || pl.w == 16) {
         const int halo = mmax - 1;
         pl.RTf = kFusedThreads - halo;
-        pl.smem_fz = em + (size_t)pl.D * 16 + (size_t)pl.w * kFusedThreads * 8 +
+        pl.smem_fz = em + (size_t)pl.D * 12 + (size_t)2 * pl.w * kFusedThreads * 8 +
                      (size_t)n_len * pl.RTf * (pl.w + 1) * vs;
         pl.fused = halo <= kFusedThreads / 4 && pl.smem_fz <= 200 * 1024;
     }
@@ -530,12 +572,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         const size_t ndw = (size_t)(si.n / w);
         return (pl.fused ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
     };
-    size_t budget = (size_t)24 << 30;
-    {
-        size_t fr = 0, tot = 0;
-        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) budget = std::min(budget, fr / 2);
-        cudaGetLastError();
-    }
+    const size_t budget = idx->budget;
     int chunk_max = o.mq_chunk > 0 ? o.mq_chunk : 65535;
     chunk_max = std::min(chunk_max, 65535);
 
@@ -564,7 +601,9 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         const int B = c1 - c0;
         n_chunks++;
         // ---- metadata ------------------------------------------------------
-        std::vector<MQMeta> meta(B);
+        MQMeta *meta;
+        int mslot;
+        TRY(meta_stage(idx, B, &meta, &mslot));
         int64_t post_tot = 0, seg_tot = 0;
         int nblk_min = INT32_MAX, nblk_max = 0;
         for (int j = 0; j < B; j++) {
@@ -630,7 +669,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             TRY(idx->out_d.ensure(4 * (size_t)nseg * pl.k));
         }
         MQMeta *d_meta = idx->meta.as<MQMeta>();
-        CU(cudaMemcpyAsync(d_meta, meta.data(), sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
+        CU(cudaMemcpyAsync(d_meta, meta, sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
+        CU(cudaEventRecord(idx->meta_ev[mslot], idx->stream));
         CU(cudaMemcpyAsync(idx->queries.p, (const char *)queries + (size_t)c0 * D * es, es * (size_t)B * D,
                            q_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, idx->stream));
         TRY(tm.mark(0));
@@ -644,8 +684,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             // ---- a3 + a4 fused ------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
             auto go = [&](auto kern) {
-                if (pl.smem_fz > 48 * 1024)
-                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_fz);
+                set_smem((const void *)kern, pl.smem_fz);
                 kern<<<grid, kFusedThreads, pl.smem_fz, idx->stream>>>(
                     (const S *)idx->d_series, (const S *)dUC, (const S *)dLC, d_meta, idx->qtab.as<V4>(), P,
                     idx->lb.as<V>(), idx->tauc.as<int32_t>());
@@ -661,13 +700,12 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         } else {
             // ---- a3 ----------------------------------------------------------
             int64_t ndw_max = 0;
-            for (auto &m : meta) ndw_max = std::max(ndw_max, m.n_dw);
+            for (int j = 0; j < B; j++) ndw_max = std::max(ndw_max, meta[j].n_dw);
             if (ndw_max > 0) {
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
-                size_t smem = sizeof(V4) * D;
+                size_t smem = 3 * sizeof(V) * D;
                 auto go = [&](auto kern) {
-                    if (smem > 48 * 1024)
-                        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                    set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
                                                            w, idx->post.as<V2>());
@@ -687,8 +725,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             // ---- a4 ----------------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
             auto go4 = [&](auto kern) {
-                if (pl.smem_gs > 48 * 1024)
-                    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_gs);
+                set_smem((const void *)kern, pl.smem_gs);
                 kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(idx->post.as<V2>(), d_meta, P, idx->lb.as<V>(),
                                                                idx->tauc.as<int32_t>());
             };
@@ -745,7 +782,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // ---- a6 ----------------------------------------------------------
         {
             int64_t nmax = 0;
-            for (auto &m : meta) nmax = std::max(nmax, m.n);
+            for (int j = 0; j < B; j++) nmax = std::max(nmax, meta[j].n);
             if (!o.no_prune) {
                 dim3 grid((unsigned)((nmax + kFiltThreads * kFiltItems - 1) / (kFiltThreads * kFiltItems)),
                           (unsigned)nseg);
