@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 #include <stdio.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 constexpr int kIters = 4096;
 constexpr int kChains = 8;
@@ -122,8 +123,74 @@ __global__ void __launch_bounds__(kThreads) lbterm_i32_mix(int *out, long long *
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
+// LB term pair with packed fp32x2 (sm_100): per pair FADD2, FADD2, FMNMX3 x2, FFMA2.
+__global__ void __launch_bounds__(kThreads) lbterm_f32x2_mix(float *out, long long *cyc, float q0) {
+    float2 acc[kChains], cc[kChains], ne[kChains];
+#pragma unroll
+    for (int i = 0; i < kChains; i++) {
+        acc[i] = make_float2(0.f, 0.f);
+        cc[i] = make_float2(i * 0.3f - 1.0f, i * 0.3f - 1.0f);
+        ne[i] = make_float2(-0.5f - threadIdx.x * 1e-3f - i, 0.5f + i);
+    }
+    long long t0 = clock64();
+    for (int it = 0; it < kIters; it++) {
+        const float q = q0 + it * 1e-4f;
+        const float2 nq = make_float2(-q, -q * 0.5f);
+        const float2 qq = make_float2(q, q);
+#pragma unroll
+        for (int i = 0; i < kChains; i++) {
+            float2 d1 = __fadd2_rn(cc[i], nq);
+            float2 d2 = __fadd2_rn(qq, ne[i]);
+            float2 m = make_float2(fmaxf(fmaxf(d1.x, -d1.y), 0.f), fmaxf(fmaxf(d2.x, -d2.y), 0.f));
+            acc[i] = __ffma2_rn(m, m, acc[i]);
+        }
+    }
+    long long t1 = clock64();
+    float s = 0;
+#pragma unroll
+    for (int i = 0; i < kChains; i++) s += acc[i].x + acc[i].y;
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+}
+
+// DTW cells, two candidates per thread with packed fp32x2: per 2 cells FADD2, FMNMX3 x2, FFMA2.
+__global__ void __launch_bounds__(kThreads) dtw_f32x2_mix(float *out, long long *cyc, float q0) {
+    float2 a[kChains], b[kChains], nc[kChains];
+#pragma unroll
+    for (int i = 0; i < kChains; i++) {
+        a[i] = make_float2(i * 0.5f, i * 0.25f);
+        b[i] = make_float2(i * 0.25f, i * 0.5f);
+        nc[i] = make_float2(-threadIdx.x * 0.001f - i, -threadIdx.x * 0.002f + i);
+    }
+    long long t0 = clock64();
+    for (int it = 0; it < kIters; it++) {
+        const float q = q0 + it;
+        const float2 qq = make_float2(q, q);
+#pragma unroll
+        for (int i = 0; i < kChains; i++) {
+            float2 diff = __fadd2_rn(qq, nc[i]);
+            float2 m = make_float2(fminf(fminf(b[i].x, a[i].x), b[i].y), fminf(fminf(b[i].y, a[i].y), b[i].x));
+            b[i] = a[i];
+            a[i] = __ffma2_rn(diff, diff, m);
+        }
+    }
+    long long t1 = clock64();
+    float s = 0;
+#pragma unroll
+    for (int i = 0; i < kChains; i++) s += a[i].x + a[i].y;
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+}
+
+struct Rate {
+    double per_clk_sm;  // units per SM per SM clock
+    double mhz;         // effective SM clock during the run
+    double per_s;       // units per second, whole GPU
+};
+
+// Launch `kern` back to back for >= min_ms of device time (sustained clock).
 template <typename K, typename T>
-static double run(K kern, T arg, int sms, int per_sm, double units_per_iter_chain, double *mhz) {
+static Rate run(K kern, T arg, int sms, int per_sm, double units_per_iter_chain, float min_ms) {
     int grid = sms * per_sm;
     T *out;
     long long *cyc;
@@ -133,41 +200,58 @@ static double run(K kern, T arg, int sms, int per_sm, double units_per_iter_chai
     cudaEvent_t e0, e1;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
-    cudaEventRecord(e0);
-    kern<<<grid, kThreads>>>(out, cyc, arg);
-    cudaEventRecord(e1);
-    cudaEventSynchronize(e1);
-    float ms;
-    cudaEventElapsedTime(&ms, e0, e1);
+    int reps = 1;
+    float ms = 0;
+    long long cycles = 0;
+    while (true) {
+        cudaEventRecord(e0);
+        for (int r = 0; r < reps; r++) kern<<<grid, kThreads>>>(out, cyc, arg);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (ms >= min_ms || reps > (1 << 16)) break;
+        reps *= 2;
+    }
     long long *h = new long long[grid];
     cudaMemcpy(h, cyc, sizeof(long long) * grid, cudaMemcpyDeviceToHost);
-    long long mx = 0;
-    for (int i = 0; i < grid; i++) mx = h[i] > mx ? h[i] : mx;
+    for (int i = 0; i < grid; i++) cycles = h[i] > cycles ? h[i] : cycles;  // last launch
     delete[] h;
     cudaFree(out);
     cudaFree(cyc);
-    // units per SM per clock: all per_sm CTAs of an SM run concurrently for ~mx cycles
-    double units = (double)per_sm * kThreads * kIters * kChains * units_per_iter_chain;
-    *mhz = mx / (ms * 1e3);
-    return units / (double)mx;
+    double units_launch = (double)grid * kThreads * kIters * kChains * units_per_iter_chain;
+    Rate R;
+    R.per_clk_sm = units_launch / sms / (double)cycles;
+    R.per_s = units_launch * reps / (ms * 1e-3);
+    R.mhz = R.per_s / (R.per_clk_sm * sms) / 1e6;
+    return R;
 }
 
-int main() {
+int main(int argc, char **argv) {
     int dev = 0, sms = 0;
     cudaSetDevice(dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int per_sm = 8;  // 64 warps per SM
-    double mz1, mz2, mz3, mz4;
-    double cf = run(dtw_f32_mix, 1.0f, sms, per_sm, 1.0, &mz1);
-    double ci = run(dtw_i32_mix, 1, sms, per_sm, 1.0, &mz2);
-    double lf = run(lbterm_f32_mix, 0.1f, sms, per_sm, 1.0, &mz3);
-    double li = run(lbterm_i32_mix, 1, sms, per_sm, 1.0, &mz4);
+    const float min_ms = argc > 1 ? (float)atof(argv[1]) : 400.f;
+    // interleaved, sustained: each mix twice, keep the second (steady clock)
+    Rate r[6];
+    for (int pass = 0; pass < 2; pass++) {
+        r[0] = run(dtw_f32_mix, 1.0f, sms, per_sm, 1.0, min_ms);
+        r[1] = run(dtw_f32x2_mix, 1.0f, sms, per_sm, 2.0, min_ms);
+        r[2] = run(lbterm_f32_mix, 0.1f, sms, per_sm, 1.0, min_ms);
+        r[3] = run(lbterm_f32x2_mix, 0.1f, sms, per_sm, 1.0, min_ms);
+        r[4] = run(dtw_i32_mix, 1, sms, per_sm, 1.0, min_ms);
+        r[5] = run(lbterm_i32_mix, 1, sms, per_sm, 1.0, min_ms);
+    }
     cudaError_t e = cudaGetLastError();
-    printf("{\"sms\": %d, \"dtw_cell_f32_per_clk_sm\": %.3f, \"dtw_cell_i32_per_clk_sm\": %.3f, "
-           "\"lbterm_per_clk_sm\": %.3f, \"lbterm_i32_per_clk_sm\": %.3f, \"sm_mhz_seen\": [%.0f, %.0f, %.0f, %.0f], "
-           "\"note\": \"units per SM per SM-clock over one full wave (8 CTAs x 256 threads per SM, 8 independent "
-           "chains per thread); dtw cell = FADD+FMNMX3+FFMA (f32) or IADD+VIMNMX3+IMAD(+LOP) (i32); lbterm = one "
-           "(SW,DW,j) EQ+EC term pair = 2x(FMNMX,FMNMX,FADD,FFMA)\", \"cuda\": \"%s\"}\n",
-           sms, cf, ci, lf, li, mz1, mz2, mz3, mz4, cudaGetErrorString(e));
+    const char *names[6] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32"};
+    printf("{\"sms\": %d, \"sustained_ms_per_mix\": %.0f", sms, min_ms);
+    for (int i = 0; i < 6; i++)
+        printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e", names[i], r[i].per_clk_sm,
+               names[i], r[i].mhz, names[i], r[i].per_s);
+    printf(", \"note\": \"units per SM per SM clock and per second over back-to-back full waves (8 CTAs x 256 threads "
+           "per SM, 8 independent chains per thread), sustained for the stated time; dtw cell = FADD+FMNMX3+FFMA (f32), "
+           "f32x2 = FADD2+2 FMNMX3+FFMA2 per 2 cells, i32 = IADD+VIMNMX3+IMAD(+LOP); lbterm = one (SW,DW,j) EQ+EC "
+           "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2\", \"cuda\": \"%s\"}\n",
+           cudaGetErrorString(e));
     return e == cudaSuccess ? 0 : 1;
 }

@@ -95,6 +95,86 @@ __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, c
     }
 }
 
+// Barrier-free epilogue for tiles whose row x is written only by thread x
+// (lb_diag_kernel): every thread writes its own W slots (t contiguous) and
+// the tau set is chosen per warp (E smallest (LB_w, t) among the warp's slots,
+// by warp-shuffle minima).  tauc slot: (mq, i) row, [blockIdx.x * NW + warp] * E + e.
+template <typename V, int W>
+__device__ void lb_tile_epilogue_warp(V *tile, int RT, int64_t e0, const MQMeta &m, const QParams &P, V *lb,
+                                      int32_t *tauc, int mq) {
+    const int nl = P.n_len;
+    const int stride = RT * (W + 1);
+    const int x = threadIdx.x, lane = x & 31, warp = x >> 5, nw = blockDim.x >> 5;
+    const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t s0 = e0 + (int64_t)x * W;  // e of this thread's slot 0
+    for (int i = 0; i < nl; i++) {
+        const int d = P.len[i];
+        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        V *out = lb + m.seg_off + (int64_t)i * m.n;
+        V *row = tile + i * stride + x * (W + 1);
+        uint64_t best = kKeyMax;
+        int bs = -1;
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            const int64_t t = s0 + b - d;
+            if (t >= tmin && t < tend) {
+                const V v = row[b];
+                out[t] = v;
+                const uint64_t key = ((uint64_t)key_bits(v) << 32) | (uint32_t)t;
+                if (key < best) {
+                    best = key;
+                    bs = b;
+                }
+            }
+        }
+        if (P.E <= 0) continue;
+        int32_t *dst = tauc + (int64_t)(mq * nl + i) * P.LT + ((int64_t)blockIdx.x * nw + warp) * P.E;
+        for (int e = 0; e < P.E; e++) {
+            if (e > 0) {
+                best = kKeyMax;
+                bs = -1;
+#pragma unroll
+                for (int b = 0; b < W; b++) {
+                    const int64_t t = s0 + b - d;
+                    const uint32_t kb = key_bits(row[b]);
+                    if (t >= tmin && t < tend && kb != 0xFFFFFFFFu) {
+                        const uint64_t key = ((uint64_t)kb << 32) | (uint32_t)t;
+                        if (key < best) {
+                            best = key;
+                            bs = b;
+                        }
+                    }
+                }
+            }
+            const uint64_t win = warp_min_u64(best);
+            if (win != kKeyMax && best == win) {
+                uint32_t allones = 0xFFFFFFFFu;
+                row[bs] = *reinterpret_cast<V *>(&allones);
+            }
+            if (lane == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+        }
+    }
+}
+
+// Posting elements of one chunk from a preloaded window (see posting_chunk).
+template <typename V, int W, int BC, bool CHECK, int WL, typename F>
+__device__ __forceinline__ void posting_chunk_w(const V (&c)[W], const V (&U)[W], const V (&L)[W], const V (&wq)[WL],
+                                                const V (&wu)[WL], const V (&wl)[WL], int nvalid, F &&store) {
+#pragma unroll
+    for (int bb = 0; bb < BC; bb++) {
+        if (!CHECK || bb < nvalid) {
+            V eq = (V)0, ec = (V)0;
+#pragma unroll
+            for (int j = 0; j < W; j++) {
+                const int k = BC - 1 - bb + j;
+                lb_term(c[j], wu[k], wl[k], eq);
+                lb_term(wq[k], U[j], L[j], ec);
+            }
+            store(bb, eq, ec);
+        }
+    }
+}
+
 // One sliding-window chunk of posting elements: SW_{b0+bb} (bb < BC) against
 // the thread's DW (c, U, L).  Window registers hold MQ positions
 // pb .. pb + W + BC - 2 (pb = D - W - b0 - (BC-1)): q, U(Q), L(Q).
@@ -104,12 +184,22 @@ __device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], 
                                               const V *qq, const V *uq, const V *lq, int pb, int nvalid,
                                               F &&store) {
     V wq[W + BC - 1], wu[W + BC - 1], wl[W + BC - 1];
+    if (CHECK) {
 #pragma unroll
-    for (int k = 0; k < W + BC - 1; k++) {
-        const int p = max(pb + k, 0);
-        wq[k] = qq[p];
-        wu[k] = uq[p];
-        wl[k] = lq[p];
+        for (int k = 0; k < W + BC - 1; k++) {
+            const int p = max(pb + k, 0);
+            wq[k] = qq[p];
+            wu[k] = uq[p];
+            wl[k] = lq[p];
+        }
+    } else {  // every position of a full chunk is >= 0: base + immediate offsets
+        const V *q0 = qq + pb, *u0 = uq + pb, *l0 = lq + pb;
+#pragma unroll
+        for (int k = 0; k < W + BC - 1; k++) {
+            wq[k] = q0[k];
+            wu[k] = u0[k];
+            wl[k] = l0[k];
+        }
     }
 #pragma unroll
     for (int bb = 0; bb < BC; bb++) {
@@ -381,4 +471,230 @@ __global__ void __launch_bounds__(kFusedThreads, (W <= 8 ? 3 : 1)) lb_fused_kern
     }
     __syncthreads();
     lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * W, m, P, lb, tauc, mq, s_red);
+}
+
+// ---------------------------------------------------------------------------
+// a3+a4 fused, diagonal form (one-shot batches, default).  Thread x owns the
+// rightmost DW r = Rb + x and walks its CSG diagonals itself: for row j it
+// reads DW r - j (points and envelope) from a transposed shared-memory tile of
+// the CTA's DWs plus a left halo of mmax-1 DWs, computes P[b + j w][r - j] for
+// all b < w with the row's 2w-1 MQ positions in registers, and adds them
+// straight into its running sums S_b.  No barrier inside the row loop, no
+// halo recomputation, no posting list in memory at all.
+// smem: em | sqq, squ, sql [D] | cs, us, ls [w][NT + HALO] | tile.
+// ---------------------------------------------------------------------------
+constexpr int kDiagThreads = 128;
+constexpr int kDiagHaloMax = 128;
+constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile stride
+
+// Write the W final LB_w values of IQ i held by this thread (slots e = s0 + b,
+// t = e - d_i contiguous) and emit its warp's tau candidates.
+template <typename V, int W>
+__device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
+                                          V *lb, int32_t *tauc, int mq) {
+    const int d = P.len[i];
+    const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t tend = min(m.t_hi, m.n - d + 1);
+    V *out = lb + m.seg_off + (int64_t)i * m.n;
+    const int64_t t0 = s0 - d;
+    const bool all = t0 >= tmin && t0 + W <= tend;
+    if (all && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
+#pragma unroll
+        for (int b = 0; b < W; b += 4) {
+            typename Tr<int16_t>::V4 pk;  // 4 x 32-bit lanes (int or float bits)
+            pk.x = *reinterpret_cast<const int32_t *>(&v[b]);
+            pk.y = *reinterpret_cast<const int32_t *>(&v[b + 1]);
+            pk.z = *reinterpret_cast<const int32_t *>(&v[b + 2]);
+            pk.w = *reinterpret_cast<const int32_t *>(&v[b + 3]);
+            *reinterpret_cast<int4 *>(out + t0 + b) = pk;
+        }
+    } else {
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            const int64_t t = t0 + b;
+            if (t >= tmin && t < tend) out[t] = v[b];
+        }
+    }
+    if (P.E <= 0) return;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + ((int64_t)blockIdx.x * nw + warp) * P.E;
+    uint32_t taken = 0;
+    for (int e = 0; e < P.E; e++) {
+        uint64_t best = kKeyMax;
+        int bs = -1;
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            const int64_t t = t0 + b;
+            if (!(taken >> b & 1u) && t >= tmin && t < tend) {
+                const uint64_t key = ((uint64_t)key_bits(v[b]) << 32) | (uint32_t)t;
+                if (key < best) {
+                    best = key;
+                    bs = b;
+                }
+            }
+        }
+        const uint64_t win = warp_min_u64(best);
+        if (win != kKeyMax && best == win) taken |= 1u << bs;
+        if (lane == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3+a4 fused, diagonal form (one-shot batches, default).  Thread x owns the
+// rightmost DW r = Rb + x and walks its CSG diagonals itself: for row j it
+// reads DW r - j (points and envelope) from a transposed shared-memory tile of
+// the CTA's DWs plus a left halo of mmax-1 DWs, computes P[b + j w][r - j] for
+// all b < w with the row's 2w-1 MQ positions in registers, and adds them
+// straight into its running sums S_b.  No barrier inside the row loop, no
+// halo recomputation, no posting list in memory at all.
+// Emission: m_i(b) = floor((d_i - b)/w) = q_i - [b > r_i] (d_i = q_i w + r_i),
+// so IQ i's slots b > r_i are final after row q_i - 2 and b <= r_i after row
+// q_i - 1; the thread saves the former and writes all w values of IQ i after
+// row q_i - 1 straight from registers (vector stores), choosing the tau set of
+// its warp with shuffles.  No LB tile, no epilogue barrier.
+// smem: sqq, squ, sql [D] | cs, us, ls [w][kDiagCols].
+// ---------------------------------------------------------------------------
+// padded column stride (floats) of the DW tile: multiple of 4 for 16-byte
+// loads, chosen so the 8 lanes of one LDS.128 phase hit distinct banks
+template <int W> struct DiagStride { static constexpr int v = (W == 4) ? 12 : W + 4; };
+
+template <typename S, int W>
+__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 4 : 2))
+    lb_diag_kernel(const S *series, const S *UC, const S *LC, const MQMeta *meta,
+                   const typename Tr<S>::V4 *qtab, const QParams P, typename Tr<S>::V *lb,
+                   int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V4 = typename Tr<S>::V4;
+    constexpr int NT = kDiagThreads;
+    constexpr int BC = W < 8 ? W : 8;
+    constexpr int DS = DiagStride<W>::v;
+    constexpr int WL = ((W + BC - 1) + 3) & ~3;  // window registers, rounded to 16-byte loads
+    extern __shared__ __align__(16) unsigned char dg_smem[];
+    const int D = P.D;
+    const int nl = P.n_len;
+    const int n_sw = D - W + 1;
+    const int mmax = D / W;
+    const int HALO = mmax - 1;
+    const int NC = NT + HALO;  // DW columns in the tile
+    // MQ arrays shifted so every row's window start is 16-byte aligned
+    const int qshift = (4 - ((D - W - BC + 1) % 4 + 4) % 4) % 4;
+    const int QL = (D + qshift + WL + 3) & ~3;
+    V *sqq = reinterpret_cast<V *>(dg_smem);
+    V *squ = sqq + QL;
+    V *sql = squ + QL;
+    V *cs = sql + QL;  // [kDiagCols][DS]
+    V *us = cs + kDiagCols * DS;
+    V *ls = us + kDiagCols * DS;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) return;
+    for (int p = threadIdx.x; p < QL; p += NT) {
+        const int src = p - qshift;
+        V q = (V)0, u = (V)0, l = (V)0;
+        if (src >= 0 && src < D) {
+            const V4 e = qtab[(int64_t)mq * D + src];
+            q = e.x;
+            u = e.y;
+            l = e.z;
+        }
+        sqq[p] = q;
+        squ[p] = u;
+        sql[p] = l;
+    }
+    const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
+    const int64_t R0 = Rb - HALO;  // DW of tile column 0
+    for (int idx = threadIdx.x; idx < NC * W; idx += NT) {
+        const int col = idx / W, jj = idx % W;
+        const int64_t rp = R0 + col;
+        V c = (V)0, u = (V)0, l = (V)0;
+        if (rp >= 0 && rp < m.n_dw) {
+            const int64_t g = m.series_off + rp * W + jj;
+            c = (V)series[g];
+            u = (V)UC[g];
+            l = (V)LC[g];
+        }
+        cs[col * DS + jj] = c;
+        us[col * DS + jj] = u;
+        ls[col * DS + jj] = l;
+    }
+    __syncthreads();
+    const int x = threadIdx.x;
+    const int64_t s0 = (Rb + 1 + x) * W;  // e of this thread's slot b = 0
+    V se[W], sc[W], saved[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) se[b] = sc[b] = saved[b] = (V)0;
+    uint64_t emit_rows = 0, save_rows = 0;  // rows q_i - 1 / q_i - 2 (block-uniform)
+    for (int i = 0; i < nl; i++) {
+        const int qi = P.len[i] / W;
+        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
+        if (qi >= 2) save_rows |= 1ull << (qi - 2);
+    }
+    // IQs shorter than W have no full DW anywhere (m = 0, R6): LB_w = 0
+    for (int i = 0; i < nl && P.len[i] < W; i++)
+        if (P.k >= 0) diag_emit<V, W>(saved, i, s0, m, P, lb, tauc, mq);
+    for (int j = 0; j < mmax; j++) {
+        const int col = x + HALO - j;  // DW r - j
+        V c[W], U[W], L[W];
+#pragma unroll
+        for (int jj = 0; jj < W; jj += 4) {
+            const V4 a = *reinterpret_cast<const V4 *>(cs + col * DS + jj);
+            const V4 u = *reinterpret_cast<const V4 *>(us + col * DS + jj);
+            const V4 l = *reinterpret_cast<const V4 *>(ls + col * DS + jj);
+            c[jj] = a.x, c[jj + 1] = a.y, c[jj + 2] = a.z, c[jj + 3] = a.w;
+            U[jj] = u.x, U[jj + 1] = u.y, U[jj + 2] = u.z, U[jj + 3] = u.w;
+            L[jj] = l.x, L[jj + 1] = l.y, L[jj + 2] = l.z, L[jj + 3] = l.w;
+        }
+        const int nrow = min(W, n_sw - j * W);
+#pragma unroll
+        for (int b0 = 0; b0 < W; b0 += BC) {
+            const int nv = nrow - b0;
+            auto acc = [&](int bb, V eq, V ec) {
+                se[b0 + bb] += eq;
+                sc[b0 + bb] += ec;
+            };
+            const int pb = D - W - j * W - b0 - (BC - 1);
+            if (nv >= BC) {  // full chunk: aligned 16-byte window loads
+                V wq[WL], wu[WL], wl[WL];
+                const int base = pb + qshift;
+#pragma unroll
+                for (int k = 0; k < WL; k += 4) {
+                    const V4 a = *reinterpret_cast<const V4 *>(sqq + base + k);
+                    const V4 u = *reinterpret_cast<const V4 *>(squ + base + k);
+                    const V4 l = *reinterpret_cast<const V4 *>(sql + base + k);
+                    wq[k] = a.x, wq[k + 1] = a.y, wq[k + 2] = a.z, wq[k + 3] = a.w;
+                    wu[k] = u.x, wu[k + 1] = u.y, wu[k + 2] = u.z, wu[k + 3] = u.w;
+                    wl[k] = l.x, wl[k + 1] = l.y, wl[k + 2] = l.z, wl[k + 3] = l.w;
+                }
+                posting_chunk_w<V, W, BC, false, WL>(c, U, L, wq, wu, wl, BC, acc);
+            } else if (nv > 0) {
+                posting_chunk<V, W, BC, true>(c, U, L, sqq + qshift, squ + qshift, sql + qshift, pb, nv, acc);
+            }
+        }
+        if (P.k < 0) continue;  // timing experiment: main loop only
+        // rows q_i - 1: compose IQ i from the values saved after row q_i - 2
+        // (slots b > r_i) and the current sums (b <= r_i), then write it
+        if (emit_rows >> j & 1ull) {
+            for (int i = 0; i < nl; i++) {
+                const int qi = P.len[i] / W, ri = P.len[i] % W;
+                if (j == qi - 1) {
+                    V v[W];
+#pragma unroll
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? saved[b] : (V)0) : vmax(se[b], sc[b]);
+                    diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
+                }
+            }
+        }
+        // rows q_i - 2: save (after composing, so a row that is q_i - 1 for one
+        // IQ and q_i' - 2 for another uses the previous row's saved values)
+        if (save_rows >> j & 1ull) {
+#pragma unroll
+            for (int b = 0; b < W; b++) saved[b] = vmax(se[b], sc[b]);
+        }
+    }
+    if (P.k < 0) {  // timing experiment: keep the sums alive
+        V acc = (V)0;
+#pragma unroll
+        for (int b = 0; b < W; b++) acc += se[b] + sc[b];
+        if (acc == (V)12345) lb[0] = acc;
+    }
 }

@@ -410,6 +410,7 @@ struct Plan {
     std::vector<int> len, rho;
     int RT;          // group-scan CTA width (two-level path)
     bool fused;      // a3+a4 fused kernel
+    int fused_kind;  // 0 = diagonal form (lb_diag_kernel), 1 = row form (lb_fused_kernel)
     int RTf;         // fused: tile DWs per CTA
     size_t smem_gs, smem_fz;
 };
@@ -451,6 +452,15 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
         pl.smem_fz = em + (size_t)pl.D * 12 + (size_t)2 * pl.w * kFusedThreads * 8 +
                      (size_t)n_len * pl.RTf * (pl.w + 1) * vs;
         pl.fused = halo <= kFusedThreads / 4 && pl.smem_fz <= 200 * 1024;
+        pl.fused_kind = 1;
+        const int ds = pl.w == 4 ? 12 : pl.w + 4;
+        const size_t smem_dg = (size_t)3 * ((pl.D + 3 + 32 + 3) & ~3) * vs + (size_t)3 * kDiagCols * ds * vs;
+        if (halo <= kDiagHaloMax && mmax <= 64 && smem_dg <= 200 * 1024) {
+            pl.fused = true;
+            pl.fused_kind = 0;
+            pl.RTf = kDiagThreads;
+            pl.smem_fz = smem_dg;
+        }
     }
     return SMILER_OK;
 }
@@ -529,6 +539,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     Plan pl;
     TRY(validate_query(idx, lens_h.data(), n_len, lb_only ? 1 : k, pl));
     if (o.two_level || (lb_only && post_out)) pl.fused = false;
+    if (pl.fused && o.reserved[0] == 1 && pl.fused_kind == 0) {  // row-form fused kernel (comparison)
+        const int mmax = pl.D / pl.w, halo = mmax - 1;
+        const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
+        pl.fused_kind = 1;
+        pl.RTf = kFusedThreads - halo;
+        pl.smem_fz = em + (size_t)pl.D * 12 + (size_t)2 * pl.w * kFusedThreads * 8 +
+                     (size_t)pl.n_len * pl.RTf * (pl.w + 1) * 4;
+        if (halo > kFusedThreads / 4 || pl.smem_fz > 200 * 1024) pl.fused = false;
+    }
     const int D = pl.D, w = pl.w, nl = pl.n_len;
     std::vector<int32_t> qsens(n_mq, 0);
     if (query_sensor_in) {
@@ -631,9 +650,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 bf_cells += (double)nc * (double)dtw_cells(pl.len[i], pl.rho[i]);
             }
         }
+        // tau-set units: CTAs (block epilogue) or warps (diagonal kernel's warp epilogue)
+        const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32 : 1;
         int E = 0;
-        if (!lb_only && !o.no_prune) E = std::min(8, std::max(1, (2 * pl.k + nblk_min - 1) / nblk_min));
-        const int LT = std::max(1, nblk_max * E);
+        if (!lb_only && !o.no_prune) {
+            const int umin = nblk_min * units_per_blk;
+            E = std::min(8, std::max(1, (2 * pl.k + umin - 1) / umin));
+        }
+        const int LT = std::max(1, nblk_max * units_per_blk * E);
         QParams P;
         memset(&P, 0, sizeof(P));
         P.D = D;
@@ -642,6 +666,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         P.k = pl.k;
         P.rho_env = pl.rho_env;
         P.E = E;
+        if (o.reserved[1] == 1) P.k = -1;  // timing experiment (results invalid)
+        if (o.reserved[1] == 2) P.E = 0;   // timing experiment: no tau set (no pruning)
         P.LT = LT;
         P.n_mq = B;
         for (int i = 0; i < nl; i++) {
@@ -683,16 +709,25 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         if (pl.fused) {
             // ---- a3 + a4 fused ------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
+            const int nthr = pl.fused_kind == 0 ? kDiagThreads : kFusedThreads;
             auto go = [&](auto kern) {
                 set_smem((const void *)kern, pl.smem_fz);
-                kern<<<grid, kFusedThreads, pl.smem_fz, idx->stream>>>(
+                kern<<<grid, nthr, pl.smem_fz, idx->stream>>>(
                     (const S *)idx->d_series, (const S *)dUC, (const S *)dLC, d_meta, idx->qtab.as<V4>(), P,
                     idx->lb.as<V>(), idx->tauc.as<int32_t>());
             };
-            switch (w) {
-                case 4: go(lb_fused_kernel<S, 4>); break;
-                case 8: go(lb_fused_kernel<S, 8>); break;
-                default: go(lb_fused_kernel<S, 16>); break;
+            if (pl.fused_kind == 0) {
+                switch (w) {
+                    case 4: go(lb_diag_kernel<S, 4>); break;
+                    case 8: go(lb_diag_kernel<S, 8>); break;
+                    default: go(lb_diag_kernel<S, 16>); break;
+                }
+            } else {
+                switch (w) {
+                    case 4: go(lb_fused_kernel<S, 4>); break;
+                    case 8: go(lb_fused_kernel<S, 8>); break;
+                    default: go(lb_fused_kernel<S, 16>); break;
+                }
             }
             CHECK_LAUNCH();
             launches++;
