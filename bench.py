@@ -139,6 +139,9 @@ def rank_workload(cfg: str, dtype: str, rank: int, world: int, mq_per_step: int)
                 qsens.append(li)
         return synth.Workload(cfg, dtype, np.concatenate(parts), np.asarray(offs, np.int64),
                               np.ascontiguousarray(np.stack(qs)), np.asarray(qsens, np.int32), lens, k, w, band)
+    if cfg == "C4":
+        # one long series; every rank holds the same MQ batch and its own window range
+        return synth.make_workload("C4", dtype, mq_per_sensor=mq_per_step)
     raise ValueError(cfg)
 
 
@@ -181,12 +184,103 @@ def oracle_sample(wl, target_s: float):
 
 
 # ---------------------------------------------------------------------------
+CFG_NAMES = {
+    "C2": "C2: one sensor, 2^20 points, ELV {16,32,64,128}, band 10%, k=32, w=8, 256 MQs/step/GPU",
+    "C3": "C3: 1024 sensors x 100k, ELV {32,64,96}, rho=8, k=64, w=16, 1 MQ/sensor, sharded by sensor",
+    "C4": "C4: one series of 1e8 points, ELV {32,64,96}, rho=8, k=32, w=16, 16 MQs/step, window ranges "
+          "sharded over GPUs, NCCL all-gather + smiler_merge_topk",
+    "C5": "C5: 1024 sensors x 100k, 10 streams/sensor (10,240 MQs/tick), ELV {16,32,64,128}, band 20%, k=128, "
+          "w=8, sharded by sensor",
+}
+
+
+class Runner:
+    """One configuration's step on this rank.  step() = device-resident inputs
+    and outputs; step_e2e() = pinned host inputs -> result on the host."""
+
+    def __init__(self, args, pkg, torch, dist, rank, world, local, dev, stream):
+        self.args, self.pkg, self.torch, self.dist = args, pkg, torch, dist
+        self.rank, self.world, self.dev, self.stream = rank, world, dev, stream
+        cfg = args.config
+        wl = rank_workload(cfg, args.dtype, rank, world, args.mq if cfg == "C2" else 16)
+        self.wl = wl
+        self.n_len, self.k = len(wl.lengths), wl.k
+        self.sharded_window = cfg == "C4"
+        if self.sharded_window:
+            from paper_conf_sigmod_zhout15_b200 import dist as sdist
+            self.sdist = sdist
+            N = len(wl.series)
+            sh = sdist.window_shards(N, wl.D, max(wl.rhos()), wl.window, world)[rank]
+            self.shard = sh
+            sl = np.ascontiguousarray(wl.series[sh.slice_begin:sh.slice_end])
+            self.idx = pkg.Index.shard(sl, sh.slice_begin, N, sh.t_begin, sh.t_end, wl.window, wl.band,
+                                       device=local, stream=stream)
+            self.index_points = len(sl)
+            self.global_mq = wl.n_mq              # every rank serves the same MQs
+        else:
+            self.idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band, device=local, stream=stream)
+            self.index_points = len(wl.series)
+            self.global_mq = None                 # summed over ranks
+        self.qd = torch.from_numpy(wl.queries).to(dev)
+        self.qs = None if self.sharded_window else np.ascontiguousarray(wl.query_sensor)
+        vt = torch.int32 if args.dtype == "i16" else torch.float32
+        self.vt = vt
+        self.ids = torch.empty((wl.n_mq, self.n_len, self.k), dtype=torch.int64, device=dev)
+        self.dd = torch.empty((wl.n_mq, self.n_len, self.k), dtype=vt, device=dev)
+        self.op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=int(args.two_level))
+
+    def mq_per_step(self):
+        """Master queries completed per step on this rank (for the value)."""
+        if self.sharded_window:
+            return self.wl.n_mq / self.world  # each MQ's work is split over the ranks
+        return self.wl.n_mq
+
+    def _merge(self, ids, dd):
+        rows = self.wl.n_mq * self.n_len
+        gi, gd = self.sdist.all_gather_results(ids.view(rows, self.k), dd.view(rows, self.k))
+        oi, od = self.sdist.merge_gathered(gi, gd, self.k)
+        return oi, od
+
+    def step(self, stats=None, opts=None):
+        pkg = self.pkg
+        pkg.smiler_knn(self.idx.handle, self.qd, self.qs, self.wl.lengths, self.k, self.ids, self.dd, stats,
+                       opts if opts is not None else (self.op if stats is not None else None))
+        if self.sharded_window:
+            with self.torch.cuda.stream(self.stream):
+                self._merge(self.ids, self.dd)
+
+    def e2e_buffers(self):
+        torch = self.torch
+        self.qh = torch.from_numpy(self.wl.queries).pin_memory()
+        rows = self.wl.n_mq * self.n_len
+        self.ih = torch.empty((rows, self.k), dtype=torch.int64).pin_memory()
+        self.dh = torch.empty((rows, self.k), dtype=self.vt).pin_memory()
+        h2d = self.qh.numel() * self.qh.element_size() + self.n_len * 4 + (0 if self.qs is None else self.qs.nbytes)
+        return int(h2d), int(self.ih.numel() * 8 + self.dh.numel() * 4)
+
+    def step_e2e(self):
+        pkg, torch = self.pkg, self.torch
+        if not self.sharded_window:
+            pkg.smiler_knn(self.idx.handle, self.qh, self.qs, self.wl.lengths, self.k,
+                           self.ih.view(self.wl.n_mq, self.n_len, self.k), self.dh.view(self.wl.n_mq, self.n_len,
+                                                                                       self.k))
+            return
+        with torch.cuda.stream(self.stream):
+            self.qd.copy_(self.qh, non_blocking=True)
+        pkg.smiler_knn(self.idx.handle, self.qd, None, self.wl.lengths, self.k, self.ids, self.dd)
+        with torch.cuda.stream(self.stream):
+            oi, od = self._merge(self.ids, self.dd)
+            self.ih.copy_(oi, non_blocking=True)
+            self.dh.copy_(od, non_blocking=True)
+        self.stream.synchronize()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C2", choices=["C2", "C3", "C5"])
+    ap.add_argument("--config", default="C2", choices=["C2", "C3", "C4", "C5"])
     ap.add_argument("--dtype", default="f32", choices=["f32", "i16"])
     ap.add_argument("--mq", type=int, default=256, help="master queries per step per GPU (C2)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -201,18 +295,16 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    cfg_name = {"C2": "C2: one sensor, 2^20 points, ELV {16,32,64,128}, band 10%, k=32, w=8",
-                "C3": "C3: 1024 sensors x 100k, ELV {32,64,96}, rho=8, k=64, w=16, sharded by sensor",
-                "C5": "C5: 1024 sensors x 100k, 10 streams/sensor, ELV {16,32,64,128}, band 20%, k=128"}[args.config]
+    cfg_name = CFG_NAMES[args.config]
+    scaling = {"C2": "weak", "C3": "strong", "C4": "strong", "C5": "strong"}[args.config]
 
     if args.impl == "reference":
         if rank != 0:
             return
-        wl = rank_workload(args.config, args.dtype, 0, 1, min(args.mq, 4))
+        wl = rank_workload(args.config, args.dtype, 0, 1, 4)
         vals = []
-        for _ in range(max(args.warmup, 0)):
-            pass  # the oracle has nothing to warm up
         total = 0.0
+        cores, sample = 0, ""
         for _ in range(args.steps):
             v, cores, dt, sample = oracle_sample(wl, max(1.0, args.oracle_seconds / max(args.steps, 1)))
             vals.append(v)
@@ -220,10 +312,10 @@ def main():
         v = statistics.median(vals)
         print(json.dumps({"metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
                           "warmup": args.warmup, "ms_per_step": 1000.0 * total / args.steps,
-                          "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                          "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
                           "dtype": "int64" if args.dtype == "i16" else "f64", "data": "synthetic",
                           "impl": "reference",
-                          "config": {"workload": cfg_name, "parallelism": "host cores"},
+                          "config": {"workload": cfg_name, "parallelism": "host cores (oracle)"},
                           "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                                            "sample": sample},
                           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
@@ -240,22 +332,19 @@ def main():
     _build.build()
     import paper_conf_sigmod_zhout15_b200 as pkg
 
-    wl = rank_workload(args.config, args.dtype, rank, world, args.mq)
     stream = torch.cuda.Stream(device=dev)
-    n_len, k = len(wl.lengths), wl.k
-    idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band, device=local, stream=stream)
-    qd = torch.from_numpy(wl.queries).to(dev)
-    qs = torch.from_numpy(wl.query_sensor).to(dev)
-    ids = torch.empty((wl.n_mq, n_len, k), dtype=torch.int64, device=dev)
-    dd = torch.empty((wl.n_mq, n_len, k), dtype=torch.int32 if args.dtype == "i16" else torch.float32, device=dev)
-    st = pkg.KnnStats()
-    op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=int(args.two_level))
-
-    def step(stats=None):
-        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, stats, op if stats is not None else None)
+    if args.config == "C4" and world == 1:
+        # single GPU: the window "shard" is the whole series; the all-gather is a no-op
+        pass
+    if args.config == "C4" and not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    R = Runner(args, pkg, torch, dist, rank, world, local, dev, stream)
+    wl, n_len, k = R.wl, R.n_len, R.k
 
     for _ in range(args.warmup):
-        step()
+        R.step()
     torch.cuda.synchronize(dev)
 
     # ---- timed region: device-resident inputs/outputs, no host sync per call --
@@ -275,7 +364,7 @@ def main():
     e1 = torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(args.steps):
-        step()
+        R.step()
     e1.record(stream)
     torch.cuda.synchronize(dev)
     ck = clocks.stop()
@@ -286,30 +375,34 @@ def main():
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max = float(t.item())
-    value = world * wl.n_mq * args.steps / (ms_max / 1000.0)
+    mq_total = (R.global_mq if R.global_mq is not None else R.mq_per_step() * world) * args.steps
+    if R.global_mq is None and world > 1:
+        tm = torch.tensor([R.mq_per_step() * args.steps], dtype=torch.float64, device=dev)
+        dist.all_reduce(tm, op=dist.ReduceOp.SUM)
+        mq_total = float(tm.item())
+    value = mq_total / (ms_max / 1000.0)
 
     # ---- profiled pass: same command with per-phase CUDA events (stats) ---------
+    st = pkg.KnnStats()
     phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_verify",
                               "ns_select", "ns_total")}
     acc = {"survivors": 0, "candidates": 0, "dtw_cells": 0.0, "bf_cells": 0.0, "posting_bytes": 0,
            "lb_bytes": 0, "kernel_launches": 0, "mq_chunks": 0, "tau_verified": 0, "finalists": 0}
     prof_steps = max(1, min(args.steps, 5))
     for _ in range(prof_steps):
-        step(st)
+        R.step(st)
         for f in phase:
             phase[f] += getattr(st, f)
         for f in acc:
             acc[f] += getattr(st, f)
-    launches_per_step = acc["kernel_launches"] / prof_steps
+    torch.cuda.synchronize(dev)
+    launches_per_step = acc["kernel_launches"] / prof_steps + (1 if R.sharded_window else 0)
 
     # ---- e2e: the same public call with pinned host buffers ------------------
     e2e = None
     if not args.no_e2e:
-        qh = torch.from_numpy(wl.queries).pin_memory()
-        ih = torch.empty((wl.n_mq, n_len, k), dtype=torch.int64).pin_memory()
-        dh = torch.empty((wl.n_mq, n_len, k), dtype=dd.dtype).pin_memory()
-        qsh = torch.from_numpy(wl.query_sensor)
-        pkg.smiler_knn(idx.handle, qh, qsh, wl.lengths, k, ih, dh)
+        h2d, d2h = R.e2e_buffers()
+        R.step_e2e()
         torch.cuda.synchronize(dev)
         if world > 1:
             dist.barrier()
@@ -317,7 +410,7 @@ def main():
         f1 = torch.cuda.Event(enable_timing=True)
         f0.record(stream)
         for _ in range(args.steps):
-            pkg.smiler_knn(idx.handle, qh, qsh, wl.lengths, k, ih, dh)
+            R.step_e2e()
         f1.record(stream)
         torch.cuda.synchronize(dev)
         ems = f0.elapsed_time(f1)
@@ -325,26 +418,24 @@ def main():
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         ems = float(te.item())
-        e2e = {"value": world * wl.n_mq * args.steps / (ems / 1000.0), "unit": UNIT,
-               "h2d_bytes_per_step": int(qh.numel() * qh.element_size() + qsh.numel() * 4 + n_len * 4),
-               "d2h_bytes_per_step": int(ih.numel() * 8 + dh.numel() * 4),
-               "ms_per_step": ems / args.steps}
+        e2e = {"value": mq_total / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": ems / args.steps}
 
     if rank != 0:
-        if world > 1:
+        if dist.is_initialized():
             dist.destroy_process_group()
         return
 
     # ---- secondary: the paper's two-level path (postings in HBM), for a4's HBM figure
     two = None
-    if args.two_level_steps > 0 and not args.two_level:
+    if args.two_level_steps > 0 and not args.two_level and args.config != "C4":
         op2 = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=1)
         st2 = pkg.KnnStats()
-        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, st2, op2)
+        R.step(st2, op2)
         ph2 = {f: 0.0 for f in phase}
         acc2 = {f: 0 for f in acc}
         for _ in range(args.two_level_steps):
-            pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, k, ids, dd, st2, op2)
+            R.step(st2, op2)
             for f in ph2:
                 ph2[f] += getattr(st2, f)
             for f in acc2:
@@ -367,12 +458,14 @@ def main():
         cell_peak = 148 * 42.7 * sm_mhz * 1e6
         alu_src = "issue-rate estimate (no alu_peaks.json) x median SM clock"
     n_sw = wl.D - wl.window + 1
+    if R.sharded_window:
+        pts = [R.index_points] * wl.n_mq
+    else:
+        pts = [int(wl.offsets[s + 1] - wl.offsets[s]) for s in wl.query_sensor.tolist()]
     # algorithmic work: (SW, DW, j) term pairs = n_sw * n_dw * w per MQ
-    win_terms = n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window * wl.window
-                           for s in wl.query_sensor.tolist())
-    post_bytes_step = 8 * n_sw * sum((wl.offsets[s + 1] - wl.offsets[s]) // wl.window
-                                     for s in wl.query_sensor.tolist())
-    lb_bytes_step = 4 * n_len * sum(int(wl.offsets[s + 1] - wl.offsets[s]) for s in wl.query_sensor.tolist())
+    win_terms = n_sw * sum(p // wl.window * wl.window for p in pts)
+    post_bytes_step = 8 * n_sw * sum(p // wl.window for p in pts)
+    lb_bytes_step = 4 * n_len * sum(pts)
 
     def rooflines(ph, ac, nsteps, fused):
         ks = {}
@@ -382,7 +475,7 @@ def main():
             ks["lb_fused" if fused else "window_lb_a3"] = {
                 "bound": "alu", "achieved": rate / 1e12, "peak": term_peak / 1e12,
                 "unit": "T term-pairs/s", "frac": rate / term_peak, "ms": win_s * 1e3,
-                "algorithmic_per_launch": "%d (SW,DW,j) term pairs x MQs in the chunk" % (win_terms // wl.n_mq)}
+                "algorithmic_per_mq": "%d (SW,DW,j) term pairs" % (win_terms // wl.n_mq)}
         gs_s = ph["ns_group_scan"] / 1e9 / nsteps
         if not fused and gs_s > 0:
             byts = post_bytes_step + lb_bytes_step
@@ -424,15 +517,18 @@ def main():
         v, cores, dt, sample = oracle_sample(wl, args.oracle_seconds)
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
 
+    par = {"C2": "dp%d (independent MQ batches)" % world, "C3": "sensor sharding x%d" % world,
+           "C5": "sensor sharding x%d" % world, "C4": "window-range sharding x%d + NCCL all-gather merge" % world}
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": args.dtype if args.dtype == "f32" else "i16->int32",
+        "scaling": scaling, "vs_baseline": None, "dtype": args.dtype if args.dtype == "f32" else "i16->int32",
         "data": "synthetic",
-        "config": {"workload": cfg_name, "master_queries_per_step_per_gpu": wl.n_mq, "item_queries": wl.lengths,
-                   "k": k, "window": wl.window, "band": wl.band, "series_points": int(len(wl.series)),
-                   "parallelism": "dp%d (independent MQ batches)" % world,
-                   "l2": "inputs larger than L2 (posting lists %.0f MB per MQ)" % (8 * n_sw * (len(wl.series) // wl.window) / 1e6)},
+        "config": {"workload": cfg_name, "master_queries_per_step": mq_total / args.steps,
+                   "item_queries": wl.lengths, "k": k, "window": wl.window, "band": wl.band,
+                   "indexed_points_rank0": int(R.index_points), "parallelism": par[args.config],
+                   "l2": "inputs larger than L2 (LB_w %.0f MB per step; two-level posting lists %.0f MB per MQ)"
+                         % (lb_bytes_step / 1e6, post_bytes_step / max(1, wl.n_mq) / 1e6)},
         "item_queries_per_s": value * n_len,
         "dtw_cells_per_s": acc["dtw_cells"] / steps / (ms_max / 1000.0 / args.steps) * world,
         "bf_equiv_cells_per_s": acc["bf_cells"] / steps / (ms_max / 1000.0 / args.steps) * world,
@@ -449,7 +545,7 @@ def main():
         "e2e": e2e,
     }
     print(json.dumps(out, default=lambda o: o.item() if hasattr(o, "item") else str(o)))
-    if world > 1:
+    if dist.is_initialized():
         dist.destroy_process_group()
 
 
