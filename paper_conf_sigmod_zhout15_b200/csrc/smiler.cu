@@ -24,6 +24,9 @@
 
 using namespace smiler;
 
+constexpr int kTauMult = 16;  // tau-set size target, multiples of k (R8 reading)
+constexpr int kTauEMax = 8;   // candidates per tau unit (CTA or warp)
+
 // ---------------------------------------------------------------------------
 // errors
 // ---------------------------------------------------------------------------
@@ -655,7 +658,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         int E = 0;
         if (!lb_only && !o.no_prune) {
             const int umin = nblk_min * units_per_blk;
-            E = std::min(8, std::max(1, (2 * pl.k + umin - 1) / umin));
+            const int mult = o.reserved[2] > 0 ? o.reserved[2] : kTauMult;  // tau set ~ mult * k per IQ
+            E = std::min(kTauEMax, std::max(1, (mult * pl.k + umin - 1) / umin));
         }
         const int LT = std::max(1, nblk_max * units_per_blk * E);
         QParams P;
