@@ -230,7 +230,7 @@ int main(int argc, char **argv) {
     int dev = 0, sms = 0;
     cudaSetDevice(dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const int per_sm = 8;  // 64 warps per SM
+    const int per_sm = argc > 2 ? atoi(argv[2]) : 8;  // CTAs of 256 threads per SM (8 = 64 warps)
     const float min_ms = argc > 1 ? (float)atof(argv[1]) : 400.f;
     // interleaved, sustained: each mix twice, keep the second (steady clock)
     Rate r[6];
@@ -244,7 +244,7 @@ int main(int argc, char **argv) {
     }
     cudaError_t e = cudaGetLastError();
     const char *names[6] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32"};
-    printf("{\"sms\": %d, \"sustained_ms_per_mix\": %.0f", sms, min_ms);
+    printf("{\"sms\": %d, \"ctas_per_sm\": %d, \"sustained_ms_per_mix\": %.0f", sms, per_sm, min_ms);
     for (int i = 0; i < 6; i++)
         printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e", names[i], r[i].per_clk_sm,
                names[i], r[i].mhz, names[i], r[i].per_s);

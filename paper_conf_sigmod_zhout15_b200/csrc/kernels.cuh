@@ -255,7 +255,7 @@ __global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, i
 // grid (tiles, segments); block-aggregated compaction, one atomic per CTA.
 // ---------------------------------------------------------------------------
 constexpr int kFiltThreads = 256;
-constexpr int kFiltItems = 8;
+constexpr int kFiltItems = 32;
 
 template <typename S>
 __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<S>::V *lb,

@@ -517,7 +517,8 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     }
     if (P.E <= 0) return;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + ((int64_t)blockIdx.x * nw + warp) * P.E;
+    const int unit = blockIdx.x * nw + warp;  // tau units are warps
+    int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)unit * P.E;
     uint32_t taken = 0;
     for (int e = 0; e < P.E; e++) {
         uint64_t best = kKeyMax;

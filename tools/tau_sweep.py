@@ -21,7 +21,7 @@ nl = len(wl.lengths)
 ids = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int64, device=dev)
 dd = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int32 if dtype == "i16" else torch.float32, device=dev)
 ref = None
-for mult in (8, 16, 32):
+for mult in (8, 16, 32, 64, 128):
     op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=0)
     op.reserved[2] = mult
     s = pkg.KnnStats()
