@@ -502,6 +502,18 @@ def main():
     rf = dict(kernels[dom])
     rf["kernel"] = dom
     rf["traffic"] = None
+    tfile = os.path.join(ROOT, "profiles", "r01", "prof_c2_traffic_per_mq.json")
+    if args.config == "C2" and os.path.exists(tfile):
+        tname = {"lb_fused": "lb_diag_kernel<%s, %d>", "window_lb_a3": "window_lb_kernel<%s, %d>",
+                 "group_scan_a4": "group_scan_kernel<%s, %d>"}.get(dom)
+        tmap = json.load(open(tfile))
+        if tname:
+            key = tname % ("float" if args.dtype == "f32" else "short", wl.window)
+            if key in tmap:
+                # DRAM bytes per launch = ncu per-MQ traffic x MQs per launch (one chunk per step)
+                rf["traffic"] = tmap[key] * wl.n_mq
+                rf["traffic_source"] = "profiles/r01/prof_c2_traffic_per_mq.json (ncu --set full, %s)" % key
+                rf["algorithmic_bytes_per_launch"] = lb_bytes_step
     rf["peak_source"] = ("MEASURED_PEAKS.json hbm_gbs (%s)" % peak_kind if rf["bound"] == "hbm" else alu_src)
     two_level = None
     if two is not None:
