@@ -96,6 +96,39 @@ __global__ void __launch_bounds__(kThreads) lbterm_f32_mix(float *out, long long
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
+// LB term pair as the kernels compute it: per term FADD, FADD, FMNMX3, FFMA
+// (max(v - U, L - v, 0)^2, bit-identical to the clamp form).
+__global__ void __launch_bounds__(kThreads) lbterm_max3_mix(float *out, long long *cyc, float q0) {
+    // EQ term: series value v vs query envelope (q + 0.5, q - 0.5);
+    // EC term: query value q vs series envelope (U2, L2): no shared subexpressions
+    float acc[kChains], v[kChains], U2[kChains], L2[kChains];
+#pragma unroll
+    for (int i = 0; i < kChains; i++) {
+        acc[i] = 0;
+        v[i] = i * 0.3f - 1.0f;
+        U2[i] = 0.5f + threadIdx.x * 1e-3f + i;
+        L2[i] = -0.5f - i;
+    }
+    long long t0 = clock64();
+    for (int it = 0; it < kIters; it++) {
+        const float q = q0 + it * 1e-4f;
+        const float uq = q + 0.5f, lq = q - 0.5f;
+#pragma unroll
+        for (int i = 0; i < kChains; i++) {
+            float m1 = fmaxf(fmaxf(v[i] - uq, lq - v[i]), 0.0f);
+            acc[i] = fmaf(m1, m1, acc[i]);
+            float m2 = fmaxf(fmaxf(q - U2[i], L2[i] - q), 0.0f);
+            acc[i] = fmaf(m2, m2, acc[i]);
+        }
+    }
+    long long t1 = clock64();
+    float s = 0;
+#pragma unroll
+    for (int i = 0; i < kChains; i++) s += acc[i];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+}
+
 __global__ void __launch_bounds__(kThreads) lbterm_i32_mix(int *out, long long *cyc, int q0) {
     int acc[kChains], v[kChains];
     int U = 500 + threadIdx.x, L = -500;
@@ -233,7 +266,7 @@ int main(int argc, char **argv) {
     const int per_sm = argc > 2 ? atoi(argv[2]) : 8;  // CTAs of 256 threads per SM (8 = 64 warps)
     const float min_ms = argc > 1 ? (float)atof(argv[1]) : 400.f;
     // interleaved, sustained: each mix twice, keep the second (steady clock)
-    Rate r[6];
+    Rate r[7];
     for (int pass = 0; pass < 2; pass++) {
         r[0] = run(dtw_f32_mix, 1.0f, sms, per_sm, 1.0, min_ms);
         r[1] = run(dtw_f32x2_mix, 1.0f, sms, per_sm, 2.0, min_ms);
@@ -241,17 +274,19 @@ int main(int argc, char **argv) {
         r[3] = run(lbterm_f32x2_mix, 0.1f, sms, per_sm, 1.0, min_ms);
         r[4] = run(dtw_i32_mix, 1, sms, per_sm, 1.0, min_ms);
         r[5] = run(lbterm_i32_mix, 1, sms, per_sm, 1.0, min_ms);
+        r[6] = run(lbterm_max3_mix, 0.1f, sms, per_sm, 1.0, min_ms);
     }
     cudaError_t e = cudaGetLastError();
-    const char *names[6] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32"};
+    const char *names[7] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32",
+                            "lbterm_max3"};
     printf("{\"sms\": %d, \"ctas_per_sm\": %d, \"sustained_ms_per_mix\": %.0f", sms, per_sm, min_ms);
-    for (int i = 0; i < 6; i++)
+    for (int i = 0; i < 7; i++)
         printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e", names[i], r[i].per_clk_sm,
                names[i], r[i].mhz, names[i], r[i].per_s);
     printf(", \"note\": \"units per SM per SM clock and per second over back-to-back full waves (8 CTAs x 256 threads "
            "per SM, 8 independent chains per thread), sustained for the stated time; dtw cell = FADD+FMNMX3+FFMA (f32), "
            "f32x2 = FADD2+2 FMNMX3+FFMA2 per 2 cells, i32 = IADD+VIMNMX3+IMAD(+LOP); lbterm = one (SW,DW,j) EQ+EC "
-           "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2\", \"cuda\": \"%s\"}\n",
+           "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), lbterm_max3 = 2x(FADD,FADD,FMNMX3,FFMA) (the kernels' form), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2\", \"cuda\": \"%s\"}\n",
            cudaGetErrorString(e));
     return e == cudaSuccess ? 0 : 1;
 }

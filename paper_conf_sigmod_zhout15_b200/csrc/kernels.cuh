@@ -18,8 +18,10 @@ template <> __device__ __forceinline__ uint32_t key_bits(int32_t v) { return (ui
 
 // e(v; U, L) of Eq. 26 accumulated: (v - clamp(v, L, U))^2.
 __device__ __forceinline__ void lb_term(float v, float U, float L, float &acc) {
-    float dd = v - fminf(fmaxf(v, L), U);
-    acc = fmaf(dd, dd, acc);
+    // (v - clamp(v, L, U))^2 = max(v - U, L - v, 0)^2 (U >= L): bit-identical,
+    // one FMNMX3 on the ALU pipe and FADD, FADD, FFMA on the FMA pipe
+    const float m = fmaxf(fmaxf(v - U, L - v), 0.0f);
+    acc = fmaf(m, m, acc);
 }
 __device__ __forceinline__ void lb_term(int32_t v, int32_t U, int32_t L, int32_t &acc) {
     int32_t dd = v - min(max(v, L), U);
