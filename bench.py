@@ -127,18 +127,23 @@ def rank_workload(cfg: str, dtype: str, rank: int, world: int, mq_per_step: int)
         # sensors round-robin over ranks; every MQ runs where its sensor lives
         _, ns, N, periods, lens, k, w, band, mqs = synth.CONFIGS[cfg]
         mine = list(range(rank, ns, world))
-        parts, qs, qsens, offs = [], [], [], [0]
+        parts, qs, qsens, offs, tails, qoff = [], [], [], [0], [], []
         D = lens[-1]
+        H = D + 7 * mqs + synth.STEP_MAX + 1   # same history for every continuous step
         for li, s in enumerate(mine):
-            z = synth.sensor_series(synth.CONFIGS[cfg][0], s, N, D + 7 * mqs + 1, periods[s % len(periods)])
+            z = synth.sensor_series(synth.CONFIGS[cfg][0], s, N, H, periods[s % len(periods)])
             x = synth.quantise(z, dtype)
             parts.append(x[:N])
             offs.append(offs[-1] + N)
+            tails.append(x[N:])
             for j in range(mqs):
                 qs.append(x[N + 7 * j:N + 7 * j + D])
                 qsens.append(li)
-        return synth.Workload(cfg, dtype, np.concatenate(parts), np.asarray(offs, np.int64),
-                              np.ascontiguousarray(np.stack(qs)), np.asarray(qsens, np.int32), lens, k, w, band)
+                qoff.append(7 * j)
+        wl = synth.Workload(cfg, dtype, np.concatenate(parts), np.asarray(offs, np.int64),
+                            np.ascontiguousarray(np.stack(qs)), np.asarray(qsens, np.int32), lens, k, w, band)
+        wl.tails, wl.qoff = tails, np.asarray(qoff, np.int64)
+        return wl
     if cfg == "C4":
         # one long series; every rank holds the same MQ batch and its own window range
         return synth.make_workload("C4", dtype, mq_per_sensor=mq_per_step)
@@ -228,6 +233,27 @@ class Runner:
         self.ids = torch.empty((wl.n_mq, self.n_len, self.k), dtype=torch.int64, device=dev)
         self.dd = torch.empty((wl.n_mq, self.n_len, self.k), dtype=vt, device=dev)
         self.op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=int(args.two_level))
+        self.op.reserved[2] = args.tau_mult
+        self.op_fast = pkg.KnnOpts(no_prune=0, timing=0, mq_chunk=0, two_level=int(args.two_level))
+        self.op_fast.reserved[2] = args.tau_mult
+        # C5 is a continuous prediction stream: every step is one tick of all
+        # streams (each MQ advances one point); after the first tick the previous
+        # tick's neighbours seed the thresholds (smiler_knn_step)
+        self.continuous = cfg == "C5" and not args.no_continuous
+        self.tick = 0
+        if self.continuous:
+            D = wl.D
+            T = 2 * args.steps + args.warmup + 12
+            idx_s = np.asarray(wl.query_sensor)
+            cols = wl.qoff[:, None] + np.arange(D)[None, :]
+            qt = np.empty((T, wl.n_mq, D), wl.queries.dtype)
+            tails = np.stack([wl.tails[s_] for s_ in range(len(wl.tails))])
+            for s_ in range(T):
+                qt[s_] = tails[idx_s[:, None], cols + s_]
+            self.qticks_host = torch.from_numpy(qt).pin_memory()
+            self.qticks = self.qticks_host.to(dev)
+            self.ids2 = torch.empty_like(self.ids)
+            self.have_prev = False
 
     def mq_per_step(self):
         """Master queries completed per step on this rank (for the value)."""
@@ -243,8 +269,20 @@ class Runner:
 
     def step(self, stats=None, opts=None):
         pkg = self.pkg
-        pkg.smiler_knn(self.idx.handle, self.qd, self.qs, self.wl.lengths, self.k, self.ids, self.dd, stats,
-                       opts if opts is not None else (self.op if stats is not None else None))
+        op = opts if opts is not None else (self.op if stats is not None else self.op_fast)
+        if self.continuous:
+            q = self.qticks[self.tick % self.qticks.shape[0]]
+            self.tick += 1
+            if self.have_prev:
+                pkg.smiler_knn_step(self.idx.handle, q, self.qs, self.wl.lengths, self.k, self.ids, 1,
+                                    self.ids2, self.dd, stats, op)
+                self.ids, self.ids2 = self.ids2, self.ids
+            else:
+                pkg.smiler_knn(self.idx.handle, q, self.qs, self.wl.lengths, self.k, self.ids, self.dd,
+                               stats, op)
+                self.have_prev = True
+            return
+        pkg.smiler_knn(self.idx.handle, self.qd, self.qs, self.wl.lengths, self.k, self.ids, self.dd, stats, op)
         if self.sharded_window:
             with self.torch.cuda.stream(self.stream):
                 self._merge(self.ids, self.dd)
@@ -260,6 +298,18 @@ class Runner:
 
     def step_e2e(self):
         pkg, torch = self.pkg, self.torch
+        if self.continuous:
+            q = self.qticks_host[self.tick % self.qticks_host.shape[0]]
+            self.tick += 1
+            ih = self.ih.view(self.wl.n_mq, self.n_len, self.k)
+            dh = self.dh.view(self.wl.n_mq, self.n_len, self.k)
+            if not hasattr(self, "prev_h"):
+                self.prev_h = torch.empty_like(ih).pin_memory()
+                pkg.smiler_knn(self.idx.handle, q, self.qs, self.wl.lengths, self.k, ih, dh)
+            else:
+                pkg.smiler_knn_step(self.idx.handle, q, self.qs, self.wl.lengths, self.k, self.prev_h, 1, ih, dh)
+            self.prev_h.copy_(ih)
+            return
         if not self.sharded_window:
             pkg.smiler_knn(self.idx.handle, self.qh, self.qs, self.wl.lengths, self.k,
                            self.ih.view(self.wl.n_mq, self.n_len, self.k), self.dh.view(self.wl.n_mq, self.n_len,
@@ -286,6 +336,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--oracle-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-continuous", action="store_true", help="C5: independent ticks (no smiler_knn_step)")
+    ap.add_argument("--tau-mult", type=int, default=0, help="tau-set size (x k per item query; -1 = none, 0 = default)")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--two-level", action="store_true", help="time the paper's two-level path (a3 -> HBM -> a4)")
     ap.add_argument("--two-level-steps", type=int, default=3,

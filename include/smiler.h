@@ -159,6 +159,25 @@ SMILER_API int smiler_knn_ex(smiler_index *idx, const void *queries, const int32
                   void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts);
 
 /*
+ * smiler_knn_step -- one step of the Continuous Suffix kNN Search (Def. 4.1,
+ * "from time t to time t+1 ... appending the latest observed point into MQ
+ * and delete the oldest point") for a batch of master-query
+ * streams.  Same arguments and results as smiler_knn, plus:
+ * prev_ids      [n_mq][n_len][k] int64 (host or device): the ids this call's
+ *               streams received at their previous step (same lengths, same k).
+ * shift         points each stream advanced since then (1 per step, >= 0).
+ * The threshold of every item query comes from the paper's second method
+ * (reading R9): the previous k neighbours, shifted by `shift`,
+ * re-scored against the new item query; tau_i = the largest of their keys.
+ * Neighbours that fall outside the series make tau_i = +inf (no pruning).
+ * Results are the exact kNN regardless of prev_ids' quality.
+ */
+SMILER_API int smiler_knn_step(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                               int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k,
+                               const int64_t *prev_ids, int32_t shift, int64_t *ids, void *dists,
+                               smiler_knn_stats *stats, const smiler_knn_opts *opts);
+
+/*
  * smiler_merge_topk -- final selection over G per-shard top-k lists (a9,
  * SURVEY §8(e)); called after an all-gather of the shards' (ids, dists).
  * ids_in [G][rows][k] int64, dists_in [G][rows][k] int32/float (dtype);

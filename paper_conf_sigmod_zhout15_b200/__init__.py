@@ -8,8 +8,8 @@ process groups.
 """
 from .smiler import (Index, KnnOpts, KnnStats, SmilerError, smiler_abi_version, smiler_dtw,  # noqa: F401
                      smiler_free, smiler_index_build, smiler_index_build_shard, smiler_index_envelope,
-                     smiler_knn, smiler_lower_bounds, smiler_merge_topk)
+                     smiler_knn, smiler_knn_step, smiler_lower_bounds, smiler_merge_topk)
 
 __all__ = ["Index", "KnnOpts", "KnnStats", "SmilerError", "smiler_abi_version", "smiler_dtw", "smiler_free",
-           "smiler_index_build", "smiler_index_build_shard", "smiler_index_envelope", "smiler_knn",
+           "smiler_index_build", "smiler_index_build_shard", "smiler_index_envelope", "smiler_knn", "smiler_knn_step",
            "smiler_lower_bounds", "smiler_merge_topk"]

@@ -233,12 +233,46 @@ __global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, i
     using V = typename Tr<S>::V;
     __shared__ int s_hist[256];
     __shared__ uint64_t s_b[2];
+    __shared__ uint64_t s_keys[kSortCap];
+    __shared__ int s_scan[32];
     const int seg = blockIdx.x;
-    const uint64_t kth = block_radix_kth(tauk + (int64_t)seg * LT, LT, k, s_hist, s_b);
+    const uint64_t *src = tauk + (int64_t)seg * LT;
+    uint64_t kth;
+    if (LT <= kSortCap) {
+        // sort, then the k-th DISTINCT key: the tau list may hold a candidate twice
+        // (a tile candidate that is also a shifted previous neighbour), and a
+        // duplicate must not count twice (k distinct candidates at or below tau)
+        int n2 = 1;
+        while (n2 < LT) n2 <<= 1;
+        for (int x = threadIdx.x; x < n2; x += blockDim.x) s_keys[x] = x < LT ? src[x] : kKeyMax;
+        bitonic_sort_smem(s_keys, n2);
+        const int per = (n2 + blockDim.x - 1) / blockDim.x;
+        const int x0 = threadIdx.x * per;
+        int cnt = 0;
+        for (int x = x0; x < min(x0 + per, n2); x++)
+            cnt += (s_keys[x] != kKeyMax && (x == 0 || s_keys[x] != s_keys[x - 1]));
+        int total;
+        int before = block_excl_scan(cnt, s_scan, &total);
+        if (threadIdx.x == 0) s_b[0] = kKeyMax;
+        __syncthreads();
+        if (total >= k) {
+            for (int x = x0; x < min(x0 + per, n2); x++) {
+                const bool first = s_keys[x] != kKeyMax && (x == 0 || s_keys[x] != s_keys[x - 1]);
+                if (first) {
+                    if (before == k - 1) s_b[0] = s_keys[x];
+                    before++;
+                }
+            }
+        }
+        __syncthreads();
+        kth = s_b[0];
+    } else {
+        kth = block_radix_kth(src, LT, k, s_hist, s_b);  // tile candidates only: unique
+    }
     if (threadIdx.x == 0) {
         tau_key[seg] = kth;
         if (kth == kKeyMax) {
-            thr[seg] = sizeof(V) == 4 && std::is_same<V, float>::value ? 0x7f800000u : 0x7FFFFFFFu;
+            thr[seg] = std::is_same<V, float>::value ? 0x7f800000u : 0x7FFFFFFFu;
         } else {
             uint32_t db = (uint32_t)(kth >> 32);
             if constexpr (std::is_same<V, float>::value) {
@@ -436,6 +470,24 @@ __global__ void __launch_bounds__(512) merge_topk_kernel(const int64_t *ids_in, 
             const uint32_t db = (uint32_t)(key >> 32);
             d_out[o] = *reinterpret_cast<const V *>(&db);
         }
+    }
+}
+
+// Continuous step (reading R9): the previous step's k neighbours
+// of each stream, shifted by the points the stream advanced, join the tau list
+// at [LTt, LTt + k) of their segment (invalid -> -1).
+__global__ void prev_tau_kernel(const int64_t *prev, int shift, const MQMeta *meta, const QParams P, int LTt,
+                                int32_t *tauc) {
+    const int seg = blockIdx.x;
+    const int mq = seg / P.n_len, i = seg % P.n_len;
+    const MQMeta m = meta[mq];
+    const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t te = min(m.t_hi, m.n - P.len[i] + 1);
+    for (int j = threadIdx.x; j < P.k; j += blockDim.x) {
+        const int64_t id = prev[(int64_t)seg * P.k + j];
+        int64_t t = id >= 0 ? id - m.origin + shift : -1;
+        if (t < tb || t >= te) t = -1;
+        tauc[(int64_t)seg * P.LT + LTt + j] = (int32_t)t;
     }
 }
 

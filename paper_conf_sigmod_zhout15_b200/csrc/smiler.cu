@@ -25,6 +25,7 @@
 using namespace smiler;
 
 constexpr int kTauMult = 16;  // tau-set size target, multiples of k (R8 reading)
+constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previous neighbours)
 constexpr int kTauEMax = 8;   // candidates per tau unit (CTA or warp)
 
 // ---------------------------------------------------------------------------
@@ -125,7 +126,7 @@ struct smiler_index {
     int num_sms = 148;
     // workspace
     DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, tauk, taukey, thr, scount, fcount,
-        taskoff, out_ids, out_d, tmp;
+        taskoff, out_ids, out_d, tmp, tmp2;
     std::vector<cudaEvent_t> events;
     size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
     // pinned staging ring for per-chunk metadata (async H2D without host sync)
@@ -275,7 +276,7 @@ static void destroy(smiler_index *idx) {
     DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
                       &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->tauk,
                       &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
-                      &idx->out_ids, &idx->out_d,  &idx->tmp};
+                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
     for (int s = 0; s < 2; s++) {
@@ -523,7 +524,8 @@ template <typename S>
 static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query_sensor_in,
                     int32_t n_mq, const int32_t *lengths_in, int32_t n_len, int32_t k, int64_t *ids,
                     void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts,
-                    bool lb_only, void *post_out, void *lb_out) {
+                    bool lb_only, void *post_out, void *lb_out, const int64_t *prev_ids = nullptr,
+                    int shift = 0) {
     using V = typename Tr<S>::V;
     using V2 = typename Tr<S>::V2;
     using V4 = typename Tr<S>::V4;
@@ -656,12 +658,22 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // tau-set units: CTAs (block epilogue) or warps (diagonal kernel's warp epilogue)
         const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32 : 1;
         int E = 0;
+        const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         if (!lb_only && !o.no_prune) {
             const int umin = nblk_min * units_per_blk;
-            const int mult = o.reserved[2] > 0 ? o.reserved[2] : kTauMult;  // tau set ~ mult * k per IQ
-            E = std::min(kTauEMax, std::max(1, (mult * pl.k + umin - 1) / umin));
+            // tau set ~ mult * k tile candidates per IQ (plus k shifted previous
+            // neighbours in a continuous step, where a smaller tile set suffices)
+            int mult = use_prev ? kTauMultCont : kTauMult;
+            if (o.reserved[2] > 0) mult = o.reserved[2];
+            if (o.reserved[2] < 0) mult = 0;
+            E = mult > 0 ? std::min(kTauEMax, std::max(1, (mult * pl.k + umin - 1) / umin)) : 0;
+            // with previous neighbours the tau list must fit the sorting (dedupe) path
+            while (use_prev && E > 0 && nblk_max * units_per_blk * E + pl.k > kSortCap) E--;
         }
-        const int LT = std::max(1, nblk_max * units_per_blk * E);
+        // tau list per segment: the LB kernel's tile candidates [0, LTt), then (continuous
+        // step, P:1452-1458 / R9) the previous step's k neighbours shifted by `shift`
+        const int LTt = nblk_max * units_per_blk * E;
+        const int LT = std::max(1, LTt + (use_prev ? pl.k : 0));
         QParams P;
         memset(&P, 0, sizeof(P));
         P.D = D;
@@ -802,6 +814,17 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         CU(cudaMemsetAsync(fcount, 0, 4 * (size_t)nseg, idx->stream));
         int32_t *taskoff = idx->taskoff.as<int32_t>();
         // ---- a5: tau ------------------------------------------------------
+        if (use_prev) {
+            const int64_t *pv = prev_ids + (size_t)c0 * nl * pl.k;
+            if (!is_device_ptr(prev_ids)) {
+                TRY(idx->tmp2.ensure(8 * (size_t)nseg * pl.k));
+                CU(cudaMemcpyAsync(idx->tmp2.p, pv, 8 * (size_t)nseg * pl.k, cudaMemcpyHostToDevice, idx->stream));
+                pv = idx->tmp2.as<int64_t>();
+            }
+            prev_tau_kernel<<<nseg, 128, 0, idx->stream>>>(pv, shift, d_meta, P, LTt, idx->tauc.as<int32_t>());
+            CHECK_LAUNCH();
+            launches++;
+        }
         if (!o.no_prune) {
             for (int i = 0; i < nl; i++) {
                 TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
@@ -914,6 +937,20 @@ extern "C" int smiler_knn(smiler_index *idx, const void *queries, const int32_t 
                           int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
                           void *dists, smiler_knn_stats *stats) {
     return smiler_knn_ex(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, nullptr);
+}
+
+extern "C" int smiler_knn_step(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                               int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k,
+                               const int64_t *prev_ids, int32_t shift, int64_t *ids, void *dists,
+                               smiler_knn_stats *stats, const smiler_knn_opts *opts) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!prev_ids) return fail(SMILER_EINVAL, "prev_ids is NULL (use smiler_knn for a first step)");
+    if (shift < 0) return fail(SMILER_EINVAL, "shift must be >= 0");
+    if (idx->dtype == SMILER_I16)
+        return knn_impl<int16_t>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, opts,
+                                 false, nullptr, nullptr, prev_ids, shift);
+    return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, opts, false,
+                           nullptr, nullptr, prev_ids, shift);
 }
 
 extern "C" int smiler_lower_bounds(smiler_index *idx, const void *queries, const int32_t *query_sensor,

@@ -66,6 +66,7 @@ def lib():
                                                ctypes.POINTER(P)]
         L.smiler_knn.argtypes = [P, P, P, i32, P, i32, i32, P, P, P]
         L.smiler_knn_ex.argtypes = [P, P, P, i32, P, i32, i32, P, P, P, P]
+        L.smiler_knn_step.argtypes = [P, P, P, i32, P, i32, i32, P, i32, P, P, P, P]
         L.smiler_merge_topk.argtypes = [P, P, i32, i32, i32, i32, P, P, i32, P]
         L.smiler_index_envelope.argtypes = [P, i32, i32, P, P]
         L.smiler_lower_bounds.argtypes = [P, P, P, i32, P, i32, P, P]
@@ -74,7 +75,7 @@ def lib():
         L.smiler_free.restype = None
         L.smiler_last_error.restype = ctypes.c_char_p
         L.smiler_abi_version.restype = i32
-        for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex",
+        for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex", "smiler_knn_step",
                   "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_dtw"):
             getattr(L, f).restype = i32
         _lib = L
@@ -155,6 +156,20 @@ def smiler_knn(handle: int, queries, query_sensor, lengths, k: int, ids, dists,
                                ctypes.byref(opts) if opts is not None else None))
 
 
+def smiler_knn_step(handle: int, queries, query_sensor, lengths, k: int, prev_ids, shift: int, ids, dists,
+                    stats: Optional[KnnStats] = None, opts: Optional[KnnOpts] = None) -> None:
+    """One continuous step: like smiler_knn, with the previous step's ids of the
+    same streams seeding each item query's threshold."""
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    qs = None if query_sensor is None else (
+        query_sensor if hasattr(query_sensor, "data_ptr") else np.ascontiguousarray(query_sensor, np.int32))
+    n_mq = int(queries.shape[0])
+    _check("smiler_knn_step",
+           lib().smiler_knn_step(handle, _ptr(queries), _ptr(qs), n_mq, _ptr(lens), len(lens), k, _ptr(prev_ids),
+                                 shift, _ptr(ids), _ptr(dists), ctypes.byref(stats) if stats is not None else None,
+                                 ctypes.byref(opts) if opts is not None else None))
+
+
 def smiler_merge_topk(ids_in, dists_in, G: int, rows: int, k: int, ids_out, dists_out,
                       device: int = 0, stream=None) -> None:
     _check("smiler_merge_topk",
@@ -223,6 +238,19 @@ class Index:
         st = KnnStats() if stats else None
         op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level))
         smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
+        if stats:
+            return ids, dists, st.as_dict()
+        return ids, dists
+
+    def knn_step(self, queries, lengths: Sequence[int], k: int, prev_ids, shift: int = 1, query_sensor=None,
+                 stats: bool = False, timing: bool = False):
+        n_mq = queries.shape[0]
+        ids = np.empty((n_mq, len(lengths), k), np.int64)
+        dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
+        st = KnnStats() if stats else None
+        op = KnnOpts(timing=int(timing))
+        smiler_knn_step(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
+                        np.ascontiguousarray(prev_ids, dtype=np.int64), shift, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()
         return ids, dists

@@ -34,6 +34,7 @@ import numpy as np
 I16_SCALE = 128.0
 I16_MAX = 1023
 SEED_BASE = 20150531
+STEP_MAX = 4096  # continuous steps supported by make_workload
 
 
 def sensor_series(config_id: int, sensor: int, n: int, h: int, period: int) -> np.ndarray:
@@ -141,7 +142,11 @@ def make_workload(name: str, dtype: str = "i16", *, n: Optional[int] = None,
     bd = band if band is not None else bd
     D = lens[-1]
     spread = 1 if consecutive else 7
-    H = D + spread * mqs + step + 1
+    # the tail length does not depend on `step`, so every continuous step of a
+    # workload sees the same indexed history (noise draws follow the walk's)
+    if not 0 <= step < STEP_MAX:
+        raise ValueError("step must be in [0, %d)" % STEP_MAX)
+    H = D + spread * mqs + STEP_MAX + 1
     parts, queries, qs = [], [], []
     offsets = [0]
     for s in range(ns):

@@ -351,3 +351,37 @@ def test_c2_full_size_sampled(pkg, orc, dtype):
                 for t, v in zip(ts.tolist(), g.tolist()):
                     assert (v, t) >= kth or t in ids[j, i]
     assert st["survivors"] < st["candidates"]
+
+
+# ---------------------------------------------------------------------------
+# continuous steps (Def. 4.1; threshold method 2, P:1452-1458 / R9)
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_continuous_steps(pkg, orc, dtype):
+    kw = dict(n=12001, n_sensors=3, mq_per_sensor=2)
+    wl = synth.make_workload("C5", dtype, step=0, **kw)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        ids, dists = idx.knn(wl.queries, wl.lengths, wl.k, wl.query_sensor)
+        for s in range(1, 4):
+            ws = synth.make_workload("C5", dtype, step=s, **kw)
+            assert (ws.series == wl.series).all()
+            ids, dists, st = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 1, ws.query_sensor, stats=True)
+            # the k previous neighbours are part of every item query's tau list
+            assert st["tau_verified"] >= ws.n_mq * len(ws.lengths) * ws.k
+            if dtype == "i16":
+                oid, od = orc.knn(ws, threads=THREADS)
+                np.testing.assert_array_equal(ids, oid)
+                np.testing.assert_array_equal(dists.astype(np.int64), od)
+            else:
+                oid, od = orc.knn(ws, mode="f32", threads=THREADS)
+                np.testing.assert_array_equal(ids, oid)
+                np.testing.assert_array_equal(dists, od)
+        # useless previous neighbours (all padding): tau = +inf, still exact
+        bad = np.full_like(ids, -1)
+        i2, d2 = idx.knn_step(ws.queries, ws.lengths, ws.k, bad, 1, ws.query_sensor)
+        np.testing.assert_array_equal(i2, ids)
+        np.testing.assert_array_equal(d2, dists)
+        # stale neighbours from far away still give a valid (loose) threshold
+        i3, d3 = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 50, ws.query_sensor)
+        np.testing.assert_array_equal(i3, ids)
+        np.testing.assert_array_equal(d3, dists)

@@ -21,12 +21,20 @@ nl = len(wl.lengths)
 ids = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int64, device=dev)
 dd = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int32 if dtype == "i16" else torch.float32, device=dev)
 ref = None
-for mult in (8, 16, 32, 64, 128):
+cont = len(sys.argv) > 3 and sys.argv[3] == "cont"
+prev = None
+for mult in ((-1, 2, 4, 8, 16) if cont else (8, 16, 32, 64, 128)):
     op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=0)
     op.reserved[2] = mult
     s = pkg.KnnStats()
     for it in range(2):
-        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, wl.k, ids, dd, s, op)
+        if cont:
+            if prev is None:
+                prev = torch.empty_like(ids)
+                pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, wl.k, prev, dd)
+            pkg.smiler_knn_step(idx.handle, qd, qs, wl.lengths, wl.k, prev, 0, ids, dd, s, op)
+        else:
+            pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, wl.k, ids, dd, s, op)
     out = (ids.cpu().numpy().copy(), dd.cpu().numpy().copy())
     if ref is None:
         ref = out
