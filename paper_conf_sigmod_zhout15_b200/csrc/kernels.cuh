@@ -23,6 +23,15 @@ __device__ __forceinline__ void lb_term(float v, float U, float L, float &acc) {
     const float m = fmaxf(fmaxf(v - U, L - v), 0.0f);
     acc = fmaf(m, m, acc);
 }
+// clamp form: 2 FMNMX (ALU pipe) + FADD + FFMA (FMA pipe); same value as lb_term
+__device__ __forceinline__ void lb_term_clamp(float v, float U, float L, float &acc) {
+    const float dd = v - fminf(fmaxf(v, L), U);
+    acc = fmaf(dd, dd, acc);
+}
+__device__ __forceinline__ void lb_term_clamp(int32_t v, int32_t U, int32_t L, int32_t &acc) {
+    const int32_t dd = v - min(max(v, L), U);
+    acc += dd * dd;
+}
 __device__ __forceinline__ void lb_term(int32_t v, int32_t U, int32_t L, int32_t &acc) {
     int32_t dd = v - min(max(v, L), U);
     acc += dd * dd;

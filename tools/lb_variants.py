@@ -12,16 +12,23 @@ import paper_conf_sigmod_zhout15_b200 as pkg
 
 dtype = sys.argv[1] if len(sys.argv) > 1 else "f32"
 nmq = int(sys.argv[2]) if len(sys.argv) > 2 else 256
-wl = synth.make_workload("C2", dtype, mq_per_sensor=nmq)
+cfg = os.environ.get("CFG", "C2")
+if cfg == "C2":
+    wl = synth.make_workload("C2", dtype, mq_per_sensor=nmq)
+else:
+    import bench
+    wl = bench.rank_workload(cfg, dtype, 0, 1, nmq)
 dev = torch.device("cuda", 0)
 st = torch.cuda.Stream()
 idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band, stream=st)
 qd = torch.from_numpy(wl.queries).to(dev)
-ids = torch.empty((nmq, 4, wl.k), dtype=torch.int64, device=dev)
-dd = torch.empty((nmq, 4, wl.k), dtype=torch.int32 if dtype == "i16" else torch.float32, device=dev)
+qs = np.ascontiguousarray(wl.query_sensor)
+nl = len(wl.lengths)
+ids = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int64, device=dev)
+dd = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int32 if dtype == "i16" else torch.float32, device=dev)
 ref = None
 variants = [("diag", 0, 0, 0), ("diag_mainonly", 0, 0, 2), ("diag_notau", 0, 0, 3), ("row", 0, 1, 0),
-            ("two_level", 1, 0, 0)]
+            ("two_level", 1, 0, 0), ("unsplit", 0, 2, 0), ("unsplit_mainonly", 0, 2, 2)]
 if len(sys.argv) > 3:
     variants = [v for v in variants if v[0] in sys.argv[3].split(",")]
 for name, tl, res, npr in variants:
@@ -30,7 +37,7 @@ for name, tl, res, npr in variants:
     op.reserved[1] = {2: 1, 3: 2}.get(npr, 0)
     s = pkg.KnnStats()
     for it in range(1 if npr in (1, 3) else 4):
-        pkg.smiler_knn(idx.handle, qd, None, wl.lengths, wl.k, ids, dd, s, op)
+        pkg.smiler_knn(idx.handle, qd, qs, wl.lengths, wl.k, ids, dd, s, op)
     out = (ids.cpu().numpy().copy(), dd.cpu().numpy().copy())
     if ref is None:
         ref = out
