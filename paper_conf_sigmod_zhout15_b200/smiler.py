@@ -15,7 +15,7 @@ from typing import Any, Optional, Sequence, Tuple
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.environ.get("SMILER_LIB_OVERRIDE") or os.path.join(_HERE, "libsmiler.so")  # override: A/B experiments only
+LIB_PATH = os.path.join(_HERE, "libsmiler.so")
 
 SMILER_I16 = 0
 SMILER_F32 = 1
