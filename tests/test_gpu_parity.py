@@ -385,3 +385,91 @@ def test_continuous_steps(pkg, orc, dtype):
         i3, d3 = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 50, ws.query_sensor)
         np.testing.assert_array_equal(i3, ids)
         np.testing.assert_array_equal(d3, dists)
+
+
+# ---------------------------------------------------------------------------
+# more edges: chunking, limits, extreme values
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_forced_chunks_equal_single_chunk(pkg, dtype):
+    wl = synth.make_workload("C5", dtype, n=9001, n_sensors=4, mq_per_sensor=3)
+    a = gpu_knn(pkg, wl)
+    for chunk in (1, 2, 5):
+        b = gpu_knn(pkg, wl, mq_chunk=chunk)
+        np.testing.assert_array_equal(a[0], b[0])
+        np.testing.assert_array_equal(a[1], b[1])
+        c = gpu_knn(pkg, wl, mq_chunk=chunk, two_level=True)
+        np.testing.assert_array_equal(a[0], c[0])
+        np.testing.assert_array_equal(a[1], c[1])
+
+
+def test_limits_long_query_many_lengths_large_k(pkg, orc):
+    """D = 1024 with 16 item queries, k = 1024 (every ABI limit at once, R23)."""
+    lens = [16 * (i + 1) for i in range(15)] + [1024]
+    wl = synth.make_workload("C2", "i16", n=2500, mq_per_sensor=1, lengths=lens, k=1024, window=16, band=0.02)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_extreme_values(pkg, orc, dtype):
+    """Series and queries saturating the i16 range (|x| = 1023): int32 sums near
+    their bound (R17); f32 with the same large values."""
+    rng = np.random.default_rng(17)
+    n, D = 3000, 128
+    base = rng.choice([-1023, 1023], size=n + D).astype(np.int16)
+    if dtype == "f32":
+        base = base.astype(np.float32)
+    wl = synth.Workload("extreme", dtype, np.ascontiguousarray(base[:n]), np.array([0, n], np.int64),
+                        np.ascontiguousarray(base[n:][None, :]), np.array([0], np.int32), [32, 64, 128], 16, 8, 0.1)
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_shards_fractional_band(pkg, orc, dtype):
+    """Window-range shards with a fractional band (rho_max from the longest IQ)."""
+    wl = synth.make_workload("C5", dtype, n=20011, n_sensors=1, mq_per_sensor=2)
+    full_ids, full_d = gpu_knn(pkg, wl)
+    N, D, w = len(wl.series), wl.D, wl.window
+    rho_env = max(wl.rhos())
+    G = 3
+    bounds = [((N * g) // G) // w * w for g in range(G)] + [N]
+    outs_i, outs_d = [], []
+    for g in range(G):
+        t0, t1 = bounds[g], bounds[g + 1]
+        s0 = max(0, t0 - rho_env) // w * w
+        s1 = min(N, t1 + D - 1 + rho_env)
+        with pkg.Index.shard(np.ascontiguousarray(wl.series[s0:s1]), s0, N, t0, t1, w, wl.band) as idx:
+            i_, d_ = idx.knn(wl.queries, wl.lengths, wl.k)
+        outs_i.append(i_)
+        outs_d.append(d_)
+    rows = wl.n_mq * len(wl.lengths)
+    mi = np.empty((rows, wl.k), np.int64)
+    md = np.empty((rows, wl.k), outs_d[0].dtype)
+    pkg.smiler_merge_topk(np.ascontiguousarray(np.stack(outs_i)), np.ascontiguousarray(np.stack(outs_d)), G, rows,
+                          wl.k, mi, md)
+    np.testing.assert_array_equal(mi.reshape(full_ids.shape), full_ids)
+    np.testing.assert_array_equal(md.reshape(full_d.shape), full_d)
+
+
+def test_shard_halo_too_small_is_einval(pkg):
+    wl = synth.make_workload("C4", "i16", n=5000, mq_per_sensor=1)
+    with pkg.Index.shard(np.ascontiguousarray(wl.series[1024:3000]), 1024, 5000, 1024, 2000, 16, 8.0) as idx:
+        with pytest.raises(pkg.SmilerError) as ei:
+            idx.knn(wl.queries, wl.lengths, wl.k)   # needs [1016, 2103): slice starts too late
+        assert ei.value.code == -1
+
+
+def test_device_buffers_and_streams(pkg):
+    """Device-resident inputs/outputs on a user stream give the host-path result."""
+    import torch
+    wl = synth.make_workload("C2", "f32", n=30000, mq_per_sensor=8)
+    st = torch.cuda.Stream()
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band, stream=st) as idx:
+        hi, hd = idx.knn(wl.queries, wl.lengths, wl.k)
+        qd = torch.from_numpy(wl.queries).cuda()
+        ids = torch.empty(hi.shape, dtype=torch.int64, device="cuda")
+        dd = torch.empty(hd.shape, dtype=torch.float32, device="cuda")
+        pkg.smiler_knn(idx.handle, qd, None, wl.lengths, wl.k, ids, dd)
+        st.synchronize()
+        np.testing.assert_array_equal(ids.cpu().numpy(), hi)
+        np.testing.assert_array_equal(dd.cpu().numpy(), hd)
