@@ -560,7 +560,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
 template <int W> struct DiagStride { static constexpr int v = (W == 4) ? 12 : W + 4; };
 
 template <typename S, int W>
-__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 4 : 2))
+__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
     lb_diag_kernel(const S *series, const S *UC, const S *LC, const MQMeta *meta,
                    const typename Tr<S>::V4 *qtab, const QParams P, typename Tr<S>::V *lb,
                    int32_t *tauc) {
