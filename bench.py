@@ -191,7 +191,8 @@ def oracle_sample(wl, target_s: float):
 # ---------------------------------------------------------------------------
 CFG_NAMES = {
     "C2": "C2: one sensor, 2^20 points, ELV {16,32,64,128}, band 10%, k=32, w=8, 256 MQs/step/GPU",
-    "C3": "C3: 1024 sensors x 100k, ELV {32,64,96}, rho=8, k=64, w=16, 1 MQ/sensor, sharded by sensor",
+    "C3": "C3: 1024 sensors x 100k, ELV {32,64,96}, rho=8, k=64, w=16, 1 MQ stream/sensor (one tick per step), "
+          "sharded by sensor",
     "C4": "C4: one series of 1e8 points, ELV {32,64,96}, rho=8, k=32, w=16, 16 MQs/step, window ranges "
           "sharded over GPUs, NCCL all-gather + smiler_merge_topk",
     "C5": "C5: 1024 sensors x 100k, 10 streams/sensor (10,240 MQs/tick), ELV {16,32,64,128}, band 20%, k=128, "
@@ -239,7 +240,10 @@ class Runner:
         # C5 is a continuous prediction stream: every step is one tick of all
         # streams (each MQ advances one point); after the first tick the previous
         # tick's neighbours seed the thresholds (smiler_knn_step)
-        self.continuous = cfg == "C5" and not args.no_continuous
+        # C3 / C5 are continuous streams: by default every step is one
+        # tick through the reused window-level index (Remark 1, smiler_stream_step)
+        self.streaming = (not args.no_stream) and cfg in ("C3", "C5")
+        self.continuous = (cfg == "C5" and not args.no_continuous) or self.streaming
         self.tick = 0
         if self.continuous:
             D = wl.D
@@ -270,6 +274,16 @@ class Runner:
     def step(self, stats=None, opts=None):
         pkg = self.pkg
         op = opts if opts is not None else (self.op if stats is not None else self.op_fast)
+        if self.streaming:
+            if not self.have_prev:
+                self.stream_h = pkg.smiler_stream_create(self.idx.handle, self.qticks[0], self.qs, self.wl.lengths,
+                                                         self.k, self.ids, self.dd)
+                self.have_prev = True
+                self.tick = 1
+            newp = self.qticks[self.tick % self.qticks.shape[0]][:, -1].contiguous()
+            self.tick += 1
+            pkg.smiler_stream_step(self.stream_h, newp, self.ids, self.dd, stats, op)
+            return
         if self.continuous:
             q = self.qticks[self.tick % self.qticks.shape[0]]
             self.tick += 1
@@ -338,6 +352,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-continuous", action="store_true", help="C5: independent ticks (no smiler_knn_step)")
     ap.add_argument("--tau-mult", type=int, default=0, help="tau-set size (x k per item query; -1 = none, 0 = default)")
+    ap.add_argument("--no-stream", action="store_true",
+                    help="C3/C5: do not use the reused window-level index (smiler_stream_step); C5 then uses "
+                         "smiler_knn_step, C3 independent searches")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--two-level", action="store_true", help="time the paper's two-level path (a3 -> HBM -> a4)")
     ap.add_argument("--two-level-steps", type=int, default=3,
@@ -546,7 +563,7 @@ def main():
                                "frac": gbs / peaks["hbm_gbs"], "ms": f_s * 1e3}
         return ks
 
-    fused_main = not args.two_level and wl.window in (4, 8, 16)
+    fused_main = not args.two_level and wl.window in (4, 8, 16) and not R.streaming
     kernels = rooflines(phase, acc, steps, fused_main)
     ph_ms = {k_[3:]: v_ / 1e6 / steps for k_, v_ in phase.items()}
     dom = max(kernels.items(), key=lambda kv: kv[1]["ms"])[0]
@@ -598,7 +615,9 @@ def main():
         "survivor_frac": acc["survivors"] / max(1, acc["candidates"]),
         "lb_scan_gbs": scan["achieved"] if scan else None,
         "lb_scan_frac_of_hbm": scan["frac"] if scan else None,
-        "lb_path": "fused a3+a4 (posting rows on chip)" if fused_main else "two-level (postings in HBM)",
+        "lb_path": ("continuous streams: window-level rows reused in an HBM ring (Remark 1) + group scan"
+                    if R.streaming else "fused a3+a4 (posting rows on chip)" if fused_main
+                    else "two-level (postings in HBM)"),
         "phase_ms_per_step": ph_ms,
         "roofline": rf, "kernels": kernels, "two_level": two_level,
         "gpu_launches": int(round(launches_per_step * args.steps)),

@@ -178,6 +178,37 @@ SMILER_API int smiler_knn_step(smiler_index *idx, const void *queries, const int
                                smiler_knn_stats *stats, const smiler_knn_opts *opts);
 
 /*
+ * Continuous streams with the reused window-level index (Remark 1, P:936-953,
+ * Fig. 6).  A stream batch keeps, for every master query, its master query and
+ * its window-level posting lists (one per sliding window) in device memory, in
+ * a ring over the sliding windows.  Each step appends one point to every
+ * master query and drops the oldest; the new SW_0 takes the ring
+ * slot of the dropped SW, LB_EQ of SW_0..SW_rho_max (whose query envelope
+ * changed) and LB_EC of SW_0 are recomputed, all other posting entries are
+ * reused (those of the oldest SWs keep a wider, still valid envelope, R21), the
+ * group-level scan reads the ring (HBM-bound), and thresholds come from the
+ * previous step's neighbours joined with a small tile set.
+ * Results are the exact kNN of the current master queries.
+ *
+ * smiler_stream_create  queries [n_streams][D] (initial master queries),
+ *                       query_sensor/lengths/k as smiler_knn; runs the first
+ *                       search and writes its ids/dists ([n][n_len][k], host
+ *                       or device).  Memory: 8 (D - w + 1) floor(N/w) bytes of
+ *                       posting lists per stream, resident; ENOMEM if absent.
+ *                       The index must outlive the stream.
+ * smiler_stream_step    new_points [n_streams] (one new point per stream, index
+ *                       dtype, host or device); writes the step's results.
+ * smiler_stream_free    NULL-safe.
+ */
+typedef struct smiler_stream smiler_stream;
+SMILER_API int smiler_stream_create(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                    int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
+                                    int64_t *ids, void *dists, smiler_stream **out);
+SMILER_API int smiler_stream_step(smiler_stream *st, const void *new_points, int64_t *ids, void *dists,
+                                  smiler_knn_stats *stats, const smiler_knn_opts *opts);
+SMILER_API void smiler_stream_free(smiler_stream *st);
+
+/*
  * smiler_merge_topk -- final selection over G per-shard top-k lists (a9,
  * SURVEY §8(e)); called after an all-gather of the shards' (ids, dists).
  * ids_in [G][rows][k] int64, dists_in [G][rows][k] int32/float (dtype);

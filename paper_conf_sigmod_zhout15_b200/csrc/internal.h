@@ -47,6 +47,7 @@ struct MQMeta {
 // Parameters common to one smiler_knn chunk.
 struct QParams {
     int D, w, n_len, k, rho_env, E, LT, n_mq;
+    int ring_cursor;  // continuous streams: physical posting row of SW_b is (b + ring_cursor) mod n_sw
     int len[kMaxLen];
     int rho[kMaxLen];
 };

@@ -227,7 +227,9 @@ template <typename S, int W>
 __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
                                                        const MQMeta *meta,
                                                        const typename Tr<S>::V4 *qtab, int D,
-                                                       int w_rt, typename Tr<S>::V2 *post) {
+                                                       int w_rt, typename Tr<S>::V2 *post,
+                                                       int nrows = 1 << 30, int cursor = 0,
+                                                       bool incremental = false) {
     using V = typename Tr<S>::V;
     using V2 = typename Tr<S>::V2;
     extern __shared__ __align__(16) unsigned char wl_smem[];
@@ -249,7 +251,8 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
     V2 *out = post + m.post_off + r;
     if constexpr (W > 0) {
         constexpr int BC = W < 8 ? W : 8;
-        const int n_sw = D - W + 1;
+        const int n_sw = min(D - W + 1, nrows);  // rows [0, nrows) only (continuous step)
+        const int n_ring = D - W + 1;
         const int64_t base = m.series_off + r * W;
         const int64_t ndw = m.n_dw;
         V c[W], U[W], L[W];
@@ -259,26 +262,40 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
             U[j] = (V)UC[base + j];
             L[j] = (V)LC[base + j];
         }
+        // continuous step: physical row (b + cursor) mod n_ring, and rows b >= 1 keep
+        // their LB_EC (same MQ points, same series envelope): store EQ only
+        auto put = [&](int b, V eq, V ec) {
+            int row = b + cursor;
+            row -= row >= n_ring ? n_ring : 0;
+            V2 *o = out + (int64_t)row * ndw;
+            if (incremental && b > 0) {
+                o->x = eq;
+            } else {
+                V2 v;
+                v.x = eq;
+                v.y = ec;
+                *o = v;
+            }
+        };
         int b0 = 0;
         for (; b0 + BC <= n_sw; b0 += BC) {
-            V2 *o = out + (int64_t)b0 * ndw;
-            posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
-                                           [&](int bb, V eq, V ec) {
-                                               V2 v;
-                                               v.x = eq;
-                                               v.y = ec;
-                                               o[bb * ndw] = v;
-                                           });
+            if (!incremental && cursor == 0) {
+                V2 *o = out + (int64_t)b0 * ndw;
+                posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                               [&](int bb, V eq, V ec) {
+                                                   V2 v;
+                                                   v.x = eq;
+                                                   v.y = ec;
+                                                   o[bb * ndw] = v;
+                                               });
+            } else {
+                posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                               [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
+            }
         }
         if (b0 < n_sw) {
-            V2 *o = out + (int64_t)b0 * ndw;
             posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-                                          [&](int bb, V eq, V ec) {
-                                              V2 v;
-                                              v.x = eq;
-                                              v.y = ec;
-                                              o[bb * ndw] = v;
-                                          });
+                                          [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
         }
     } else {
         const int w = w_rt;
@@ -297,6 +314,62 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
             out[(int64_t)b * m.n_dw] = o;
         }
     }
+}
+
+// ---------------------------------------------------------------------------
+// Continuous streams (Remark 1, Fig. 6): after a stream advances by
+// one point, the new SW_0 takes the ring slot of the dropped oldest SW, and the
+// LB_EQ entries of SW_0 .. SW_rho (whose MQ envelope changed with the new point)
+// are recomputed; LB_EC of SW_b for b >= 1 is unchanged (same MQ points, same
+// series envelope).  One thread per DW r; rows b in [0, nrows), physical row
+// (b + cursor) mod n_sw.  EQ and EC for b = 0, EQ only for b >= 1.
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void __launch_bounds__(128) posting_rows_kernel(const S *series, const S *UC, const S *LC,
+                                                          const MQMeta *meta, const typename Tr<S>::V4 *qtab,
+                                                          int D, int w, int nrows, int cursor,
+                                                          typename Tr<S>::V2 *post) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    using V4 = typename Tr<S>::V4;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= m.n_dw) return;
+    const int n_sw = D - w + 1;
+    const int64_t base = m.series_off + r * w;
+    const V4 *qt = qtab + (int64_t)mq * D;
+    for (int b = 0; b < nrows && b < n_sw; b++) {
+        const int p0 = D - w - b;
+        V eq = (V)0, ec = (V)0;
+        for (int j = 0; j < w; j++) {
+            const V4 Q = qt[p0 + j];
+            lb_term((V)series[base + j], Q.y, Q.z, eq);
+            if (b == 0) lb_term(Q.x, (V)UC[base + j], (V)LC[base + j], ec);
+        }
+        int row = b + cursor;
+        row -= row >= n_sw ? n_sw : 0;
+        V2 *o = post + m.post_off + (int64_t)row * m.n_dw + r;
+        if (b == 0) {
+            V2 v;
+            v.x = eq;
+            v.y = ec;
+            *o = v;
+        } else {
+            o->x = eq;
+        }
+    }
+}
+
+// Advance every stream's master query by one point: MQ[0..D-1) = MQ[1..D),
+// MQ[D-1] = new point.
+template <typename S>
+__global__ void __launch_bounds__(256) stream_shift_kernel(S *mq, int D, const S *newpt) {
+    __shared__ S s[kMaxD];
+    S *q = mq + (int64_t)blockIdx.x * D;
+    for (int p = threadIdx.x; p < D; p += blockDim.x) s[p] = q[p];
+    __syncthreads();
+    for (int p = threadIdx.x; p < D; p += blockDim.x) q[p] = p + 1 < D ? s[p + 1] : newpt[blockIdx.x];
 }
 
 // ---------------------------------------------------------------------------
@@ -342,7 +415,13 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
 #pragma unroll
                 for (int u = 0; u < 8; u++) {
                     const int j = j0 + u;
-                    if (j < jlim) pv[u] = pp[(int64_t)(b + j * w) * m.n_dw - j];
+                    if (j < jlim) {
+                        // continuous streams keep the posting lists in a ring over SWs
+                        // (Remark 1): physical row of SW_{b+jw} = (b+jw+cursor) mod n_sw
+                        int row = b + j * w + P.ring_cursor;
+                        row -= row >= n_sw ? n_sw : 0;
+                        pv[u] = pp[(int64_t)row * m.n_dw - j];
+                    }
                 }
 #pragma unroll
                 for (int u = 0; u < 8; u++) {
@@ -358,8 +437,14 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
             }
         }
     }
-    __syncthreads();
-    lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * w, m, P, lb, tauc, mq, s_red);
+    if constexpr (W > 0) {
+        // row threadIdx.x of the tile was written by this thread only: barrier-free
+        // warp epilogue (the tau units of this kernel are warps)
+        lb_tile_epilogue_warp<V, W>(tile, RT, (Rb + 1) * w, m, P, lb, tauc, mq);
+    } else {
+        __syncthreads();
+        lb_tile_epilogue<V, W>(tile, RT, (Rb + 1) * w, m, P, lb, tauc, mq, s_red);
+    }
 }
 
 // ---------------------------------------------------------------------------

@@ -520,12 +520,22 @@ struct PhaseTimer {
     }
 };
 
+// Continuous-stream context (Remark 1): posting lists live in a per-stream ring.
+struct StreamCtx {
+    void *ring;                // V2 [sum over streams of n_sw * n_dw]
+    const int64_t *ring_off;   // per stream (global index) offset into ring, in pairs
+    int cursor;                // physical row of SW_0
+    int mode;                  // 0: build every row; 1: incremental rows [0, nrows)
+    int nrows;
+    int64_t *d_prev_out;       // device copy of the results (next step's tau seeds)
+};
+
 template <typename S>
 static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query_sensor_in,
                     int32_t n_mq, const int32_t *lengths_in, int32_t n_len, int32_t k, int64_t *ids,
                     void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts,
                     bool lb_only, void *post_out, void *lb_out, const int64_t *prev_ids = nullptr,
-                    int shift = 0) {
+                    int shift = 0, const StreamCtx *sctx = nullptr) {
     using V = typename Tr<S>::V;
     using V2 = typename Tr<S>::V2;
     using V4 = typename Tr<S>::V4;
@@ -543,7 +553,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     else memcpy(lens_h.data(), lengths_in, 4 * n_len);
     Plan pl;
     TRY(validate_query(idx, lens_h.data(), n_len, lb_only ? 1 : k, pl));
-    if (o.two_level || (lb_only && post_out)) pl.fused = false;
+    if (o.two_level || (lb_only && post_out) || sctx) pl.fused = false;
     if (pl.fused && o.reserved[0] == 1 && pl.fused_kind == 0) {  // row-form fused kernel (comparison)
         const int mmax = pl.D / pl.w, halo = mmax - 1;
         const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
@@ -594,7 +604,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     auto mq_bytes = [&](int j) -> size_t {
         const SensorInfo &si = idx->sensors[qsens[j]];
         const size_t ndw = (size_t)(si.n / w);
-        return (pl.fused ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
+        return ((pl.fused || sctx) ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
     };
     const size_t budget = idx->budget;
     int chunk_max = o.mq_chunk > 0 ? o.mq_chunk : 65535;
@@ -639,7 +649,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             m.t_lo = si.t_lo;
             m.t_hi = si.t_hi;
             m.n_dw = si.n / w;
-            m.post_off = post_tot;
+            m.post_off = sctx ? sctx->ring_off[c0 + j] : post_tot;
             m.seg_off = seg_tot;
             m.nblk = (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
             m.sensor = qsens[c0 + j];
@@ -656,7 +666,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
         }
         // tau-set units: CTAs (block epilogue) or warps (diagonal kernel's warp epilogue)
-        const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32 : 1;
+        // tau units: warps of the diagonal kernel / of group_scan (w in {4,8,16,32}), else CTAs
+        const bool w_static = pl.w == 4 || pl.w == 8 || pl.w == 16 || pl.w == 32;
+        const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32
+                                  : (!pl.fused && w_static) ? pl.RT / 32 : 1;
         int E = 0;
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         if (!lb_only && !o.no_prune) {
@@ -685,6 +698,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         if (o.reserved[1] == 1) P.k = -1;  // timing experiment (results invalid)
         if (o.reserved[1] == 2) P.E = 0;   // timing experiment: no tau set (no pruning)
         P.LT = LT;
+        P.ring_cursor = sctx ? sctx->cursor : 0;
         P.n_mq = B;
         for (int i = 0; i < nl; i++) {
             P.len[i] = pl.len[i];
@@ -695,7 +709,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         TRY(idx->queries.ensure(es * (size_t)B * D));
         TRY(idx->qv.ensure(sizeof(V) * (size_t)B * D));
         TRY(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
-        TRY(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
+        if (!sctx) TRY(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
+        V2 *postbuf = sctx ? reinterpret_cast<V2 *>(sctx->ring) : idx->post.as<V2>();
         TRY(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
         if (!lb_only) {
             TRY(idx->surv.ensure(4 * (size_t)seg_tot));
@@ -752,14 +767,26 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             // ---- a3 ----------------------------------------------------------
             int64_t ndw_max = 0;
             for (int j = 0; j < B; j++) ndw_max = std::max(ndw_max, meta[j].n_dw);
-            if (ndw_max > 0) {
+            const bool w_static = w == 4 || w == 8 || w == 16 || w == 32;
+            if (ndw_max > 0 && sctx && sctx->mode == 1 && !w_static) {
+                // continuous step: only SW_0 (EQ + EC) and SW_1..SW_rho (EQ) change
+                dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
+                posting_rows_kernel<S><<<grid, 128, 0, idx->stream>>>(
+                    (const S *)idx->d_series, (const S *)dUC, (const S *)dLC, d_meta, idx->qtab.as<V4>(), D, w,
+                    sctx->nrows, sctx->cursor, postbuf);
+                CHECK_LAUNCH();
+                launches++;
+            } else if (ndw_max > 0) {
+                const bool inc = sctx && sctx->mode == 1;
+                const int nrows = inc ? sctx->nrows : (1 << 30);
+                const int cur = sctx ? sctx->cursor : 0;
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
                 size_t smem = 3 * sizeof(V) * D;
                 auto go = [&](auto kern) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           w, idx->post.as<V2>());
+                                                           w, postbuf, nrows, cur, inc);
                 };
                 switch (w) {
                     case 4: go(window_lb_kernel<S, 4>); break;
@@ -777,7 +804,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             dim3 grid((unsigned)nblk_max, (unsigned)B);
             auto go4 = [&](auto kern) {
                 set_smem((const void *)kern, pl.smem_gs);
-                kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(idx->post.as<V2>(), d_meta, P, idx->lb.as<V>(),
+                kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(postbuf, d_meta, P, idx->lb.as<V>(),
                                                                idx->tauc.as<int32_t>());
             };
             switch (w) {
@@ -878,6 +905,9 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                            out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
         CU(cudaMemcpyAsync((char *)dists + (size_t)c0 * nl * pl.k * 4, idx->out_d.p, 4 * ob,
                            out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
+        if (sctx && sctx->d_prev_out)
+            CU(cudaMemcpyAsync(sctx->d_prev_out + (size_t)c0 * nl * pl.k, idx->out_ids.p, 8 * ob,
+                               cudaMemcpyDeviceToDevice, idx->stream));
         if (stats) {
             accum_counts_kernel<<<1, 256, 0, idx->stream>>>(scount, fcount, nseg, nl,
                                                             idx->tmp.as<unsigned long long>());
@@ -952,6 +982,152 @@ extern "C" int smiler_knn_step(smiler_index *idx, const void *queries, const int
     return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats, opts, false,
                            nullptr, nullptr, prev_ids, shift);
 }
+
+// ---------------------------------------------------------------------------
+// Continuous streams (Def. 4.1; Remark 1; tau method 2,
+// P:1452-1458)
+// ---------------------------------------------------------------------------
+struct smiler_stream {
+    smiler_index *idx = nullptr;
+    int n = 0, D = 0, n_len = 0, k = 0, n_sw = 0, nrows = 0;
+    std::vector<int32_t> lens, qsens;
+    std::vector<int64_t> ring_off;
+    void *d_mq = nullptr;      // [n][D] current master queries (storage type)
+    void *d_new = nullptr;     // [n] staging for new points
+    void *ring = nullptr;      // posting-list rings
+    int64_t *d_prev = nullptr; // [n][n_len][k] last results
+    int cursor = 0;
+    int64_t steps = 0;
+};
+
+static void stream_release(smiler_stream *st) {
+    if (!st) return;
+    if (st->idx) cudaSetDevice(st->idx->device);
+    if (st->idx && st->idx->stream) cudaStreamSynchronize(st->idx->stream);
+    if (st->d_mq) cudaFree(st->d_mq);
+    if (st->d_new) cudaFree(st->d_new);
+    if (st->ring) cudaFree(st->ring);
+    if (st->d_prev) cudaFree(st->d_prev);
+    delete st;
+}
+
+template <typename S>
+static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_stats *stats,
+                      const smiler_knn_opts *opts, int mode) {
+    StreamCtx sc;
+    sc.ring = st->ring;
+    sc.ring_off = st->ring_off.data();
+    sc.cursor = st->cursor;
+    sc.mode = mode;
+    sc.nrows = st->nrows;
+    sc.d_prev_out = st->d_prev;
+    return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
+                       stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
+}
+
+extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                    int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
+                                    int64_t *ids, void *dists, smiler_stream **out) {
+    if (!out) return fail(SMILER_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!idx || !queries || !lengths || !ids || !dists) return fail(SMILER_EINVAL, "NULL argument");
+    if (idx->shard) return fail(SMILER_EINVAL, "streams on window-range shards are not supported");
+    if (n_streams < 1) return fail(SMILER_EINVAL, "n_streams must be >= 1");
+    if (n_len < 1 || n_len > kMaxLen) return fail(SMILER_EINVAL, "n_len must be in [1, %d]", kMaxLen);
+    TRY(set_device(idx));
+    smiler_stream *st = new smiler_stream();
+    st->idx = idx;
+    st->n = n_streams;
+    st->n_len = n_len;
+    st->k = k;
+    st->lens.resize(n_len);
+    if (is_device_ptr(lengths)) {
+        if (cudaMemcpy(st->lens.data(), lengths, 4 * n_len, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            stream_release(st);
+            return fail(SMILER_ECUDA, "reading lengths");
+        }
+    } else {
+        memcpy(st->lens.data(), lengths, 4 * n_len);
+    }
+    Plan pl;
+    int rc = validate_query(idx, st->lens.data(), n_len, k, pl);
+    if (rc) {
+        stream_release(st);
+        return rc;
+    }
+    st->D = pl.D;
+    st->n_sw = pl.D - pl.w + 1;
+    st->nrows = std::min(pl.rho_env + 1, st->n_sw);
+    st->qsens.assign(n_streams, 0);
+    if (query_sensor) {
+        if (is_device_ptr(query_sensor)) cudaMemcpy(st->qsens.data(), query_sensor, 4 * (size_t)n_streams, cudaMemcpyDeviceToHost);
+        else memcpy(st->qsens.data(), query_sensor, 4 * (size_t)n_streams);
+    }
+    int64_t tot = 0;
+    st->ring_off.resize(n_streams);
+    for (int j = 0; j < n_streams; j++) {
+        if (st->qsens[j] < 0 || st->qsens[j] >= (int)idx->sensors.size()) {
+            stream_release(st);
+            return fail(SMILER_EINVAL, "query_sensor[%d] out of range", j);
+        }
+        st->ring_off[j] = tot;
+        tot += (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
+    }
+    const size_t es = esize(idx->dtype);
+    cudaError_t e = cudaMalloc(&st->ring, 8 * (size_t)std::max<int64_t>(tot, 1));
+    if (e == cudaSuccess) e = cudaMalloc(&st->d_mq, es * (size_t)n_streams * pl.D);
+    if (e == cudaSuccess) e = cudaMalloc(&st->d_new, es * (size_t)n_streams);
+    if (e == cudaSuccess) e = cudaMalloc(&st->d_prev, 8 * (size_t)n_streams * n_len * k);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        stream_release(st);
+        return fail(SMILER_ENOMEM, "stream buffers (%lld posting pairs): %s", (long long)tot, cudaGetErrorString(e));
+    }
+    e = cudaMemcpyAsync(st->d_mq, queries, es * (size_t)n_streams * pl.D, cudaMemcpyDefault, idx->stream);
+    if (e != cudaSuccess) {
+        stream_release(st);
+        return fail(SMILER_ECUDA, "copying queries: %s", cudaGetErrorString(e));
+    }
+    rc = idx->dtype == SMILER_I16 ? stream_run<int16_t>(st, ids, dists, nullptr, nullptr, 0)
+                                  : stream_run<float>(st, ids, dists, nullptr, nullptr, 0);
+    if (rc) {
+        stream_release(st);
+        return rc;
+    }
+    *out = st;
+    return SMILER_OK;
+}
+
+extern "C" int smiler_stream_step(smiler_stream *st, const void *new_points, int64_t *ids, void *dists,
+                                  smiler_knn_stats *stats, const smiler_knn_opts *opts) {
+    if (!st) return fail(SMILER_EINVAL, "stream is NULL");
+    if (!new_points || !ids || !dists) return fail(SMILER_EINVAL, "NULL argument");
+    smiler_index *idx = st->idx;
+    TRY(set_device(idx));
+    const size_t es = esize(idx->dtype);
+    CU(cudaMemcpyAsync(st->d_new, new_points, es * (size_t)st->n, cudaMemcpyDefault, idx->stream));
+    if (idx->dtype == SMILER_I16) {
+        // R17 range of the appended points, checked on the host copy when available
+        if (!is_device_ptr(new_points)) {
+            const int16_t *np = (const int16_t *)new_points;
+            for (int j = 0; j < st->n; j++)
+                if (np[j] > 1023 || np[j] < -1023) return fail(SMILER_ERANGE, "new point %d outside [-1023, 1023]", j);
+        }
+        stream_shift_kernel<int16_t><<<st->n, 256, 0, idx->stream>>>((int16_t *)st->d_mq, st->D,
+                                                                     (const int16_t *)st->d_new);
+    } else {
+        stream_shift_kernel<float><<<st->n, 256, 0, idx->stream>>>((float *)st->d_mq, st->D,
+                                                                   (const float *)st->d_new);
+    }
+    CHECK_LAUNCH();
+    // ring: the new SW_0 takes the slot of the dropped oldest SW (Fig. 6)
+    st->cursor = (st->cursor + st->n_sw - 1) % st->n_sw;
+    st->steps++;
+    return idx->dtype == SMILER_I16 ? stream_run<int16_t>(st, ids, dists, stats, opts, 1)
+                                    : stream_run<float>(st, ids, dists, stats, opts, 1);
+}
+
+extern "C" void smiler_stream_free(smiler_stream *st) { stream_release(st); }
 
 extern "C" int smiler_lower_bounds(smiler_index *idx, const void *queries, const int32_t *query_sensor,
                                    int32_t n_mq, const int32_t *lengths, int32_t n_len, void *postings,

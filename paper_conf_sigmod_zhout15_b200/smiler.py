@@ -67,6 +67,10 @@ def lib():
         L.smiler_knn.argtypes = [P, P, P, i32, P, i32, i32, P, P, P]
         L.smiler_knn_ex.argtypes = [P, P, P, i32, P, i32, i32, P, P, P, P]
         L.smiler_knn_step.argtypes = [P, P, P, i32, P, i32, i32, P, i32, P, P, P, P]
+        L.smiler_stream_create.argtypes = [P, P, P, i32, P, i32, i32, P, P, ctypes.POINTER(P)]
+        L.smiler_stream_step.argtypes = [P, P, P, P, P, P]
+        L.smiler_stream_free.argtypes = [P]
+        L.smiler_stream_free.restype = None
         L.smiler_merge_topk.argtypes = [P, P, i32, i32, i32, i32, P, P, i32, P]
         L.smiler_index_envelope.argtypes = [P, i32, i32, P, P]
         L.smiler_lower_bounds.argtypes = [P, P, P, i32, P, i32, P, P]
@@ -76,6 +80,7 @@ def lib():
         L.smiler_last_error.restype = ctypes.c_char_p
         L.smiler_abi_version.restype = i32
         for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex", "smiler_knn_step",
+                  "smiler_stream_create", "smiler_stream_step",
                   "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_dtw"):
             getattr(L, f).restype = i32
         _lib = L
@@ -170,6 +175,29 @@ def smiler_knn_step(handle: int, queries, query_sensor, lengths, k: int, prev_id
                                  ctypes.byref(opts) if opts is not None else None))
 
 
+def smiler_stream_create(handle: int, queries, query_sensor, lengths, k: int, ids, dists) -> int:
+    """Create a batch of continuous streams (Remark 1) and run their first search."""
+    h = ctypes.c_void_p()
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    qs = None if query_sensor is None else np.ascontiguousarray(query_sensor, np.int32)
+    _check("smiler_stream_create",
+           lib().smiler_stream_create(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens), len(lens),
+                                      k, _ptr(ids), _ptr(dists), ctypes.byref(h)))
+    return h.value
+
+
+def smiler_stream_step(stream: int, new_points, ids, dists, stats: Optional[KnnStats] = None,
+                       opts: Optional[KnnOpts] = None) -> None:
+    _check("smiler_stream_step",
+           lib().smiler_stream_step(stream, _ptr(new_points), _ptr(ids), _ptr(dists),
+                                    ctypes.byref(stats) if stats is not None else None,
+                                    ctypes.byref(opts) if opts is not None else None))
+
+
+def smiler_stream_free(stream: Optional[int]) -> None:
+    lib().smiler_stream_free(stream)
+
+
 def smiler_merge_topk(ids_in, dists_in, G: int, rows: int, k: int, ids_out, dists_out,
                       device: int = 0, stream=None) -> None:
     _check("smiler_merge_topk",
@@ -215,6 +243,46 @@ def smiler_abi_version() -> int:
 # ---------------------------------------------------------------------------
 # Convenience wrapper (host numpy in, host numpy out)
 # ---------------------------------------------------------------------------
+class Stream:
+    """A batch of continuous master-query streams over one Index (host numpy I/O)."""
+
+    def __init__(self, index: "Index", queries, lengths: Sequence[int], k: int, query_sensor=None):
+        self.index, self.lengths, self.k = index, list(lengths), k
+        self.n = int(queries.shape[0])
+        self.vt = np.int32 if index.dtype == SMILER_I16 else np.float32
+        ids = np.empty((self.n, len(lengths), k), np.int64)
+        dists = np.empty((self.n, len(lengths), k), self.vt)
+        self.handle = smiler_stream_create(index.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
+                                           ids, dists)
+        self.first = (ids, dists)
+
+    def step(self, new_points, stats: bool = False, timing: bool = False):
+        ids = np.empty((self.n, len(self.lengths), self.k), np.int64)
+        dists = np.empty((self.n, len(self.lengths), self.k), self.vt)
+        st = KnnStats() if stats else None
+        smiler_stream_step(self.handle, np.ascontiguousarray(new_points), ids, dists, st, KnnOpts(timing=int(timing)))
+        if stats:
+            return ids, dists, st.as_dict()
+        return ids, dists
+
+    def close(self):
+        if self.handle:
+            smiler_stream_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
 class Index:
     """RAII-style owner of one smiler_index handle."""
 

@@ -473,3 +473,43 @@ def test_device_buffers_and_streams(pkg):
         st.synchronize()
         np.testing.assert_array_equal(ids.cpu().numpy(), hi)
         np.testing.assert_array_equal(dd.cpu().numpy(), hd)
+
+
+# ---------------------------------------------------------------------------
+# continuous streams with the reused window-level index (Remark 1)
+# ---------------------------------------------------------------------------
+def _stream_case(pkg, orc, dtype, name, steps, **kw):
+    wl = synth.make_workload(name, dtype, step=0, **kw)
+    D = wl.D
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        with pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor) as st:
+            ids, dists = st.first
+            for s in range(steps + 1):
+                ws = wl if s == 0 else synth.make_workload(name, dtype, step=s, **kw)
+                if s > 0:
+                    newp = np.ascontiguousarray(ws.queries[:, D - 1])   # the point appended at step s
+                    assert (ws.queries[:, :D - 1] == prev_q[:, 1:]).all()
+                    ids, dists, stt = st.step(newp, stats=True)
+                    assert stt["posting_bytes"] > 0
+                prev_q = ws.queries
+                if s % 3 and s != steps:
+                    continue   # check every third step against the oracle (and the last)
+                if dtype == "i16":
+                    oid, od = orc.knn(ws, threads=THREADS)
+                    np.testing.assert_array_equal(ids, oid)
+                    np.testing.assert_array_equal(dists.astype(np.int64), od)
+                else:
+                    oid, od = orc.knn(ws, mode="f32", threads=THREADS)
+                    np.testing.assert_array_equal(ids, oid)
+                    np.testing.assert_array_equal(dists, od)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_stream_steps_c5_shape(pkg, orc, dtype):
+    _stream_case(pkg, orc, dtype, "C5", 6, n=12001, n_sensors=3, mq_per_sensor=2)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_stream_ring_wraps(pkg, orc, dtype):
+    """D = 32, w = 8: 25 sliding windows, so 30 steps wrap the ring cursor."""
+    _stream_case(pkg, orc, dtype, "C1", 30, n=3000, lengths=[16, 32], window=8, band=3.0, k=6, mq_per_sensor=3)
