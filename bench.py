@@ -308,10 +308,21 @@ class Runner:
         self.ih = torch.empty((rows, self.k), dtype=torch.int64).pin_memory()
         self.dh = torch.empty((rows, self.k), dtype=self.vt).pin_memory()
         h2d = self.qh.numel() * self.qh.element_size() + self.n_len * 4 + (0 if self.qs is None else self.qs.nbytes)
+        if self.streaming:  # a tick uploads one new point per stream
+            h2d = self.wl.n_mq * self.qh.element_size()
         return int(h2d), int(self.ih.numel() * 8 + self.dh.numel() * 4)
 
     def step_e2e(self):
         pkg, torch = self.pkg, self.torch
+        if self.streaming:
+            # one tick through the public stream API with pinned host buffers
+            if not hasattr(self, "newp_h"):
+                self.newp_h = torch.empty((self.wl.n_mq,), dtype=self.qticks_host.dtype).pin_memory()
+            self.newp_h.copy_(self.qticks_host[self.tick % self.qticks_host.shape[0]][:, -1])
+            self.tick += 1
+            pkg.smiler_stream_step(self.stream_h, self.newp_h, self.ih.view(self.wl.n_mq, self.n_len, self.k),
+                                   self.dh.view(self.wl.n_mq, self.n_len, self.k))
+            return
         if self.continuous:
             q = self.qticks_host[self.tick % self.qticks_host.shape[0]]
             self.tick += 1
@@ -535,15 +546,22 @@ def main():
     post_bytes_step = 8 * n_sw * sum(p // wl.window for p in pts)
     lb_bytes_step = 4 * n_len * sum(pts)
 
+    # continuous streams recompute only SW_0 (EQ + EC) and SW_1..SW_rho_max (EQ):
+    # (rho_max + 2) / 2 term-pair equivalents per (DW, j) instead of n_sw
+    rho_env = max(wl.rhos())
+    inc_terms = (min(rho_env + 1, n_sw) + 1) / 2.0 * sum(p // wl.window * wl.window for p in pts)
+
     def rooflines(ph, ac, nsteps, fused):
         ks = {}
         win_s = ph["ns_window_lb"] / 1e9 / nsteps
         if win_s > 0:
-            rate = win_terms / win_s
-            ks["lb_fused" if fused else "window_lb_a3"] = {
+            terms = inc_terms if R.streaming else win_terms
+            rate = terms / win_s
+            ks["lb_fused" if fused else ("window_lb_a3_incremental" if R.streaming else "window_lb_a3")] = {
                 "bound": "alu", "achieved": rate / 1e12, "peak": term_peak / 1e12,
                 "unit": "T term-pairs/s", "frac": rate / term_peak, "ms": win_s * 1e3,
-                "algorithmic_per_mq": "%d (SW,DW,j) term pairs" % (win_terms // wl.n_mq)}
+                "algorithmic_per_mq": "%d (SW,DW,j) term pairs" % ((inc_terms if R.streaming else win_terms)
+                                                                     // wl.n_mq)}
         gs_s = ph["ns_group_scan"] / 1e9 / nsteps
         if not fused and gs_s > 0:
             byts = post_bytes_step + lb_bytes_step

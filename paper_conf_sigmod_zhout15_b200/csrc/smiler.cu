@@ -606,7 +606,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         const size_t ndw = (size_t)(si.n / w);
         return ((pl.fused || sctx) ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
     };
-    const size_t budget = idx->budget;
+    size_t budget = idx->budget;  // halved on ENOMEM (e.g. a resident stream ring)
     int chunk_max = o.mq_chunk > 0 ? o.mq_chunk : 65535;
     chunk_max = std::min(chunk_max, 65535);
 
@@ -634,6 +634,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         }
         const int B = c1 - c0;
         n_chunks++;
+        const int64_t cand_before = cand_total;
+        const double bf_before = bf_cells;
         // ---- metadata ------------------------------------------------------
         MQMeta *meta;
         int mslot;
@@ -705,26 +707,48 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             P.rho[i] = pl.rho[i];
         }
         const int nseg = B * nl;
-        TRY(idx->meta.ensure(sizeof(MQMeta) * B));
-        TRY(idx->queries.ensure(es * (size_t)B * D));
-        TRY(idx->qv.ensure(sizeof(V) * (size_t)B * D));
-        TRY(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
-        if (!sctx) TRY(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
-        V2 *postbuf = sctx ? reinterpret_cast<V2 *>(sctx->ring) : idx->post.as<V2>();
-        TRY(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
+        auto ensure_all = [&]() -> int {
+#define ENS(x)                          \
+    do {                                \
+        int r_ = (x);                   \
+        if (r_ != SMILER_OK) return r_; \
+    } while (0)
+        ENS(idx->meta.ensure(sizeof(MQMeta) * B));
+        ENS(idx->queries.ensure(es * (size_t)B * D));
+        ENS(idx->qv.ensure(sizeof(V) * (size_t)B * D));
+        ENS(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
+        if (!sctx) ENS(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
+        ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
         if (!lb_only) {
-            TRY(idx->surv.ensure(4 * (size_t)seg_tot));
-            TRY(idx->fin.ensure(8 * (size_t)seg_tot));
-            TRY(idx->tauc.ensure(4 * (size_t)nseg * LT));
-            TRY(idx->tauk.ensure(8 * (size_t)nseg * LT));
-            TRY(idx->taukey.ensure(8 * (size_t)nseg));
-            TRY(idx->thr.ensure(4 * (size_t)nseg));
-            TRY(idx->scount.ensure(4 * (size_t)nseg));
-            TRY(idx->fcount.ensure(4 * (size_t)nseg));
-            TRY(idx->taskoff.ensure(4 * (size_t)(B + 1) * nl * 2));
-            TRY(idx->out_ids.ensure(8 * (size_t)nseg * pl.k));
-            TRY(idx->out_d.ensure(4 * (size_t)nseg * pl.k));
+            ENS(idx->surv.ensure(4 * (size_t)seg_tot));
+            ENS(idx->fin.ensure(8 * (size_t)seg_tot));
+            ENS(idx->tauc.ensure(4 * (size_t)nseg * LT));
+            ENS(idx->tauk.ensure(8 * (size_t)nseg * LT));
+            ENS(idx->taukey.ensure(8 * (size_t)nseg));
+            ENS(idx->thr.ensure(4 * (size_t)nseg));
+            ENS(idx->scount.ensure(4 * (size_t)nseg));
+            ENS(idx->fcount.ensure(4 * (size_t)nseg));
+            ENS(idx->taskoff.ensure(4 * (size_t)(B + 1) * nl * 2));
+            ENS(idx->out_ids.ensure(8 * (size_t)nseg * pl.k));
+            ENS(idx->out_d.ensure(4 * (size_t)nseg * pl.k));
         }
+#undef ENS
+            return SMILER_OK;
+        };
+        {
+            const int rc_ = ensure_all();
+            if (rc_ == SMILER_ENOMEM && B > 1) {  // retry this chunk with half the budget
+                budget /= 2;
+                n_chunks--;
+                cand_total = cand_before;
+                bf_cells = bf_before;
+                g_err.clear();
+                cudaGetLastError();
+                continue;
+            }
+            TRY(rc_);
+        }
+        V2 *postbuf = sctx ? reinterpret_cast<V2 *>(sctx->ring) : idx->post.as<V2>();
         MQMeta *d_meta = idx->meta.as<MQMeta>();
         CU(cudaMemcpyAsync(d_meta, meta, sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
         CU(cudaEventRecord(idx->meta_ev[mslot], idx->stream));
