@@ -134,7 +134,33 @@ struct smiler_index {
     size_t h_meta_cap[2] = {0, 0};
     cudaEvent_t meta_ev[2] = {nullptr, nullptr};
     int meta_slot = 0;
+    // side streams: the per-item-query DTW launches (different rho templates)
+    // run concurrently so their grid tails overlap
+    cudaStream_t side[kMaxLen] = {};
+    cudaEvent_t fork_ev = nullptr;
+    cudaEvent_t join_ev[kMaxLen] = {};
 };
+
+static int side_fork(smiler_index *idx, int n) {
+    if (!idx->fork_ev) CU(cudaEventCreateWithFlags(&idx->fork_ev, cudaEventDisableTiming));
+    CU(cudaEventRecord(idx->fork_ev, idx->stream));
+    for (int i = 0; i < n; i++) {
+        if (!idx->side[i]) {
+            CU(cudaStreamCreateWithFlags(&idx->side[i], cudaStreamNonBlocking));
+            CU(cudaEventCreateWithFlags(&idx->join_ev[i], cudaEventDisableTiming));
+        }
+        CU(cudaStreamWaitEvent(idx->side[i], idx->fork_ev, 0));
+    }
+    return SMILER_OK;
+}
+
+static int side_join(smiler_index *idx, int n) {
+    for (int i = 0; i < n; i++) {
+        CU(cudaEventRecord(idx->join_ev[i], idx->side[i]));
+        CU(cudaStreamWaitEvent(idx->stream, idx->join_ev[i], 0));
+    }
+    return SMILER_OK;
+}
 
 // Pinned staging slot for n MQMeta; waits until the copy that last used the
 // slot has completed.
@@ -279,6 +305,11 @@ static void destroy(smiler_index *idx) {
                       &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
+    for (int i = 0; i < kMaxLen; i++) {
+        if (idx->side[i]) cudaStreamDestroy(idx->side[i]);
+        if (idx->join_ev[i]) cudaEventDestroy(idx->join_ev[i]);
+    }
+    if (idx->fork_ev) cudaEventDestroy(idx->fork_ev);
     for (int s = 0; s < 2; s++) {
         if (idx->h_meta[s]) cudaFreeHost(idx->h_meta[s]);
         if (idx->meta_ev[s]) cudaEventDestroy(idx->meta_ev[s]);
@@ -474,9 +505,9 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
                         const int32_t *list, int LT, const int32_t *counts, int32_t *task_off,
                         uint64_t *keys_out, const uint64_t *tau_key, uint64_t *fin,
                         int32_t *fin_count, const MQMeta *d_meta, const typename Tr<S>::V *qv,
-                        int D) {
-    task_prefix_kernel<<<1, 1024, 0, idx->stream>>>(counts, mode == 0 ? LT : -1, n_mq, pl.n_len, li,
-                                                    task_off);
+                        int D, cudaStream_t st = nullptr) {
+    if (!st) st = idx->stream;
+    task_prefix_kernel<<<1, 1024, 0, st>>>(counts, mode == 0 ? LT : -1, n_mq, pl.n_len, li, task_off);
     CHECK_LAUNCH();
     DtwParams<S> p;
     p.series = (const S *)idx->d_series;
@@ -496,7 +527,7 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
     p.tau_key = tau_key;
     p.fin = fin;
     p.fin_count = fin_count;
-    launch_dtw<S>(pl.rho[li], p, 0, idx->stream);
+    launch_dtw<S>(pl.rho[li], p, 0, st);
     CHECK_LAUNCH();
     return SMILER_OK;
 }
@@ -877,14 +908,16 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             launches++;
         }
         if (!o.no_prune) {
+            TRY(side_fork(idx, nl));
             for (int i = 0; i < nl; i++) {
                 TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
                                     taskoff + (size_t)i * (B + 1), idx->tauk.as<uint64_t>(), nullptr,
-                                    nullptr, nullptr, d_meta, idx->qv.as<V>(), D));
+                                    nullptr, nullptr, d_meta, idx->qv.as<V>(), D, idx->side[i]));
                 launches += 2;
                 tau_slots_total += (int64_t)B * LT;
                 cells_acc += (double)B * LT * (double)dtw_cells(pl.len[i], pl.rho[i]);
             }
+            TRY(side_join(idx, nl));
             tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
             CHECK_LAUNCH();
             launches++;
@@ -911,12 +944,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         TRY(tm.mark(5));
         // ---- a7 ----------------------------------------------------------
         int32_t *taskoff2 = taskoff + (size_t)nl * (B + 1);
+        TRY(side_fork(idx, nl));
         for (int i = 0; i < nl; i++) {
             TRY(run_dtw_list<S>(idx, pl, i, B, 1, idx->surv.as<int32_t>(), 0, scount,
                                 taskoff2 + (size_t)i * (B + 1), nullptr, taukey, idx->fin.as<uint64_t>(),
-                                fcount, d_meta, idx->qv.as<V>(), D));
+                                fcount, d_meta, idx->qv.as<V>(), D, idx->side[i]));
             launches += 2;
         }
+        TRY(side_join(idx, nl));
         TRY(tm.mark(6));
         // ---- a8 ----------------------------------------------------------
         topk_kernel<S><<<nseg, 512, 0, idx->stream>>>(idx->fin.as<uint64_t>(), fcount, d_meta, P,
