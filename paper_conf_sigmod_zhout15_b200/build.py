@@ -25,6 +25,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
+# tuning experiments only (tools/): extra -D knobs, e.g. "-DSMILER_GS_MINB=3"
+FLAGS += os.environ.get("SMILER_EXTRA_NVFLAGS", "").split()
 
 
 def _stale(target: str, deps) -> bool:

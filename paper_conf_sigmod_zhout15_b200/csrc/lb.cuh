@@ -784,3 +784,116 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
         if (acc == (V)12345) lb[0] = acc;
     }
 }
+
+// ---------------------------------------------------------------------------
+// a4 for static w (two-level path, continuous-stream ring): thread x owns the
+// rightmost DW r = Rb + x and walks CSG row j = 0 .. mmax-1 itself, summing
+// P[b + j w][r - j] for all b < w into register sums S_b (the same j order as
+// the generic scan, so LB_w is bit-identical).  Emission is lb_diag_kernel's:
+// m_i(b) = q_i - [b > r_i], so IQ i's slots b > r_i are final after row
+// q_i - 2 (saved) and b <= r_i after row q_i - 1, written straight from
+// registers by diag_emit (vector stores, per-warp tau set).  No shared memory,
+// no barrier.  Posting addresses are 32-bit offsets from the MQ's posting block
+// (host guarantees n_sw * n_dw < 2^31).  Only CTA 0 (DWs r < mmax - 1 lack
+// some r - j) and the last CSG row (fewer than w SWs) take predicated loads;
+// elsewhere threads past the last DW read DW n_dw - 1 and their slots are
+// masked at emission (t >= tend).
+// ---------------------------------------------------------------------------
+constexpr int kScanThreads = 256;
+// measured on C3/C5 streams (profiles/r01/history/group_scan_variants.txt)
+#ifndef SMILER_GS_MINB
+#define SMILER_GS_MINB(W) ((W) <= 8 ? 4 : (W) <= 16 ? 2 : 1)
+#endif
+
+template <typename V2, int W, bool CHECK>
+__device__ __forceinline__ void gs_load_row(V2 (&pv)[W], const V2 *pp, uint32_t off, int bw, uint32_t ndw,
+                                            uint32_t wrap, int nrow, bool ok) {
+#pragma unroll
+    for (int b = 0; b < W; b++) {
+        // physical rows rr + b >= n_sw wrap to the ring start (bw = n_sw - rr)
+        const uint32_t o = off + (uint32_t)b * ndw - (b >= bw ? wrap : 0u);
+        if constexpr (CHECK) {
+            pv[b] = V2{};
+            if (ok && b < nrow) pv[b] = __ldg(pp + o);
+        } else {
+            pv[b] = __ldg(pp + o);
+        }
+    }
+}
+
+template <typename S, int W>
+__global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_reg_kernel(
+    const typename Tr<S>::V2 *post, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    const int D = P.D;
+    const int nl = P.n_len;
+    const int n_sw = D - W + 1;
+    const int mmax = D / W;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) return;
+    const int64_t r = (int64_t)blockIdx.x * kScanThreads - 1 + threadIdx.x;
+    const int64_t s0 = (r + 1) * W;  // e of slot b = 0
+    const bool valid = r >= 0 && r < m.n_dw;
+    const int jall = valid ? (int)min((int64_t)mmax, r + 1) : 0;  // DW r - j must exist
+    const bool first = blockIdx.x == 0;
+    const uint32_t ndw = (uint32_t)m.n_dw;
+    const uint32_t wrap = (uint32_t)n_sw * ndw;
+    const int64_t rc = r < 0 ? 0 : (r < m.n_dw ? r : m.n_dw - 1);
+    // offsets count from pp - mmax so they stay non-negative across the ring wrap
+    const V2 *pp = post + m.post_off + rc - mmax;
+    // values saved after row q_i - 2 live in shared memory ([b][thread]: no
+    // bank conflicts), keeping the registers for sums and loads in flight
+    __shared__ V s_saved[W][kScanThreads];
+    const int x = threadIdx.x;
+    V se[W], sc[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
+    uint64_t emit_rows = 0, save_rows = 0;
+    for (int i = 0; i < nl; i++) {
+        const int qi = P.len[i] / W;
+        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
+        if (qi >= 2) save_rows |= 1ull << (qi - 2);
+    }
+    if (nl > 0 && P.len[0] < W) {
+        V z[W];
+#pragma unroll
+        for (int b = 0; b < W; b++) z[b] = (V)0;
+        for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq);
+    }
+    // ring row of SW_{j w} (Remark 1): rr = (j w + cursor) mod n_sw,
+    // advanced by w per row (mmax >= 2 implies n_sw > w)
+    int rr = P.ring_cursor;
+    for (int j = 0; j < mmax; j++) {
+        V2 pv[W];
+        const uint32_t off = (uint32_t)rr * ndw + (uint32_t)(mmax - j);
+        const int nrow = n_sw - j * W;
+        if (first || nrow < W)
+            gs_load_row<V2, W, true>(pv, pp, off, n_sw - rr, ndw, wrap, nrow, j < jall);
+        else
+            gs_load_row<V2, W, false>(pv, pp, off, n_sw - rr, ndw, wrap, nrow, true);
+        rr += W;
+        rr -= rr >= n_sw ? n_sw : 0;
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            se[b] += pv[b].x;
+            sc[b] += pv[b].y;
+        }
+        if (emit_rows >> j & 1ull) {
+            for (int i = 0; i < nl; i++) {
+                const int qi = P.len[i] / W, ri = P.len[i] % W;
+                if (j == qi - 1) {
+                    V v[W];
+#pragma unroll
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : vmax(se[b], sc[b]);
+                    diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
+                }
+            }
+        }
+        if (save_rows >> j & 1ull) {
+#pragma unroll
+            for (int b = 0; b < W; b++) s_saved[b][x] = vmax(se[b], sc[b]);
+        }
+    }
+}

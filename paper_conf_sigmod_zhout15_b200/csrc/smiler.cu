@@ -444,6 +444,7 @@ struct Plan {
     int D, n_len, k, w, rho_env;
     std::vector<int> len, rho;
     int RT;          // group-scan CTA width (two-level path)
+    bool scan_reg;   // a4 by group_scan_reg_kernel (static w, mmax <= 64)
     bool fused;      // a3+a4 fused kernel
     int fused_kind;  // 0 = diagonal form (lb_diag_kernel), 1 = row form (lb_fused_kernel)
     int RTf;         // fused: tile DWs per CTA
@@ -477,9 +478,19 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
     const size_t vs = 4;
     const int mmax = pl.D / pl.w;
     const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
-    pl.RT = 256;
-    while (pl.RT > 32 && em + (size_t)n_len * pl.RT * (pl.w + 1) * vs > 160 * 1024) pl.RT >>= 1;
-    pl.smem_gs = em + (size_t)n_len * pl.RT * (pl.w + 1) * vs;
+    int64_t n_max = 0;
+    for (const auto &si : idx->sensors) n_max = std::max<int64_t>(n_max, si.n);
+    // register scan: emission bitmasks hold mmax rows; posting offsets are int32
+    pl.scan_reg = (pl.w == 4 || pl.w == 8 || pl.w == 16 || pl.w == 32) && mmax <= 64 &&
+                  (int64_t)(pl.D - pl.w + 1) * (n_max / pl.w) < ((int64_t)1 << 31);
+    if (pl.scan_reg) {
+        pl.RT = kScanThreads;
+        pl.smem_gs = 0;
+    } else {
+        pl.RT = 256;
+        while (pl.RT > 32 && em + (size_t)n_len * pl.RT * (pl.w + 1) * vs > 160 * 1024) pl.RT >>= 1;
+        pl.smem_gs = em + (size_t)n_len * pl.RT * (pl.w + 1) * vs;
+    }
     pl.fused = false;
     if (pl.w == 4 || pl.w == 8 || pl.w == 16) {
         const int halo = mmax - 1;
@@ -700,9 +711,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         }
         // tau-set units: CTAs (block epilogue) or warps (diagonal kernel's warp epilogue)
         // tau units: warps of the diagonal kernel / of group_scan (w in {4,8,16,32}), else CTAs
-        const bool w_static = pl.w == 4 || pl.w == 8 || pl.w == 16 || pl.w == 32;
         const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32
-                                  : (!pl.fused && w_static) ? pl.RT / 32 : 1;
+                                  : (!pl.fused && pl.scan_reg) ? kScanThreads / 32 : 1;
         int E = 0;
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         if (!lb_only && !o.no_prune) {
@@ -862,11 +872,11 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(postbuf, d_meta, P, idx->lb.as<V>(),
                                                                idx->tauc.as<int32_t>());
             };
-            switch (w) {
-                case 4: go4(group_scan_kernel<S, 4>); break;
-                case 8: go4(group_scan_kernel<S, 8>); break;
-                case 16: go4(group_scan_kernel<S, 16>); break;
-                case 32: go4(group_scan_kernel<S, 32>); break;
+            switch (pl.scan_reg ? w : 0) {
+                case 4: go4(group_scan_reg_kernel<S, 4>); break;
+                case 8: go4(group_scan_reg_kernel<S, 8>); break;
+                case 16: go4(group_scan_reg_kernel<S, 16>); break;
+                case 32: go4(group_scan_reg_kernel<S, 32>); break;
                 default: go4(group_scan_kernel<S, 0>); break;
             }
             CHECK_LAUNCH();
