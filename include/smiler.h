@@ -228,7 +228,8 @@ SMILER_API int smiler_merge_topk(const int64_t *ids_in, const void *dists_in, sm
 SMILER_API int smiler_index_envelope(smiler_index *idx, int32_t sensor, int32_t rho, void *U, void *L);
 
 /* Steps a2-a4 only: for each MQ, the window-level posting lists (P_EQ, P_EC)
- * (may be NULL) as [n_mq][D-window+1][n_dw][2] int32/float (n_dw = floor(N/w)
+ * (may be NULL) as [n_mq][2][D-window+1][n_dw] int32/float, plane 0 = P_EQ,
+ * plane 1 = P_EC (the device layout of the two-level path; n_dw = floor(N/w)
  * of the MQ's sensor; all MQs must search sensors of equal length), and LB_w
  * per candidate as [n_mq][n_len][N] int32/float indexed by t (entries with
  * t > N - d_i are unspecified).  Envelope width rho_max as in smiler_knn. */

@@ -38,7 +38,7 @@ struct MQMeta {
     int64_t origin;      // global id of local t = 0
     int64_t t_lo, t_hi;  // owned candidate starts, local coordinates
     int64_t n_dw;        // floor(N / w) disjoint windows
-    int64_t post_off;    // offset (in pairs) of this MQ's posting lists
+    int64_t post_off;    // element offset of this MQ's P_EQ plane [n_sw][n_dw]; P_EC plane follows
     int64_t seg_off;     // offset of this MQ's per-candidate segments; (mq,i) at seg_off + i*n
     int32_t nblk;        // group-scan CTAs for this MQ
     int32_t sensor;

@@ -179,7 +179,7 @@ __device__ __forceinline__ void posting_chunk_w(const V (&c)[W], const V (&U)[W]
 // the thread's DW (c, U, L).  Window registers hold MQ positions
 // pb .. pb + W + BC - 2 (pb = D - W - b0 - (BC-1)): q, U(Q), L(Q).
 // CHECK: per-bb validity test (only for the last chunk of a CSG row).
-template <typename V, int W, int BC, bool CHECK, typename F>
+template <typename V, int W, int BC, bool CHECK, bool EQONLY = false, typename F>
 __device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], const V (&L)[W],
                                               const V *qq, const V *uq, const V *lq, int pb, int nvalid,
                                               F &&store) {
@@ -209,7 +209,7 @@ __device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], 
             for (int j = 0; j < W; j++) {
                 const int k = BC - 1 - bb + j;
                 lb_term(c[j], wu[k], wl[k], eq);
-                lb_term(wq[k], U[j], L[j], ec);
+                if constexpr (!EQONLY) lb_term(wq[k], U[j], L[j], ec);
             }
             store(bb, eq, ec);
         }
@@ -227,11 +227,8 @@ template <typename S, int W>
 __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
                                                        const MQMeta *meta,
                                                        const typename Tr<S>::V4 *qtab, int D,
-                                                       int w_rt, typename Tr<S>::V2 *post,
-                                                       int nrows = 1 << 30, int cursor = 0,
-                                                       bool incremental = false) {
+                                                       int w_rt, typename Tr<S>::V *post) {
     using V = typename Tr<S>::V;
-    using V2 = typename Tr<S>::V2;
     extern __shared__ __align__(16) unsigned char wl_smem[];
     V *sqq = reinterpret_cast<V *>(wl_smem);
     V *squ = sqq + D;
@@ -248,13 +245,13 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
     __syncthreads();
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= m.n_dw) return;
-    V2 *out = post + m.post_off + r;
+    const int64_t ndw = m.n_dw;
+    V *oe = post + m.post_off + r;  // P_EQ plane; P_EC plane `plane` further
     if constexpr (W > 0) {
         constexpr int BC = W < 8 ? W : 8;
-        const int n_sw = min(D - W + 1, nrows);  // rows [0, nrows) only (continuous step)
-        const int n_ring = D - W + 1;
+        const int n_sw = D - W + 1;
+        const int64_t plane = (int64_t)n_sw * ndw;
         const int64_t base = m.series_off + r * W;
-        const int64_t ndw = m.n_dw;
         V c[W], U[W], L[W];
 #pragma unroll
         for (int j = 0; j < W; j++) {
@@ -262,44 +259,27 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
             U[j] = (V)UC[base + j];
             L[j] = (V)LC[base + j];
         }
-        // continuous step: physical row (b + cursor) mod n_ring, and rows b >= 1 keep
-        // their LB_EC (same MQ points, same series envelope): store EQ only
-        auto put = [&](int b, V eq, V ec) {
-            int row = b + cursor;
-            row -= row >= n_ring ? n_ring : 0;
-            V2 *o = out + (int64_t)row * ndw;
-            if (incremental && b > 0) {
-                o->x = eq;
-            } else {
-                V2 v;
-                v.x = eq;
-                v.y = ec;
-                *o = v;
-            }
-        };
         int b0 = 0;
         for (; b0 + BC <= n_sw; b0 += BC) {
-            if (!incremental && cursor == 0) {
-                V2 *o = out + (int64_t)b0 * ndw;
-                posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
-                                               [&](int bb, V eq, V ec) {
-                                                   V2 v;
-                                                   v.x = eq;
-                                                   v.y = ec;
-                                                   o[bb * ndw] = v;
-                                               });
-            } else {
-                posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
-                                               [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
-            }
+            V *o = oe + (int64_t)b0 * ndw;
+            posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                           [&](int bb, V eq, V ec) {
+                                               o[bb * ndw] = eq;
+                                               o[bb * ndw + plane] = ec;
+                                           });
         }
         if (b0 < n_sw) {
+            V *o = oe + (int64_t)b0 * ndw;
             posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-                                          [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
+                                          [&](int bb, V eq, V ec) {
+                                              o[bb * ndw] = eq;
+                                              o[bb * ndw + plane] = ec;
+                                          });
         }
     } else {
         const int w = w_rt;
         const int n_sw = D - w + 1;
+        const int64_t plane = (int64_t)n_sw * ndw;
         const int64_t base = m.series_off + r * w;
         for (int b = 0; b < n_sw; b++) {
             const int p0 = D - w - b;
@@ -308,12 +288,74 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
                 lb_term((V)series[base + j], squ[p0 + j], sql[p0 + j], eq);
                 lb_term(sqq[p0 + j], (V)UC[base + j], (V)LC[base + j], ec);
             }
-            V2 o;
-            o.x = eq;
-            o.y = ec;
-            out[(int64_t)b * m.n_dw] = o;
+            oe[(int64_t)b * ndw] = eq;
+            oe[(int64_t)b * ndw + plane] = ec;
         }
     }
+}
+
+// ---------------------------------------------------------------------------
+// Continuous step, static w (Remark 1): rows b in [0, nrows) of the
+// ring (physical row (b + cursor) mod n_sw).  SW_0 gets P_EQ and P_EC; SW_1 ..
+// SW_{nrows-1} only P_EQ (their MQ envelope changed with the new point; their
+// P_EC, same MQ points against the same series envelope, is unchanged), so
+// the EC terms are not even computed and the EQ plane takes full 4-byte
+// coalesced rows.
+// ---------------------------------------------------------------------------
+template <typename S, int W>
+__global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, const S *UC, const S *LC,
+                                                           const MQMeta *meta,
+                                                           const typename Tr<S>::V4 *qtab, int D, int nrows,
+                                                           int cursor, typename Tr<S>::V *post) {
+    using V = typename Tr<S>::V;
+    constexpr int BC = W < 8 ? W : 8;
+    extern __shared__ __align__(16) unsigned char wi_smem[];
+    V *sqq = reinterpret_cast<V *>(wi_smem);
+    V *squ = sqq + D;
+    V *sql = squ + D;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int64_t)blockIdx.x * blockDim.x >= m.n_dw) return;
+    for (int p = threadIdx.x; p < D; p += blockDim.x) {
+        const typename Tr<S>::V4 e = qtab[(int64_t)mq * D + p];
+        sqq[p] = e.x;
+        squ[p] = e.y;
+        sql[p] = e.z;
+    }
+    __syncthreads();
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= m.n_dw) return;
+    const int64_t ndw = m.n_dw;
+    const int n_ring = D - W + 1;
+    const int n_sw = min(n_ring, nrows);
+    V *oe = post + m.post_off + r;
+    const int64_t base = m.series_off + r * W;
+    V c[W], U[W], L[W];
+#pragma unroll
+    for (int j = 0; j < W; j++) {
+        c[j] = (V)series[base + j];
+        U[j] = (V)UC[base + j];
+        L[j] = (V)LC[base + j];
+    }
+    auto row_ptr = [&](int b) {
+        int row = b + cursor;
+        row -= row >= n_ring ? n_ring : 0;
+        return oe + (int64_t)row * ndw;
+    };
+    // SW_0: both lists
+    posting_chunk<V, W, 1, false>(c, U, L, sqq, squ, sql, D - W, 1, [&](int, V eq, V ec) {
+        V *o = row_ptr(0);
+        o[0] = eq;
+        o[(int64_t)n_ring * ndw] = ec;
+    });
+    int b0 = 1;
+    for (; b0 + BC <= n_sw; b0 += BC)
+        posting_chunk<V, W, BC, false, true>(
+            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC, [&](int bb, V eq, V) { *row_ptr(b0 + bb) = eq; });
+    if (b0 < n_sw)
+        posting_chunk<V, W, BC, true, true>(
+            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
+            [&](int bb, V eq, V) { *row_ptr(b0 + bb) = eq; });
 }
 
 // ---------------------------------------------------------------------------
@@ -328,9 +370,8 @@ template <typename S>
 __global__ void __launch_bounds__(128) posting_rows_kernel(const S *series, const S *UC, const S *LC,
                                                           const MQMeta *meta, const typename Tr<S>::V4 *qtab,
                                                           int D, int w, int nrows, int cursor,
-                                                          typename Tr<S>::V2 *post) {
+                                                          typename Tr<S>::V *post) {
     using V = typename Tr<S>::V;
-    using V2 = typename Tr<S>::V2;
     using V4 = typename Tr<S>::V4;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
@@ -349,15 +390,9 @@ __global__ void __launch_bounds__(128) posting_rows_kernel(const S *series, cons
         }
         int row = b + cursor;
         row -= row >= n_sw ? n_sw : 0;
-        V2 *o = post + m.post_off + (int64_t)row * m.n_dw + r;
-        if (b == 0) {
-            V2 v;
-            v.x = eq;
-            v.y = ec;
-            *o = v;
-        } else {
-            o->x = eq;
-        }
+        V *o = post + m.post_off + (int64_t)row * m.n_dw + r;
+        *o = eq;
+        if (b == 0) o[(int64_t)n_sw * m.n_dw] = ec;
     }
 }
 
@@ -380,7 +415,7 @@ __global__ void __launch_bounds__(256) stream_shift_kernel(S *mq, int D, const S
 // smem: em [mmax*w] u16 | tile [n_len][RT*(w+1)] V.
 // ---------------------------------------------------------------------------
 template <typename S, int W>
-__global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V2 *post,
+__global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V *post,
                                                         const MQMeta *meta, const QParams P,
                                                         typename Tr<S>::V *lb, int32_t *tauc) {
     using V = typename Tr<S>::V;
@@ -404,7 +439,8 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
     const int64_t Rb = (int64_t)blockIdx.x * RT - 1;
     const int64_t r = Rb + threadIdx.x;
     if (r >= 0 && r < m.n_dw) {
-        const V2 *pp = post + m.post_off + r;
+        const V *pp = post + m.post_off + r;
+        const int64_t plane = (int64_t)n_sw * m.n_dw;
         V *trow = tile + threadIdx.x * (w + 1);
         for (int b = 0; b < w && b < n_sw; b++) {
             const int jmax = (n_sw - 1 - b) / w + 1;
@@ -420,7 +456,9 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
                         // (Remark 1): physical row of SW_{b+jw} = (b+jw+cursor) mod n_sw
                         int row = b + j * w + P.ring_cursor;
                         row -= row >= n_sw ? n_sw : 0;
-                        pv[u] = pp[(int64_t)row * m.n_dw - j];
+                        const V *q = pp + (int64_t)row * m.n_dw - j;
+                        pv[u].x = q[0];
+                        pv[u].y = q[plane];
                     }
                 }
 #pragma unroll
@@ -794,7 +832,7 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
 // q_i - 2 (saved) and b <= r_i after row q_i - 1, written straight from
 // registers by diag_emit (vector stores, per-warp tau set).  No shared memory,
 // no barrier.  Posting addresses are 32-bit offsets from the MQ's posting block
-// (host guarantees n_sw * n_dw < 2^31).  Only CTA 0 (DWs r < mmax - 1 lack
+// (host guarantees 2 n_sw n_dw < 2^31: both planes).  Only CTA 0 (DWs r < mmax - 1 lack
 // some r - j) and the last CSG row (fewer than w SWs) take predicated loads;
 // elsewhere threads past the last DW read DW n_dw - 1 and their slots are
 // masked at emission (t >= tend).
@@ -805,27 +843,31 @@ constexpr int kScanThreads = 256;
 #define SMILER_GS_MINB(W) ((W) <= 8 ? 4 : (W) <= 16 ? 2 : 1)
 #endif
 
-template <typename V2, int W, bool CHECK>
-__device__ __forceinline__ void gs_load_row(V2 (&pv)[W], const V2 *pp, uint32_t off, int bw, uint32_t ndw,
-                                            uint32_t wrap, int nrow, bool ok) {
+template <typename V, int W, bool CHECK>
+__device__ __forceinline__ void gs_load_row(V (&pe)[W], V (&pc)[W], const V *pp, uint32_t off, int bw,
+                                            uint32_t ndw, uint32_t wrap, int nrow, bool ok) {
 #pragma unroll
     for (int b = 0; b < W; b++) {
-        // physical rows rr + b >= n_sw wrap to the ring start (bw = n_sw - rr)
+        // physical rows rr + b >= n_sw wrap to the ring start (bw = n_sw - rr);
+        // the P_EC plane sits `wrap` (= n_sw * n_dw) elements after P_EQ
         const uint32_t o = off + (uint32_t)b * ndw - (b >= bw ? wrap : 0u);
         if constexpr (CHECK) {
-            pv[b] = V2{};
-            if (ok && b < nrow) pv[b] = __ldg(pp + o);
+            pe[b] = pc[b] = (V)0;
+            if (ok && b < nrow) {
+                pe[b] = __ldg(pp + o);
+                pc[b] = __ldg(pp + o + wrap);
+            }
         } else {
-            pv[b] = __ldg(pp + o);
+            pe[b] = __ldg(pp + o);
+            pc[b] = __ldg(pp + o + wrap);
         }
     }
 }
 
 template <typename S, int W>
 __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_reg_kernel(
-    const typename Tr<S>::V2 *post, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
+    const typename Tr<S>::V *post, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
     using V = typename Tr<S>::V;
-    using V2 = typename Tr<S>::V2;
     const int D = P.D;
     const int nl = P.n_len;
     const int n_sw = D - W + 1;
@@ -842,7 +884,7 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
     const uint32_t wrap = (uint32_t)n_sw * ndw;
     const int64_t rc = r < 0 ? 0 : (r < m.n_dw ? r : m.n_dw - 1);
     // offsets count from pp - mmax so they stay non-negative across the ring wrap
-    const V2 *pp = post + m.post_off + rc - mmax;
+    const V *pp = post + m.post_off + rc - mmax;
     // values saved after row q_i - 2 live in shared memory ([b][thread]: no
     // bank conflicts), keeping the registers for sums and loads in flight
     __shared__ V s_saved[W][kScanThreads];
@@ -866,19 +908,19 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
     // advanced by w per row (mmax >= 2 implies n_sw > w)
     int rr = P.ring_cursor;
     for (int j = 0; j < mmax; j++) {
-        V2 pv[W];
+        V pe[W], pc[W];
         const uint32_t off = (uint32_t)rr * ndw + (uint32_t)(mmax - j);
         const int nrow = n_sw - j * W;
         if (first || nrow < W)
-            gs_load_row<V2, W, true>(pv, pp, off, n_sw - rr, ndw, wrap, nrow, j < jall);
+            gs_load_row<V, W, true>(pe, pc, pp, off, n_sw - rr, ndw, wrap, nrow, j < jall);
         else
-            gs_load_row<V2, W, false>(pv, pp, off, n_sw - rr, ndw, wrap, nrow, true);
+            gs_load_row<V, W, false>(pe, pc, pp, off, n_sw - rr, ndw, wrap, nrow, true);
         rr += W;
         rr -= rr >= n_sw ? n_sw : 0;
 #pragma unroll
         for (int b = 0; b < W; b++) {
-            se[b] += pv[b].x;
-            sc[b] += pv[b].y;
+            se[b] += pe[b];
+            sc[b] += pc[b];
         }
         if (emit_rows >> j & 1ull) {
             for (int i = 0; i < nl; i++) {

@@ -482,7 +482,7 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
     for (const auto &si : idx->sensors) n_max = std::max<int64_t>(n_max, si.n);
     // register scan: emission bitmasks hold mmax rows; posting offsets are int32
     pl.scan_reg = (pl.w == 4 || pl.w == 8 || pl.w == 16 || pl.w == 32) && mmax <= 64 &&
-                  (int64_t)(pl.D - pl.w + 1) * (n_max / pl.w) < ((int64_t)1 << 31);
+                  2 * (int64_t)(pl.D - pl.w + 1) * (n_max / pl.w) < ((int64_t)1 << 31);
     if (pl.scan_reg) {
         pl.RT = kScanThreads;
         pl.smem_gs = 0;
@@ -564,8 +564,8 @@ struct PhaseTimer {
 
 // Continuous-stream context (Remark 1): posting lists live in a per-stream ring.
 struct StreamCtx {
-    void *ring;                // V2 [sum over streams of n_sw * n_dw]
-    const int64_t *ring_off;   // per stream (global index) offset into ring, in pairs
+    void *ring;                // V [sum over streams of 2 n_sw n_dw]: P_EQ plane, P_EC plane
+    const int64_t *ring_off;   // per stream (global index) element offset into ring
     int cursor;                // physical row of SW_0
     int mode;                  // 0: build every row; 1: incremental rows [0, nrows)
     int nrows;
@@ -697,7 +697,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             m.seg_off = seg_tot;
             m.nblk = (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
             m.sensor = qsens[c0 + j];
-            post_tot += (int64_t)n_sw * m.n_dw;
+            post_tot += 2 * (int64_t)n_sw * m.n_dw;  // P_EQ and P_EC planes
             seg_tot += (int64_t)nl * si.n;
             nblk_min = std::min(nblk_min, m.nblk);
             nblk_max = std::max(nblk_max, m.nblk);
@@ -758,7 +758,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         ENS(idx->queries.ensure(es * (size_t)B * D));
         ENS(idx->qv.ensure(sizeof(V) * (size_t)B * D));
         ENS(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
-        if (!sctx) ENS(idx->post.ensure(sizeof(V2) * (size_t)std::max<int64_t>(post_tot, 1)));
+        if (!sctx) ENS(idx->post.ensure(sizeof(V) * (size_t)std::max<int64_t>(post_tot, 1)));
         ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
         if (!lb_only) {
             ENS(idx->surv.ensure(4 * (size_t)seg_tot));
@@ -789,7 +789,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
             TRY(rc_);
         }
-        V2 *postbuf = sctx ? reinterpret_cast<V2 *>(sctx->ring) : idx->post.as<V2>();
+        V *postbuf = sctx ? reinterpret_cast<V *>(sctx->ring) : idx->post.as<V>();
         MQMeta *d_meta = idx->meta.as<MQMeta>();
         CU(cudaMemcpyAsync(d_meta, meta, sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
         CU(cudaEventRecord(idx->meta_ev[mslot], idx->stream));
@@ -841,17 +841,33 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     sctx->nrows, sctx->cursor, postbuf);
                 CHECK_LAUNCH();
                 launches++;
-            } else if (ndw_max > 0) {
-                const bool inc = sctx && sctx->mode == 1;
-                const int nrows = inc ? sctx->nrows : (1 << 30);
-                const int cur = sctx ? sctx->cursor : 0;
+            } else if (ndw_max > 0 && sctx && sctx->mode == 1) {
+                // continuous step, static w: SW_0 (EQ + EC) and SW_1..SW_rho (EQ only)
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
                 size_t smem = 3 * sizeof(V) * D;
                 auto go = [&](auto kern) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           w, postbuf, nrows, cur, inc);
+                                                           sctx->nrows, sctx->cursor, postbuf);
+                };
+                switch (w) {
+                    case 4: go(window_lb_inc_kernel<S, 4>); break;
+                    case 8: go(window_lb_inc_kernel<S, 8>); break;
+                    case 16: go(window_lb_inc_kernel<S, 16>); break;
+                    default: go(window_lb_inc_kernel<S, 32>); break;
+                }
+                CHECK_LAUNCH();
+                launches++;
+            } else if (ndw_max > 0) {
+                // every row (ring cursor 0 when a stream is created)
+                dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
+                size_t smem = 3 * sizeof(V) * D;
+                auto go = [&](auto kern) {
+                    set_smem((const void *)kern, smem);
+                    kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
+                                                           (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
+                                                           w, postbuf);
                 };
                 switch (w) {
                     case 4: go(window_lb_kernel<S, 4>); break;
@@ -863,7 +879,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 CHECK_LAUNCH();
                 launches++;
             }
-            post_bytes += post_tot * 8;
+            post_bytes += post_tot * (int64_t)sizeof(V);
             TRY(tm.mark(2));
             // ---- a4 ----------------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
@@ -891,8 +907,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             CU(cudaMemcpyAsync((char *)lb_out + lb_off * sizeof(V), idx->lb.p, lbb,
                                out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
             if (post_out) {
-                const int64_t po = (int64_t)n_sw * meta[0].n_dw * c0;
-                CU(cudaMemcpyAsync((char *)post_out + po * sizeof(V2), idx->post.p, sizeof(V2) * (size_t)post_tot,
+                const int64_t po = 2 * (int64_t)n_sw * meta[0].n_dw * c0;
+                CU(cudaMemcpyAsync((char *)post_out + po * sizeof(V), idx->post.p, sizeof(V) * (size_t)post_tot,
                                    out_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, idx->stream));
             }
             c0 = c1;
@@ -1140,17 +1156,17 @@ extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, cons
             return fail(SMILER_EINVAL, "query_sensor[%d] out of range", j);
         }
         st->ring_off[j] = tot;
-        tot += (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
+        tot += 2 * (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
     }
     const size_t es = esize(idx->dtype);
-    cudaError_t e = cudaMalloc(&st->ring, 8 * (size_t)std::max<int64_t>(tot, 1));
+    cudaError_t e = cudaMalloc(&st->ring, 4 * (size_t)std::max<int64_t>(tot, 1));
     if (e == cudaSuccess) e = cudaMalloc(&st->d_mq, es * (size_t)n_streams * pl.D);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_new, es * (size_t)n_streams);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_prev, 8 * (size_t)n_streams * n_len * k);
     if (e != cudaSuccess) {
         cudaGetLastError();
         stream_release(st);
-        return fail(SMILER_ENOMEM, "stream buffers (%lld posting pairs): %s", (long long)tot, cudaGetErrorString(e));
+        return fail(SMILER_ENOMEM, "stream buffers (%lld posting entries): %s", (long long)tot, cudaGetErrorString(e));
     }
     e = cudaMemcpyAsync(st->d_mq, queries, es * (size_t)n_streams * pl.D, cudaMemcpyDefault, idx->stream);
     if (e != cudaSuccess) {

@@ -335,7 +335,7 @@ class Index:
         postings=False: the fused path (returns post=None)."""
         n_mq, D = queries.shape
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32
-        post = np.empty((n_mq, D - window + 1, n // window, 2), vt) if postings else None
+        post = np.empty((n_mq, 2, D - window + 1, n // window), vt) if postings else None
         lbw = np.empty((n_mq, len(lengths), n), vt)
         smiler_lower_bounds(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, post, lbw)
         return post, lbw

@@ -113,11 +113,11 @@ def test_postings_and_lbw(pkg, orc, dtype, cfg, n, lengths, window, band):
                 else:
                     np.testing.assert_allclose(got, exp, rtol=2e-5, atol=1e-6)
         if dtype == "i16":
-            np.testing.assert_array_equal(post[j, :, :, 0].astype(np.int64), PE)
-            np.testing.assert_array_equal(post[j, :, :, 1].astype(np.int64), PC)
+            np.testing.assert_array_equal(post[j, 0].astype(np.int64), PE)
+            np.testing.assert_array_equal(post[j, 1].astype(np.int64), PC)
         else:
-            np.testing.assert_allclose(post[j, :, :, 0], PE, rtol=2e-5, atol=1e-6)
-            np.testing.assert_allclose(post[j, :, :, 1], PC, rtol=2e-5, atol=1e-6)
+            np.testing.assert_allclose(post[j, 0], PE, rtol=2e-5, atol=1e-6)
+            np.testing.assert_allclose(post[j, 1], PC, rtol=2e-5, atol=1e-6)
 
 
 # ---------------------------------------------------------------------------
@@ -163,8 +163,8 @@ def test_golden_appendix_a_gpu(pkg, orc, dtype):
         assert ids[0, li].tolist() == iq["knn_ids"]
         assert (dists[0, li] * scale).tolist() == iq["knn_dists"]
         assert (lbw[0, li, :len(iq["t"])] * scale).tolist() == iq["LB_w"]
-    assert (post[0, :, :, 0] * scale).tolist() == g["P_EQ"]
-    assert (post[0, :, :, 1] * scale).tolist() == g["P_EC"]
+    assert (post[0, 0] * scale).tolist() == g["P_EQ"]
+    assert (post[0, 1] * scale).tolist() == g["P_EC"]
 
 
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
