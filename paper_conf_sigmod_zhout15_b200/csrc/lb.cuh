@@ -642,24 +642,35 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int unit = blockIdx.x * nw + warp;  // tau units are warps
     int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)unit * P.E;
-    uint32_t taken = 0;
-    for (int e = 0; e < P.E; e++) {
-        uint64_t best = kKeyMax;
-        int bs = -1;
+    // The E smallest (LB_w, t) keys of the warp with 32-bit compares only: t
+    // grows with the slot b inside a thread and with the lane across the warp,
+    // so among equal LB_w bits the lowest lane, then the lowest b, has the
+    // smallest t (the same keys as a 64-bit (LB_w bits << 32 | t) minimum).
+    uint32_t kb[W];
 #pragma unroll
-        for (int b = 0; b < W; b++) {
-            const int64_t t = t0 + b;
-            if (!(taken >> b & 1u) && t >= tmin && t < tend) {
-                const uint64_t key = ((uint64_t)key_bits(v[b]) << 32) | (uint32_t)t;
-                if (key < best) {
-                    best = key;
-                    bs = b;
-                }
+    for (int b = 0; b < W; b++) {
+        const int64_t t = t0 + b;
+        kb[b] = (t >= tmin && t < tend) ? key_bits(v[b]) : 0xFFFFFFFFu;
+    }
+    for (int e = 0; e < P.E; e++) {
+        uint32_t best = kb[0];
+        int bs = 0;
+#pragma unroll
+        for (int b = 1; b < W; b++) {
+            if (kb[b] < best) {
+                best = kb[b];
+                bs = b;
             }
         }
-        const uint64_t win = warp_min_u64(best);
-        if (win != kKeyMax && best == win) taken |= 1u << bs;
-        if (lane == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+        const uint32_t win = __reduce_min_sync(0xffffffffu, best);
+        const int wl = __ffs(__ballot_sync(0xffffffffu, best == win)) - 1;
+        const int tw = __shfl_sync(0xffffffffu, (int)(t0 + bs), wl);
+        if (lane == wl) {
+#pragma unroll
+            for (int b = 0; b < W; b++)
+                if (b == bs) kb[b] = 0xFFFFFFFFu;
+        }
+        if (lane == 0) dst[e] = win != 0xFFFFFFFFu ? tw : -1;
     }
 }
 
@@ -727,6 +738,8 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
     }
     const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
     const int64_t R0 = Rb - HALO;  // DW of tile column 0
+    // 8 iterations' loads in flight before their shared-memory stores
+#pragma unroll 8
     for (int idx = threadIdx.x; idx < NC * W; idx += NT) {
         const int col = idx / W, jj = idx % W;
         const int64_t rp = R0 + col;
@@ -769,12 +782,19 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
             L[jj] = l.x, L[jj + 1] = l.y, L[jj + 2] = l.z, L[jj + 3] = l.w;
         }
         const int nrow = min(W, n_sw - j * W);
-#pragma unroll
-        for (int b0 = 0; b0 < W; b0 += BC) {
+        // W / BC chunks of BC sliding windows.  With more than one chunk the
+        // chunk loop is NOT unrolled (a fully unrolled w = 16 row is 2048 ALU
+        // instructions, 32 KB of code: it thrashes the 32 KB L1.5 I-cache); the
+        // chunk always accumulates into slots 0..BC-1 and the slot arrays are
+        // rotated by BC afterwards (identity again after W / BC chunks).
+        constexpr int NCH = W / BC;
+#pragma unroll 1
+        for (int h = 0; h < NCH; h++) {
+            const int b0 = h * BC;
             const int nv = nrow - b0;
             auto acc = [&](int bb, V eq, V ec) {
-                se[b0 + bb] += eq;
-                sc[b0 + bb] += ec;
+                se[bb] += eq;
+                sc[bb] += ec;
             };
             const int pb = D - W - j * W - b0 - (BC - 1);
             if (nv >= BC) {  // full chunk: aligned 16-byte window loads
@@ -792,6 +812,15 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                 posting_chunk_w<V, W, BC, false, WL>(c, U, L, wq, wu, wl, BC, acc);
             } else if (nv > 0) {
                 posting_chunk<V, W, BC, true>(c, U, L, sqq + qshift, squ + qshift, sql + qshift, pb, nv, acc);
+            }
+            if (NCH > 1) {  // rotate the slots left by BC
+                V te[BC], tc[BC];
+#pragma unroll
+                for (int b = 0; b < BC; b++) te[b] = se[b], tc[b] = sc[b];
+#pragma unroll
+                for (int b = 0; b + BC < W; b++) se[b] = se[b + BC], sc[b] = sc[b + BC];
+#pragma unroll
+                for (int b = 0; b < BC; b++) se[W - BC + b] = te[b], sc[W - BC + b] = tc[b];
             }
         }
         if (P.k < 0) continue;  // timing experiment: main loop only
