@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define SMILER_ABI_VERSION 1
+#define SMILER_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define SMILER_API __attribute__((visibility("default")))
@@ -79,8 +79,37 @@ typedef struct smiler_knn_opts {
     int32_t two_level;/* 1: materialise the window-level posting lists in HBM (a3) and
                          scan them (a4), as the paper's two-level index; 0: automatic
                          (fused a3+a4 with posting rows kept on chip when w is 4/8/16) */
+    int32_t lb_kind;  /* which lower bound filters the candidates (SMILER_LB_*); all of
+                         them are valid DTW lower bounds, so the kNN result is the same */
+    int32_t horizon;  /* h >= 0: only segments C_{t,d} whose h-step-ahead value
+                         c_{t+d-1+h} exists are candidates, i.e. t <= N - d - h (the
+                         kNN data (X_{k,d}, Y_h) of the predictors);
+                         0 = every segment (Def. 4.1).  Shards: N is the full series. */
     int32_t reserved[4];
 } smiler_knn_opts;
+
+/* smiler_knn_opts.lb_kind.  The default is the paper's method; the others are
+ * the ablations of Table 3 and Fig. 8 (P:1916-1919,
+ * P:2094-2102).
+ *   SMILER_LB_INDEX     LB_w = max(sum EQ, sum EC) over the full disjoint windows
+ *                       of the candidate, through the two-level index (Thm 4.3,
+ *                       Eq. 5)
+ *   SMILER_LB_INDEX_EQ  the EQ sum of LB_w only ("LB_EQ" row of Table 3)
+ *   SMILER_LB_INDEX_EC  the EC sum of LB_w only ("LB_EC" row of Table 3)
+ *   SMILER_LB_DIRECT    SMiLer-Dir: LB_en = max(LB_EQ, LB_EC) over all d_i points of
+ *                       the candidate (Thm 4.1), computed directly from
+ *                       the series for each item query separately
+ *   SMILER_LB_DIRECT_SHARED  the same LB_en values for every item query from ONE
+ *                       pass: item queries are suffixes of the MQ, so
+ *                       the candidates of all item queries that end at the same
+ *                       series point share one running sum (cf. Remark 2) */
+enum {
+    SMILER_LB_INDEX = 0,
+    SMILER_LB_INDEX_EQ = 1,
+    SMILER_LB_INDEX_EC = 2,
+    SMILER_LB_DIRECT = 3,
+    SMILER_LB_DIRECT_SHARED = 4
+};
 
 /*
  * smiler_index_build -- upload sensor series and build the index (a1).
@@ -236,6 +265,50 @@ SMILER_API int smiler_index_envelope(smiler_index *idx, int32_t sensor, int32_t 
 SMILER_API int smiler_lower_bounds(smiler_index *idx, const void *queries, const int32_t *query_sensor,
                         int32_t n_mq, const int32_t *lengths, int32_t n_len, void *postings,
                         void *lbw);
+
+/* Steps a2-a4 with the lower bound `lb_kind` (SMILER_LB_*): the per-candidate
+ * bound that smiler_knn_ex filters with, as [n_mq][n_len][N] int32/float
+ * indexed by t (entries with t > N - d_i unspecified).  SMILER_LB_INDEX gives
+ * the LB_w of smiler_lower_bounds; SMILER_LB_INDEX_EQ / _EC its two sums
+ * (Eq. 5); SMILER_LB_DIRECT / _DIRECT_SHARED give LB_en (Thm 4.1) per
+ * candidate, with the series envelope of width rho_max and the MQ envelope
+ * (R4, R20).  All MQs must search sensors of equal length.
+ * Errors: EINVAL (NULL lb, bad lb_kind, as smiler_knn), ENOMEM, ECUDA. */
+SMILER_API int smiler_lower_bounds_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                        int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t lb_kind,
+                        void *lb);
+
+/*
+ * smiler_predict -- the predictors that consume the kNN (
+ * Sec. 5.2; App. B.3).
+ *
+ * For master query m (its sensor query_sensor[m], NULL -> 0), item query i
+ * (IQ_i = the last lengths[i] points of queries[m]) and k_j = ekv[j],
+ * the predictor f_{i,j} uses the kNN data of the first k_j neighbours
+ * ids[m][i][0..k_j) (multi-k by prefix):
+ *   X = {c[t_a .. t_a+d_i)},  Y_h = {c[t_a + d_i - 1 + horizon]}
+ * and returns
+ *   ar_mean, ar_var  Eq. 12-13: mean of Y_h and sum (y - mean)^2 / k_j
+ *   gp_mean, gp_var  Eq. 16-17 with the covariance of Eq. 18,
+ *                    c(x_a, x_b) = th0^2 exp(-|x_a - x_b|^2 / (2 th1^2)) + delta_ab th2^2,
+ *                    c(x0, x0) = th0^2 + th2^2 (reading P1)
+ * theta: [n_mq][n_len][n_k][3] doubles (th0, th1, th2) per predictor (their
+ * online training, Eq. 19-20, is not part of the library).
+ * ids: the smiler_knn output [n_mq][n_len][k] (run it with
+ * smiler_knn_opts.horizon = horizon so every neighbour has its h-step-ahead
+ * value); a predictor whose first k_j ids contain -1 or a t with
+ * t + d_i - 1 + horizon >= N, or whose C is not positive definite, gets NaN.
+ * Outputs: [n_mq][n_len][n_k] doubles each, row-major.  Every pointer may be
+ * host or device memory; the call returns when the outputs are written.
+ * Arithmetic: fp64 (Cholesky factor of C in shared memory).
+ * Errors: EINVAL (NULL argument, shard index, n_len or lengths as smiler_knn,
+ *         ekv not strictly increasing within [1, min(k, 128)], n_k > 64,
+ *         horizon < 0, bad sensor), ENOMEM, ECUDA.
+ */
+SMILER_API int smiler_predict(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                   int32_t n_mq, const int32_t *lengths, int32_t n_len, const int64_t *ids, int32_t k,
+                   const int32_t *ekv, int32_t n_k, int32_t horizon, const double *theta,
+                   double *ar_mean, double *ar_var, double *gp_mean, double *gp_var);
 
 /* Step a7 only: banded DTW (Eq. 21-24) of item query q[0..d) against
  * C_{t,d} of `sensor` for each t in ts[0..n_t), warping width rho.  dists:

@@ -61,8 +61,8 @@ def lib():
         L.orc_dtw_list_f32.argtypes = [P, P, i32, i32, P, i64, P, P]
         L.orc_postings_i64.argtypes = [P, i64, P, P, P, P, P, i32, i32, P, P]
         L.orc_postings_f64.argtypes = [P, i64, P, P, P, P, P, i32, i32, P, P]
-        L.orc_lb_i64.argtypes = [P, i64, P, P, P, P, P, i32, i32, i32, P, P, P, P, P, P, P]
-        L.orc_lb_f64.argtypes = [P, i64, P, P, P, P, P, i32, i32, i32, P, P, P, P]
+        L.orc_lb_i64.argtypes = [P, i64, P, P, P, P, P, i32, i32, i32, P, P, P, P, P, P, P, P, P]
+        L.orc_lb_f64.argtypes = [P, i64, P, P, P, P, P, i32, i32, i32, P, P, P, P, P, P]
         _lib = L
     return _lib
 
@@ -217,17 +217,18 @@ def lower_bounds(c: np.ndarray, UC, LC, mq, UQ, LQ, d: int, w: int) -> Dict[str,
     nt = max(n - d + 1, 0)
     if _is_int(c):
         cv = lambda a: np.ascontiguousarray(a, np.int64)
-        out = {k: np.empty(nt, np.int64) for k in ("eq", "ec", "en", "w", "b", "r", "m")}
+        out = {k: np.empty(nt, np.int64) for k in ("eq", "ec", "en", "w", "b", "r", "m", "weq", "wec")}
         args = [cv(c), cv(UC), cv(LC), cv(mq), cv(UQ), cv(LQ)]
         lib().orc_lb_i64(_p(args[0]), n, _p(args[1]), _p(args[2]), _p(args[3]), _p(args[4]),
                          _p(args[5]), D, d, w, _p(out["eq"]), _p(out["ec"]), _p(out["en"]),
-                         _p(out["w"]), _p(out["b"]), _p(out["r"]), _p(out["m"]))
+                         _p(out["w"]), _p(out["b"]), _p(out["r"]), _p(out["m"]), _p(out["weq"]), _p(out["wec"]))
         return out
     cv = lambda a: np.ascontiguousarray(a, np.float64)
-    out = {k: np.empty(nt, np.float64) for k in ("eq", "ec", "en", "w")}
+    out = {k: np.empty(nt, np.float64) for k in ("eq", "ec", "en", "w", "weq", "wec")}
     args = [cv(c), cv(UC), cv(LC), cv(mq), cv(UQ), cv(LQ)]
     lib().orc_lb_f64(_p(args[0]), n, _p(args[1]), _p(args[2]), _p(args[3]), _p(args[4]),
-                     _p(args[5]), D, d, w, _p(out["eq"]), _p(out["ec"]), _p(out["en"]), _p(out["w"]))
+                     _p(args[5]), D, d, w, _p(out["eq"]), _p(out["ec"]), _p(out["en"]), _p(out["w"]),
+                     _p(out["weq"]), _p(out["wec"]))
     return out
 
 

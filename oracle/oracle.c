@@ -420,11 +420,13 @@ void orc_postings_f64(const double *c, int64_t n, const double *UC, const double
  *   b      = t + d - (r+1) w           (Thm. 4.2 proof)
  *   LB_w   = max(sum over s in [r_left w, (r+1) w) of the EQ terms,
  *                same for the EC terms)              if m >= 1, else 0 (R6)
- * Outputs (each [n-d+1]): lb_eq, lb_ec, lb_en, lb_w, and b, r, m. */
+ * Outputs (each [n-d+1]): lb_eq, lb_ec, lb_en, lb_w, and b, r, m; lb_weq and
+ * lb_wec (may be NULL) are the two sums inside LB_w's max (Eq. 5), the bounds
+ * of Table 3's "LB_EQ" / "LB_EC" rows over the full windows. */
 void orc_lb_i64(const int64_t *c, int64_t n, const int64_t *UC, const int64_t *LC,
                 const int64_t *mq, const int64_t *UQ, const int64_t *LQ, int D, int d, int w,
                 int64_t *lb_eq, int64_t *lb_ec, int64_t *lb_en, int64_t *lb_w,
-                int64_t *ob, int64_t *orr, int64_t *om)
+                int64_t *ob, int64_t *orr, int64_t *om, int64_t *lb_weq, int64_t *lb_wec)
 {
     for (int64_t t = 0; t + d <= n; t++) {
         int64_t eq = 0, ec = 0, weq = 0, wec = 0;
@@ -446,6 +448,8 @@ void orc_lb_i64(const int64_t *c, int64_t n, const int64_t *UC, const int64_t *L
         lb_ec[t] = ec;
         lb_en[t] = eq > ec ? eq : ec;
         lb_w[t] = m >= 1 ? (weq > wec ? weq : wec) : 0;
+        if (lb_weq) lb_weq[t] = m >= 1 ? weq : 0;
+        if (lb_wec) lb_wec[t] = m >= 1 ? wec : 0;
         ob[t] = t + d - (r + 1) * w;
         orr[t] = r;
         om[t] = m;
@@ -454,7 +458,7 @@ void orc_lb_i64(const int64_t *c, int64_t n, const int64_t *UC, const int64_t *L
 
 void orc_lb_f64(const double *c, int64_t n, const double *UC, const double *LC,
                 const double *mq, const double *UQ, const double *LQ, int D, int d, int w,
-                double *lb_eq, double *lb_ec, double *lb_en, double *lb_w)
+                double *lb_eq, double *lb_ec, double *lb_en, double *lb_w, double *lb_weq, double *lb_wec)
 {
     for (int64_t t = 0; t + d <= n; t++) {
         double eq = 0, ec = 0, weq = 0, wec = 0;
@@ -476,5 +480,7 @@ void orc_lb_f64(const double *c, int64_t n, const double *UC, const double *LC,
         lb_ec[t] = ec;
         lb_en[t] = eq > ec ? eq : ec;
         lb_w[t] = m >= 1 ? (weq > wec ? weq : wec) : 0.0;
+        if (lb_weq) lb_weq[t] = m >= 1 ? weq : 0.0;
+        if (lb_wec) lb_wec[t] = m >= 1 ? wec : 0.0;
     }
 }

@@ -9,9 +9,12 @@ process groups.
 from .smiler import (Index, KnnOpts, KnnStats, SmilerError, Stream, smiler_stream_create, smiler_stream_free,
                      smiler_stream_step, smiler_abi_version, smiler_dtw,  # noqa: F401
                      smiler_free, smiler_index_build, smiler_index_build_shard, smiler_index_envelope,
-                     smiler_knn, smiler_knn_step, smiler_lower_bounds, smiler_merge_topk)
+                     smiler_knn, smiler_knn_step, smiler_lower_bounds, smiler_lower_bounds_ex, smiler_merge_topk,
+                     smiler_predict,
+                     LB_KINDS)
 
 __all__ = ["Index", "KnnOpts", "KnnStats", "SmilerError", "Stream", "smiler_stream_create", "smiler_stream_free",
            "smiler_stream_step", "smiler_abi_version", "smiler_dtw", "smiler_free",
            "smiler_index_build", "smiler_index_build_shard", "smiler_index_envelope", "smiler_knn", "smiler_knn_step",
-           "smiler_lower_bounds", "smiler_merge_topk"]
+           "smiler_lower_bounds", "smiler_lower_bounds_ex", "smiler_merge_topk", "LB_KINDS",
+           "smiler_predict"]

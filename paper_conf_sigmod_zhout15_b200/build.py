@@ -19,11 +19,12 @@ ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libsmiler.so")
 BUILD = os.path.join(HERE, "_build")
 ALU_BENCH = os.path.join(BUILD, "alu_bench")
-SOURCES = ["smiler.cu", "dtw.cu"]
+SOURCES = ["smiler.cu", "dtw.cu", "predict.cu"]
 HEADERS = ["internal.h", "kernels.cuh", "lb.cuh", os.path.join("..", "..", "include", "smiler.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
+         "-Xcompiler", "-Werror=return-type",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
 # tuning experiments only (tools/): extra -D knobs, e.g. "-DSMILER_GS_MINB=3"
 FLAGS += os.environ.get("SMILER_EXTRA_NVFLAGS", "").split()

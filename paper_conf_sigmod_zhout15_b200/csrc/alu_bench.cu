@@ -215,6 +215,26 @@ __global__ void __launch_bounds__(kThreads) dtw_f32x2_mix(float *out, long long 
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
+// fp64 FMA (the predictors' Gram / Cholesky arithmetic, smiler_predict):
+// independent DFMA chains; unit = one DFMA (2 flops)
+__global__ void __launch_bounds__(kThreads) dfma_mix(double *out, long long *cyc, double q0) {
+    double a[kChains];
+    const double c = 1.0 + threadIdx.x * 1e-9;
+#pragma unroll
+    for (int i = 0; i < kChains; i++) a[i] = i * 0.5 + q0;
+    long long t0 = clock64();
+    for (int it = 0; it < kIters; it++) {
+#pragma unroll
+        for (int i = 0; i < kChains; i++) a[i] = fma(a[i], c, -0.5);
+    }
+    long long t1 = clock64();
+    double s = 0;
+#pragma unroll
+    for (int i = 0; i < kChains; i++) s += a[i];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+}
+
 struct Rate {
     double per_clk_sm;  // units per SM per SM clock
     double mhz;         // effective SM clock during the run
@@ -266,7 +286,7 @@ int main(int argc, char **argv) {
     const int per_sm = argc > 2 ? atoi(argv[2]) : 8;  // CTAs of 256 threads per SM (8 = 64 warps)
     const float min_ms = argc > 1 ? (float)atof(argv[1]) : 400.f;
     // interleaved, sustained: each mix twice, keep the second (steady clock)
-    Rate r[7];
+    Rate r[8];
     for (int pass = 0; pass < 2; pass++) {
         r[0] = run(dtw_f32_mix, 1.0f, sms, per_sm, 1.0, min_ms);
         r[1] = run(dtw_f32x2_mix, 1.0f, sms, per_sm, 2.0, min_ms);
@@ -275,18 +295,19 @@ int main(int argc, char **argv) {
         r[4] = run(dtw_i32_mix, 1, sms, per_sm, 1.0, min_ms);
         r[5] = run(lbterm_i32_mix, 1, sms, per_sm, 1.0, min_ms);
         r[6] = run(lbterm_max3_mix, 0.1f, sms, per_sm, 1.0, min_ms);
+        r[7] = run(dfma_mix, 1.0, sms, per_sm, 1.0, min_ms);
     }
     cudaError_t e = cudaGetLastError();
-    const char *names[7] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32",
-                            "lbterm_max3"};
+    const char *names[8] = {"dtw_cell_f32", "dtw_cell_f32x2", "lbterm", "lbterm_f32x2", "dtw_cell_i32", "lbterm_i32",
+                            "lbterm_max3", "dfma"};
     printf("{\"sms\": %d, \"ctas_per_sm\": %d, \"sustained_ms_per_mix\": %.0f", sms, per_sm, min_ms);
-    for (int i = 0; i < 7; i++)
+    for (int i = 0; i < 8; i++)
         printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e", names[i], r[i].per_clk_sm,
                names[i], r[i].mhz, names[i], r[i].per_s);
     printf(", \"note\": \"units per SM per SM clock and per second over back-to-back full waves (8 CTAs x 256 threads "
            "per SM, 8 independent chains per thread), sustained for the stated time; dtw cell = FADD+FMNMX3+FFMA (f32), "
            "f32x2 = FADD2+2 FMNMX3+FFMA2 per 2 cells, i32 = IADD+VIMNMX3+IMAD(+LOP); lbterm = one (SW,DW,j) EQ+EC "
-           "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), lbterm_max3 = 2x(FADD,FADD,FMNMX3,FFMA) (the kernels' form), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2\", \"cuda\": \"%s\"}\n",
+           "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), lbterm_max3 = 2x(FADD,FADD,FMNMX3,FFMA) (the kernels' form), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2; dfma = one fp64 FMA (2 flops)\", \"cuda\": \"%s\"}\n",
            cudaGetErrorString(e));
     return e == cudaSuccess ? 0 : 1;
 }

@@ -28,7 +28,10 @@
 
 namespace smiler {
 
-constexpr int kDtwThreads = 256;
+#ifndef SMILER_DTW_THREADS
+#define SMILER_DTW_THREADS 256
+#endif
+constexpr int kDtwThreads = SMILER_DTW_THREADS;
 constexpr int kDtwWarps = kDtwThreads / 32;
 constexpr int kRows = 4;                       // rows per register block
 

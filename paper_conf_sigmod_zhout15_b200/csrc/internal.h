@@ -14,6 +14,7 @@ constexpr int kMaxK = 1024;      // max k
 constexpr int kMaxWindow = 64;   // max omega
 constexpr int kMaxRhoFast = 32;  // rho handled by the register-band DTW kernels
 constexpr int kSortCap = 4096;   // keys sorted in shared memory by one CTA
+constexpr int kMaxPredK = 128;   // neighbours per GP predictor (k x k fp64 factor in shared memory)
 constexpr uint64_t kKeyMax = ~0ull;
 
 // Value type of the arithmetic for a storage type (R16, R17).
@@ -40,6 +41,8 @@ struct MQMeta {
     int64_t n_dw;        // floor(N / w) disjoint windows
     int64_t post_off;    // element offset of this MQ's P_EQ plane [n_sw][n_dw]; P_EC plane follows
     int64_t seg_off;     // offset of this MQ's per-candidate segments; (mq,i) at seg_off + i*n
+    int64_t hz;          // prediction horizon h (local): candidates must end by n - hz (C_{t,d} with
+                         // c_{t+d-1+h} in the series); 0 = every segment
     int32_t nblk;        // group-scan CTAs for this MQ
     int32_t sensor;
 };
@@ -48,6 +51,7 @@ struct MQMeta {
 struct QParams {
     int D, w, n_len, k, rho_env, E, LT, n_mq;
     int ring_cursor;  // continuous streams: physical posting row of SW_b is (b + ring_cursor) mod n_sw
+    int lbsel;        // which sums make the bound: 0 = max(EQ, EC) (Eq. 5 / Thm 4.1), 1 = EQ, 2 = EC
     int len[kMaxLen];
     int rho[kMaxLen];
 };

@@ -315,7 +315,7 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
     const MQMeta m = meta[mq];
     const int d = P.len[i];
     const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
-    const int64_t te = min(m.t_hi, m.n - d + 1);
+    const int64_t te = min(m.t_hi, m.n - m.hz - d + 1);
     const int64_t t0 = tb + (int64_t)blockIdx.x * kFiltThreads * kFiltItems;
     if (t0 >= te) return;
     const uint32_t th = thr[seg];
@@ -352,7 +352,7 @@ __global__ void all_candidates_kernel(const MQMeta *meta, const QParams P, int32
     const MQMeta m = meta[mq];
     const int d = P.len[i];
     const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
-    const int64_t te = min(m.t_hi, m.n - d + 1);
+    const int64_t te = min(m.t_hi, m.n - m.hz - d + 1);
     const int64_t nc = te > tb ? te - tb : 0;
     int32_t *dst = surv + m.seg_off + (int64_t)i * m.n;
     for (int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < nc;
@@ -491,7 +491,7 @@ __global__ void prev_tau_kernel(const int64_t *prev, int shift, const MQMeta *me
     const int mq = seg / P.n_len, i = seg % P.n_len;
     const MQMeta m = meta[mq];
     const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
-    const int64_t te = min(m.t_hi, m.n - P.len[i] + 1);
+    const int64_t te = min(m.t_hi, m.n - m.hz - P.len[i] + 1);
     for (int j = threadIdx.x; j < P.k; j += blockDim.x) {
         const int64_t id = prev[(int64_t)seg * P.k + j];
         int64_t t = id >= 0 ? id - m.origin + shift : -1;

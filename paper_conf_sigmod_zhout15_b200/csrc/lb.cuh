@@ -22,6 +22,25 @@
 #pragma once
 // (included inside namespace smiler by kernels.cuh)
 
+// The bound of a candidate from its EQ and EC sums: LB = max(EQ, EC) (Eq. 5,
+// Thm 4.1), or one of the two sums alone (the Table 3 ablation).
+template <typename V> __device__ __forceinline__ V lbpick(const QParams &P, V eq, V ec) {
+    return P.lbsel == 0 ? vmax(eq, ec) : (P.lbsel == 1 ? eq : ec);
+}
+
+// CTAs past an MQ's last tile (grids are sized for the longest sensor of the
+// chunk) still own tau-list slots: mark them empty (-1) so the tau DTW pass
+// never reads a stale t from an earlier call.
+__device__ __forceinline__ void tau_clear(const QParams &P, int mq, int units_per_blk, int li0, int li1,
+                                          int32_t *tauc) {
+    if (P.E <= 0 || P.k < 0) return;
+    const int n = units_per_blk * P.E;
+    for (int i = li0; i < li1; i++) {
+        int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)blockIdx.x * n;
+        for (int x = threadIdx.x; x < n; x += blockDim.x) dst[x] = -1;
+    }
+}
+
 // emission table: em[j*w + b] = lo | hi << 8, the IQ range [lo, hi) with
 // m_i(b) == j + 1 (contiguous in i because d_i increases).
 __device__ __forceinline__ void build_emit_table(uint16_t *em, int mmax, int w, const QParams &P) {
@@ -47,7 +66,7 @@ __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, c
     const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
     for (int i = 0; i < nl; i++) {
         const int d = P.len[i];
-        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
         V *out = lb + m.seg_off + (int64_t)i * m.n;
         V *row = tile + i * stride;
         uint64_t best = kKeyMax;
@@ -109,7 +128,7 @@ __device__ void lb_tile_epilogue_warp(V *tile, int RT, int64_t e0, const MQMeta 
     const int64_t s0 = e0 + (int64_t)x * W;  // e of this thread's slot 0
     for (int i = 0; i < nl; i++) {
         const int d = P.len[i];
-        const int64_t tend = min(m.t_hi, m.n - d + 1);
+        const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
         V *out = lb + m.seg_off + (int64_t)i * m.n;
         V *row = tile + i * stride + x * (W + 1);
         uint64_t best = kKeyMax;
@@ -432,7 +451,10 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
     V *tile = reinterpret_cast<V *>(gs_smem + ((mmax * w * 2 + 15) & ~15));
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) return;
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, 1, 0, P.n_len, tauc);
+        return;
+    }
     build_emit_table(em, mmax, w, P);
     for (int x = threadIdx.x; x < nl * stride; x += RT) tile[x] = (V)0;
     __syncthreads();
@@ -468,7 +490,7 @@ __global__ void __launch_bounds__(256) group_scan_kernel(const typename Tr<S>::V
                         se += pv[u].x;
                         sc += pv[u].y;
                         const int rng = em[j * w + b];
-                        const V lbv = vmax(se, sc);
+                        const V lbv = lbpick(P, se, sc);
                         for (int i = rng & 255; i < (rng >> 8); i++) trow[i * stride + b] = lbv;
                     }
                 }
@@ -525,7 +547,10 @@ __global__ void __launch_bounds__(kFusedThreads, (W <= 8 ? 3 : 1)) lb_fused_kern
     V *tile = sql + D;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) return;
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, 1, 0, P.n_len, tauc);
+        return;
+    }
     build_emit_table(em, mmax, W, P);
     for (int p = threadIdx.x; p < D; p += NT) {
         const typename Tr<S>::V4 e = qtab[(int64_t)mq * D + p];
@@ -584,7 +609,7 @@ __global__ void __launch_bounds__(kFusedThreads, (W <= 8 ? 3 : 1)) lb_fused_kern
                     sc[b] += pv.y;
                     const int rng = em[j * W + b];
                     if ((rng & 255) != (rng >> 8)) {
-                        const V lbv = vmax(se[b], sc[b]);
+                        const V lbv = lbpick(P, se[b], sc[b]);
                         for (int i = rng & 255; i < (rng >> 8); i++) trow[i * stride + b] = lbv;
                     }
                 }
@@ -617,7 +642,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
                                           V *lb, int32_t *tauc, int mq) {
     const int d = P.len[i];
     const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
-    const int64_t tend = min(m.t_hi, m.n - d + 1);
+    const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
     V *out = lb + m.seg_off + (int64_t)i * m.n;
     const int64_t t0 = s0 - d;
     const bool all = t0 >= tmin && t0 + W <= tend;
@@ -722,7 +747,10 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
     V *ls = us + kDiagCols * DS;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) return;
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, kDiagThreads / 32, 0, P.n_len, tauc);
+        return;
+    }
     for (int p = threadIdx.x; p < QL; p += NT) {
         const int src = p - qshift;
         V q = (V)0, u = (V)0, l = (V)0;
@@ -832,7 +860,7 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                 if (j == qi - 1) {
                     V v[W];
 #pragma unroll
-                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? saved[b] : (V)0) : vmax(se[b], sc[b]);
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? saved[b] : (V)0) : lbpick(P, se[b], sc[b]);
                     diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }
@@ -841,7 +869,7 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
         // IQ and q_i' - 2 for another uses the previous row's saved values)
         if (save_rows >> j & 1ull) {
 #pragma unroll
-            for (int b = 0; b < W; b++) saved[b] = vmax(se[b], sc[b]);
+            for (int b = 0; b < W; b++) saved[b] = lbpick(P, se[b], sc[b]);
         }
     }
     if (P.k < 0) {  // timing experiment: keep the sums alive
@@ -903,7 +931,10 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
     const int mmax = D / W;
     const int mq = blockIdx.y;
     const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) return;
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, kScanThreads / 32, 0, P.n_len, tauc);
+        return;
+    }
     const int64_t r = (int64_t)blockIdx.x * kScanThreads - 1 + threadIdx.x;
     const int64_t s0 = (r + 1) * W;  // e of slot b = 0
     const bool valid = r >= 0 && r < m.n_dw;
@@ -957,14 +988,160 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
                 if (j == qi - 1) {
                     V v[W];
 #pragma unroll
-                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : vmax(se[b], sc[b]);
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
                     diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }
         }
         if (save_rows >> j & 1ull) {
 #pragma unroll
-            for (int b = 0; b < W; b++) s_saved[b][x] = vmax(se[b], sc[b]);
+            for (int b = 0; b < W; b++) s_saved[b][x] = lbpick(P, se[b], sc[b]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// SMiLer-Dir (ablation, NEXT-4): LB_en(IQ_i, C_t) = max(LB_EQ, LB_EC) over all
+// d_i points of the candidate (Thm 4.1; LB_Keogh Eq. 26 with the
+// series envelope and the MQ envelope, R4/R20), computed straight from the
+// series with no window level -- the "SMiLer-Dir" of Fig. 8 (P:1916-1919,
+// P:2094-2097).  Candidates are addressed by their END e = t + d_i: with
+// u = 0, 1, ... counted back from the end, the term pair u of every item query
+// ending at e is the same (series point e-1-u against MQ position D-1-u, since
+// every IQ is a suffix of the MQ), so running sums over u give the
+// bound of IQ i as soon as u reaches d_i.  One launch emits the IQs
+// [li0, li1): li1 = li0 + 1 is the paper's per-item-query scan
+// (SMILER_LB_DIRECT), [0, n_len) shares one pass (SMILER_LB_DIRECT_SHARED).
+// Thread x owns the kDirP consecutive ends E0 + x kDirP + p; the CTA stages
+// the series (and envelope) range it touches in shared memory with a 4-float
+// skew every 32 floats (conflict-free 16-byte loads at an 8-float lane
+// stride) and the reversed MQ arrays rq[u] = MQ[D-1-u].  Per chunk of 8 u:
+// 16 series values per array and 8 query values per array in registers,
+// 8 x 8 term pairs.  Emission reuses diag_emit (slots e = s0 + p, t = e - d_i
+// contiguous; tau units are warps).
+// ---------------------------------------------------------------------------
+constexpr int kDirThreads = 128;
+constexpr int kDirP = 8;
+constexpr int kDirEnds = kDirThreads * kDirP;  // ends per CTA
+
+__host__ __device__ constexpr int dir_skew(int i) { return i + (i >> 5) * 4; }
+// shared memory (elements of V) of lb_direct_kernel for a pass of length dmax
+__host__ __device__ inline int dir_tile_len(int dmax) { return kDirEnds + ((dmax + 7) & ~7) + 8; }
+__host__ __device__ inline size_t dir_smem_elems(int dmax, int D) {
+    return (size_t)3 * dir_skew(dir_tile_len(dmax)) + 3 * (size_t)(((D + 7) & ~7) + 8);
+}
+
+template <typename V, bool CHECK>
+__device__ __forceinline__ void dir_chunk(const V (&c)[16], const V (&uc)[16], const V (&lc)[16], const V (&q)[8],
+                                          const V (&uq)[8], const V (&lq)[8], int ua, int ub, V (&se)[kDirP],
+                                          V (&sc)[kDirP]) {
+#pragma unroll
+    for (int uu = 0; uu < 8; uu++) {
+        if (!CHECK || (uu >= ua && uu < ub)) {
+#pragma unroll
+            for (int p = 0; p < kDirP; p++) {
+                const int x = p - uu + 7;  // series point e - 1 - u in the 16-value window
+                lb_term(c[x], uq[uu], lq[uu], se[p]);
+                lb_term(q[uu], uc[x], lc[x], sc[p]);
+            }
+        }
+    }
+}
+
+template <typename S>
+__global__ void __launch_bounds__(kDirThreads) lb_direct_kernel(const S *series, const S *UC, const S *LC,
+                                                                const MQMeta *meta, const typename Tr<S>::V4 *qtab,
+                                                                const QParams P, int li0, int li1,
+                                                                typename Tr<S>::V *lb, int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    using V4 = typename Tr<S>::V4;
+    extern __shared__ __align__(16) unsigned char dir_smem[];
+    const int D = P.D;
+    const int dmax = P.len[li1 - 1];
+    const int TL = dir_tile_len(dmax);
+    const int DP = TL - kDirEnds;  // tile position of series point E0 is DP
+    const int TS = dir_skew(TL);
+    const int QL = ((D + 7) & ~7) + 8;
+    V *tc = reinterpret_cast<V *>(dir_smem);
+    V *tu = tc + TS;
+    V *tl = tu + TS;
+    V *rq = tl + TS;
+    V *ru = rq + QL;
+    V *rl = ru + QL;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    const int64_t E0 = (int64_t)blockIdx.x * kDirEnds;
+    if ((int)blockIdx.x >= m.nblk) {  // nblk = n / kDirEnds + 1 (ends 0..n)
+        tau_clear(P, mq, kDirThreads / 32, li0, li1, tauc);
+        return;
+    }
+    for (int u = threadIdx.x; u < QL; u += kDirThreads) {
+        V a = (V)0, b = (V)0, c = (V)0;
+        if (u < D) {
+            const V4 e = qtab[(int64_t)mq * D + (D - 1 - u)];
+            a = e.x, b = e.y, c = e.z;
+        }
+        rq[u] = a, ru[u] = b, rl[u] = c;
+    }
+    const int64_t T0 = E0 - DP;  // series point of tile position 0
+#pragma unroll 8
+    for (int i = threadIdx.x; i < TL; i += kDirThreads) {
+        const int64_t s = T0 + i;
+        V a = (V)0, b = (V)0, c = (V)0;
+        if (s >= 0 && s < m.n) {
+            const int64_t g = m.series_off + s;
+            a = (V)series[g], b = (V)UC[g], c = (V)LC[g];
+        }
+        const int k = dir_skew(i);
+        tc[k] = a, tu[k] = b, tl[k] = c;
+    }
+    __syncthreads();
+    const int x = threadIdx.x;
+    V se[kDirP], sc[kDirP];
+#pragma unroll
+    for (int p = 0; p < kDirP; p++) se[p] = sc[p] = (V)0;
+    const int64_t s0 = E0 + (int64_t)x * kDirP;  // end e of slot p = 0
+    int nexti = li0;
+    for (int u0 = 0; u0 < dmax; u0 += 8) {
+        // window: tile positions ib .. ib+15 hold series points e0 - 1 - u for the chunk
+        const int ib = DP + x * kDirP - u0 - 8;
+        V c[16], uc[16], lc[16], q[8], uq[8], lq[8];
+#pragma unroll
+        for (int g = 0; g < 16; g += 4) {
+            const int k = dir_skew(ib + g);
+            const V4 a = *reinterpret_cast<const V4 *>(tc + k);
+            const V4 b = *reinterpret_cast<const V4 *>(tu + k);
+            const V4 d = *reinterpret_cast<const V4 *>(tl + k);
+            c[g] = a.x, c[g + 1] = a.y, c[g + 2] = a.z, c[g + 3] = a.w;
+            uc[g] = b.x, uc[g + 1] = b.y, uc[g + 2] = b.z, uc[g + 3] = b.w;
+            lc[g] = d.x, lc[g + 1] = d.y, lc[g + 2] = d.z, lc[g + 3] = d.w;
+        }
+#pragma unroll
+        for (int g = 0; g < 8; g += 4) {
+            const V4 a = *reinterpret_cast<const V4 *>(rq + u0 + g);
+            const V4 b = *reinterpret_cast<const V4 *>(ru + u0 + g);
+            const V4 d = *reinterpret_cast<const V4 *>(rl + u0 + g);
+            q[g] = a.x, q[g + 1] = a.y, q[g + 2] = a.z, q[g + 3] = a.w;
+            uq[g] = b.x, uq[g + 1] = b.y, uq[g + 2] = b.z, uq[g + 3] = b.w;
+            lq[g] = d.x, lq[g + 1] = d.y, lq[g + 2] = d.z, lq[g + 3] = d.w;
+        }
+        // split the chunk at item-query lengths (emit when u reaches d_i)
+        int ua = 0;
+        while (ua < 8) {
+            const int dn = nexti < li1 ? P.len[nexti] : 0x7fffffff;
+            const int ub = (int)min((int64_t)8, (int64_t)dn - u0);
+            if (ua == 0 && ub == 8)
+                dir_chunk<V, false>(c, uc, lc, q, uq, lq, 0, 8, se, sc);
+            else
+                dir_chunk<V, true>(c, uc, lc, q, uq, lq, ua, ub, se, sc);
+            if (u0 + ub == dn) {
+                V v[kDirP];
+#pragma unroll
+                for (int p = 0; p < kDirP; p++) v[p] = lbpick(P, se[p], sc[p]);
+                diag_emit<V, kDirP>(v, nexti, s0, m, P, lb, tauc, mq);
+                nexti++;
+            }
+            ua = ub;
         }
     }
 }

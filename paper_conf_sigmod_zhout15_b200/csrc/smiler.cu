@@ -126,7 +126,7 @@ struct smiler_index {
     int num_sms = 148;
     // workspace
     DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, tauk, taukey, thr, scount, fcount,
-        taskoff, out_ids, out_d, tmp, tmp2;
+        taskoff, out_ids, out_d, tmp, tmp2, pred;
     std::vector<cudaEvent_t> events;
     size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
     // pinned staging ring for per-chunk metadata (async H2D without host sync)
@@ -302,7 +302,7 @@ static void destroy(smiler_index *idx) {
     DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
                       &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->tauk,
                       &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
-                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2};
+                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
     for (int i = 0; i < kMaxLen; i++) {
@@ -447,6 +447,8 @@ struct Plan {
     bool scan_reg;   // a4 by group_scan_reg_kernel (static w, mmax <= 64)
     bool fused;      // a3+a4 fused kernel
     int fused_kind;  // 0 = diagonal form (lb_diag_kernel), 1 = row form (lb_fused_kernel)
+    int lb_kind;     // smiler_knn_opts.lb_kind (SMILER_LB_*)
+    bool direct;     // SMILER_LB_DIRECT*: lb_direct_kernel, no window level
     int RTf;         // fused: tile DWs per CTA
     size_t smem_gs, smem_fz;
 };
@@ -596,6 +598,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     Plan pl;
     TRY(validate_query(idx, lens_h.data(), n_len, lb_only ? 1 : k, pl));
     if (o.two_level || (lb_only && post_out) || sctx) pl.fused = false;
+    if (o.lb_kind < SMILER_LB_INDEX || o.lb_kind > SMILER_LB_DIRECT_SHARED)
+        return fail(SMILER_EINVAL, "lb_kind %d is not a SMILER_LB_* value", o.lb_kind);
+    pl.lb_kind = o.lb_kind;
+    if (o.horizon < 0) return fail(SMILER_EINVAL, "horizon must be >= 0");
+    pl.direct = o.lb_kind >= SMILER_LB_DIRECT;
+    if (pl.direct && (sctx || (lb_only && post_out)))
+        return fail(SMILER_EINVAL, "the direct lower bounds have no window level (posting lists / streams)");
+    if (pl.direct) pl.fused = false;
     if (pl.fused && o.reserved[0] == 1 && pl.fused_kind == 0) {  // row-form fused kernel (comparison)
         const int mmax = pl.D / pl.w, halo = mmax - 1;
         const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
@@ -646,7 +656,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     auto mq_bytes = [&](int j) -> size_t {
         const SensorInfo &si = idx->sensors[qsens[j]];
         const size_t ndw = (size_t)(si.n / w);
-        return ((pl.fused || sctx) ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) + 4096;
+        return ((pl.fused || pl.direct || sctx) ? 0 : (size_t)n_sw * ndw * 8) + (size_t)nl * si.n * (4 + 4 + 8) +
+               4096;
     };
     size_t budget = idx->budget;  // halved on ENOMEM (e.g. a resident stream ring)
     int chunk_max = o.mq_chunk > 0 ? o.mq_chunk : 65535;
@@ -692,18 +703,21 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             m.origin = si.origin;
             m.t_lo = si.t_lo;
             m.t_hi = si.t_hi;
+            // horizon: t + d + h <= N of the full series; a shard's slice ends at
+            // slice_begin + n <= n_global, so locally t + d + hz <= n
+            m.hz = std::max<int64_t>(0, (int64_t)o.horizon - (si.n_global - (si.slice_begin + si.n)));
             m.n_dw = si.n / w;
             m.post_off = sctx ? sctx->ring_off[c0 + j] : post_tot;
             m.seg_off = seg_tot;
-            m.nblk = (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
+            m.nblk = pl.direct ? (int)(m.n / kDirEnds + 1) : (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
             m.sensor = qsens[c0 + j];
-            post_tot += 2 * (int64_t)n_sw * m.n_dw;  // P_EQ and P_EC planes
+            if (!pl.direct) post_tot += 2 * (int64_t)n_sw * m.n_dw;  // P_EQ and P_EC planes
             seg_tot += (int64_t)nl * si.n;
             nblk_min = std::min(nblk_min, m.nblk);
             nblk_max = std::max(nblk_max, m.nblk);
             for (int i = 0; i < nl; i++) {
                 const int64_t tb = std::max<int64_t>(0, si.t_lo);
-                const int64_t te = std::min<int64_t>(si.t_hi, si.n - pl.len[i] + 1);
+                const int64_t te = std::min<int64_t>(si.t_hi, si.n - meta[j].hz - pl.len[i] + 1);
                 const int64_t nc = te > tb ? te - tb : 0;
                 cand_total += nc;
                 bf_cells += (double)nc * (double)dtw_cells(pl.len[i], pl.rho[i]);
@@ -711,8 +725,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         }
         // tau-set units: CTAs (block epilogue) or warps (diagonal kernel's warp epilogue)
         // tau units: warps of the diagonal kernel / of group_scan (w in {4,8,16,32}), else CTAs
-        const int units_per_blk = (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32
-                                  : (!pl.fused && pl.scan_reg) ? kScanThreads / 32 : 1;
+        const int units_per_blk = pl.direct                          ? kDirThreads / 32
+                                  : (pl.fused && pl.fused_kind == 0) ? kDiagThreads / 32
+                                  : (!pl.fused && pl.scan_reg)       ? kScanThreads / 32
+                                                                     : 1;
         int E = 0;
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         if (!lb_only && !o.no_prune) {
@@ -742,6 +758,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         if (o.reserved[1] == 2) P.E = 0;   // timing experiment: no tau set (no pruning)
         P.LT = LT;
         P.ring_cursor = sctx ? sctx->cursor : 0;
+        P.lbsel = pl.lb_kind == SMILER_LB_INDEX_EQ ? 1 : pl.lb_kind == SMILER_LB_INDEX_EC ? 2 : 0;
         P.n_mq = B;
         for (int i = 0; i < nl; i++) {
             P.len[i] = pl.len[i];
@@ -802,7 +819,25 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         CHECK_LAUNCH();
         launches++;
         TRY(tm.mark(1));
-        if (pl.fused) {
+        if (pl.direct) {
+            // ---- SMiLer-Dir (ablation): LB_en per candidate, no window level --
+            dim3 grid((unsigned)nblk_max, (unsigned)B);
+            auto go = [&](int li0, int li1) -> int {
+                const size_t smem = dir_smem_elems(pl.len[li1 - 1], D) * sizeof(V);
+                set_smem((const void *)lb_direct_kernel<S>, smem);
+                lb_direct_kernel<S><<<grid, kDirThreads, smem, idx->stream>>>(
+                    (const S *)idx->d_series, (const S *)dUC, (const S *)dLC, d_meta, idx->qtab.as<V4>(), P, li0,
+                    li1, idx->lb.as<V>(), idx->tauc.as<int32_t>());
+                CHECK_LAUNCH();
+                launches++;
+                return SMILER_OK;
+            };
+            if (pl.lb_kind == SMILER_LB_DIRECT)
+                for (int i = 0; i < nl; i++) TRY(go(i, i + 1));  // one scan per item query
+            else
+                TRY(go(0, nl));
+            TRY(tm.mark(2));
+        } else if (pl.fused) {
             // ---- a3 + a4 fused ------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
             const int nthr = pl.fused_kind == 0 ? kDiagThreads : kFusedThreads;
@@ -1226,6 +1261,105 @@ extern "C" int smiler_lower_bounds(smiler_index *idx, const void *queries, const
                                  nullptr, &o, true, postings, lbw);
     return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, 1, nullptr, nullptr, nullptr,
                            &o, true, postings, lbw);
+}
+
+extern "C" int smiler_lower_bounds_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                      int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t lb_kind,
+                                      void *lb) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!lb) return fail(SMILER_EINVAL, "lb is NULL");
+    smiler_knn_opts o;
+    memset(&o, 0, sizeof(o));
+    o.lb_kind = lb_kind;
+    if (idx->dtype == SMILER_I16)
+        return knn_impl<int16_t>(idx, queries, query_sensor, n_mq, lengths, n_len, 1, nullptr, nullptr,
+                                 nullptr, &o, true, nullptr, lb);
+    return knn_impl<float>(idx, queries, query_sensor, n_mq, lengths, n_len, 1, nullptr, nullptr, nullptr, &o,
+                           true, nullptr, lb);
+}
+
+// ---------------------------------------------------------------------------
+// smiler_predict (NEXT-3): AR and GP predictors on the kNN data (Sec. 5.2)
+// ---------------------------------------------------------------------------
+namespace smiler {
+template <typename S>
+int launch_predict(const void *series, const int64_t *soff_n, int n_sensors, const int32_t *qsens,
+                   const void *queries, int D, const int32_t *lens, int n_len, const int64_t *ids, int k,
+                   const int32_t *ekv, int n_k, int kmax, int h, const double *theta, int n_pred, double *ar_mean,
+                   double *ar_var, double *gp_mean, double *gp_var, cudaStream_t st);
+}
+
+extern "C" int smiler_predict(smiler_index *idx, const void *queries, const int32_t *query_sensor, int32_t n_mq,
+                              const int32_t *lengths, int32_t n_len, const int64_t *ids, int32_t k,
+                              const int32_t *ekv, int32_t n_k, int32_t horizon, const double *theta,
+                              double *ar_mean, double *ar_var, double *gp_mean, double *gp_var) {
+    if (!idx) return fail(SMILER_EINVAL, "index is NULL");
+    if (!queries || !lengths || !ids || !ekv || !theta || !ar_mean || !ar_var || !gp_mean || !gp_var)
+        return fail(SMILER_EINVAL, "NULL argument");
+    if (idx->shard) return fail(SMILER_EINVAL, "smiler_predict needs a whole-series index (not a shard)");
+    if (n_mq < 1 || n_len < 1 || n_len > kMaxLen || k < 1 || n_k < 1 || n_k > 64 || horizon < 0)
+        return fail(SMILER_EINVAL, "need n_mq >= 1, 1 <= n_len <= %d, k >= 1, 1 <= n_k <= 64, horizon >= 0",
+                    kMaxLen);
+    TRY(set_device(idx));
+    std::vector<int32_t> lens(n_len), ek(n_k), qs(n_mq, 0);
+    CU(cudaMemcpy(lens.data(), lengths, 4 * (size_t)n_len, cudaMemcpyDefault));
+    CU(cudaMemcpy(ek.data(), ekv, 4 * (size_t)n_k, cudaMemcpyDefault));
+    if (query_sensor) CU(cudaMemcpy(qs.data(), query_sensor, 4 * (size_t)n_mq, cudaMemcpyDefault));
+    for (int i = 0; i < n_len; i++)
+        if (lens[i] < 1 || (i && lens[i] <= lens[i - 1])) return fail(SMILER_EINVAL, "lengths must increase");
+    const int D = lens[n_len - 1];
+    if (D > kMaxD) return fail(SMILER_EINVAL, "D = %d exceeds %d", D, kMaxD);
+    for (int j = 0; j < n_k; j++)
+        if (ek[j] < 1 || ek[j] > k || ek[j] > kMaxPredK || (j && ek[j] <= ek[j - 1]))
+            return fail(SMILER_EINVAL, "ekv must increase within [1, min(k, %d)]", kMaxPredK);
+    for (int m = 0; m < n_mq; m++)
+        if (qs[m] < 0 || qs[m] >= (int)idx->sensors.size())
+            return fail(SMILER_EINVAL, "query_sensor[%d] out of range", m);
+    const int kmax = ek[n_k - 1];
+    const int64_t n_pred = (int64_t)n_mq * n_len * n_k;
+    if (n_pred > INT32_MAX) return fail(SMILER_EINVAL, "too many predictors");
+    const size_t es = esize(idx->dtype);
+    // device workspace: sensors | qsens | lens | ekv | queries | ids | theta | 4 outputs
+    const size_t ns = idx->sensors.size();
+    size_t off = 0;
+    auto take = [&](size_t b) { size_t o = off; off += (b + 255) & ~(size_t)255; return o; };
+    const size_t o_sens = take(16 * ns), o_qs = take(4 * (size_t)n_mq), o_len = take(4 * (size_t)n_len),
+                 o_ek = take(4 * (size_t)n_k), o_q = take(es * (size_t)n_mq * D),
+                 o_ids = take(8 * (size_t)n_mq * n_len * k), o_th = take(24 * (size_t)n_pred),
+                 o_out = take(32 * (size_t)n_pred);
+    TRY(idx->pred.ensure(off));
+    char *b = idx->pred.as<char>();
+    std::vector<int64_t> sn(2 * ns);
+    for (size_t x = 0; x < ns; x++) {
+        sn[2 * x] = idx->sensors[x].off;
+        sn[2 * x + 1] = idx->sensors[x].n;
+    }
+    cudaStream_t st = idx->stream;
+    CU(cudaMemcpyAsync(b + o_sens, sn.data(), 16 * ns, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(b + o_qs, qs.data(), 4 * (size_t)n_mq, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(b + o_len, lens.data(), 4 * (size_t)n_len, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(b + o_ek, ek.data(), 4 * (size_t)n_k, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(b + o_q, queries, es * (size_t)n_mq * D, cudaMemcpyDefault, st));
+    CU(cudaMemcpyAsync(b + o_ids, ids, 8 * (size_t)n_mq * n_len * k, cudaMemcpyDefault, st));
+    CU(cudaMemcpyAsync(b + o_th, theta, 24 * (size_t)n_pred, cudaMemcpyDefault, st));
+    double *outs = reinterpret_cast<double *>(b + o_out);
+    int rc = idx->dtype == SMILER_I16
+                 ? smiler::launch_predict<int16_t>(idx->d_series, (const int64_t *)(b + o_sens), (int)ns,
+                                           (const int32_t *)(b + o_qs), b + o_q, D, (const int32_t *)(b + o_len),
+                                           n_len, (const int64_t *)(b + o_ids), k, (const int32_t *)(b + o_ek), n_k,
+                                           kmax, horizon, (const double *)(b + o_th), (int)n_pred, outs,
+                                           outs + n_pred, outs + 2 * n_pred, outs + 3 * n_pred, st)
+                 : smiler::launch_predict<float>(idx->d_series, (const int64_t *)(b + o_sens), (int)ns,
+                                         (const int32_t *)(b + o_qs), b + o_q, D, (const int32_t *)(b + o_len),
+                                         n_len, (const int64_t *)(b + o_ids), k, (const int32_t *)(b + o_ek), n_k,
+                                         kmax, horizon, (const double *)(b + o_th), (int)n_pred, outs,
+                                         outs + n_pred, outs + 2 * n_pred, outs + 3 * n_pred, st);
+    if (rc != cudaSuccess) return fail(SMILER_ECUDA, "predict_kernel: %s", cudaGetErrorString((cudaError_t)rc));
+    double *dst[4] = {ar_mean, ar_var, gp_mean, gp_var};
+    for (int x = 0; x < 4; x++)
+        CU(cudaMemcpyAsync(dst[x], outs + x * n_pred, 8 * (size_t)n_pred, cudaMemcpyDefault, st));
+    CU(cudaStreamSynchronize(st));
+    return SMILER_OK;
 }
 
 extern "C" int smiler_index_envelope(smiler_index *idx, int32_t sensor, int32_t rho, void *U, void *L) {

@@ -46,7 +46,12 @@ class KnnStats(ctypes.Structure):
 class KnnOpts(ctypes.Structure):
     _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
                 ("mq_chunk", ctypes.c_int32), ("two_level", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 4)]
+                ("lb_kind", ctypes.c_int32), ("horizon", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+
+
+# smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
+SMILER_LB_INDEX, SMILER_LB_INDEX_EQ, SMILER_LB_INDEX_EC, SMILER_LB_DIRECT, SMILER_LB_DIRECT_SHARED = 0, 1, 2, 3, 4
+LB_KINDS = {"index": 0, "index_eq": 1, "index_ec": 2, "direct": 3, "direct_shared": 4}
 
 
 _lib = None
@@ -74,6 +79,8 @@ def lib():
         L.smiler_merge_topk.argtypes = [P, P, i32, i32, i32, i32, P, P, i32, P]
         L.smiler_index_envelope.argtypes = [P, i32, i32, P, P]
         L.smiler_lower_bounds.argtypes = [P, P, P, i32, P, i32, P, P]
+        L.smiler_lower_bounds_ex.argtypes = [P, P, P, i32, P, i32, i32, P]
+        L.smiler_predict.argtypes = [P, P, P, i32, P, i32, P, i32, P, i32, i32, P, P, P, P, P]
         L.smiler_dtw.argtypes = [P, i32, P, i32, i32, P, i64, P]
         L.smiler_free.argtypes = [P]
         L.smiler_free.restype = None
@@ -81,7 +88,8 @@ def lib():
         L.smiler_abi_version.restype = i32
         for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex", "smiler_knn_step",
                   "smiler_stream_create", "smiler_stream_step",
-                  "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_dtw"):
+                  "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_lower_bounds_ex",
+                  "smiler_dtw", "smiler_predict"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -226,6 +234,28 @@ def smiler_lower_bounds(handle: int, queries, query_sensor, lengths, postings, l
                                      len(lens), _ptr(postings), _ptr(lbw)))
 
 
+def smiler_lower_bounds_ex(handle: int, queries, query_sensor, lengths, lb_kind: int, lb) -> None:
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    qs = None if query_sensor is None else np.ascontiguousarray(query_sensor, np.int32)
+    _check("smiler_lower_bounds_ex",
+           lib().smiler_lower_bounds_ex(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens),
+                                        len(lens), int(lb_kind), _ptr(lb)))
+
+
+def smiler_predict(handle: int, queries, query_sensor, lengths, ids, ekv, horizon: int, theta,
+                   ar_mean, ar_var, gp_mean, gp_var) -> None:
+    """AR (Eq. 12-13) and GP (Eq. 16-18) predictors of every (MQ, item query, k_j in ekv)
+    from the kNN ids (see include/smiler.h).  Host (numpy) or device (torch) buffers."""
+    lens = np.ascontiguousarray(lengths, dtype=np.int32)
+    ek = np.ascontiguousarray(ekv, dtype=np.int32)
+    qs = query_sensor if (query_sensor is None or hasattr(query_sensor, "data_ptr")) \
+        else np.ascontiguousarray(query_sensor, np.int32)
+    _check("smiler_predict",
+           lib().smiler_predict(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens), len(lens),
+                                _ptr(ids), int(ids.shape[-1]), _ptr(ek), len(ek), int(horizon), _ptr(theta),
+                                _ptr(ar_mean), _ptr(ar_var), _ptr(gp_mean), _ptr(gp_var)))
+
+
 def smiler_dtw(handle: int, sensor: int, q, rho: int, ts, dists) -> None:
     tsa = np.ascontiguousarray(ts, dtype=np.int64) if not hasattr(ts, "data_ptr") else ts
     _check("smiler_dtw", lib().smiler_dtw(handle, sensor, _ptr(q), int(q.shape[0]), rho, _ptr(tsa),
@@ -299,16 +329,28 @@ class Index:
         return cls(slice_, _handle=h)
 
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
-            no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False):
+            no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False,
+            lb_kind: int = 0, horizon: int = 0):
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
-        op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level))
+        op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level),
+                     lb_kind=int(lb_kind), horizon=int(horizon))
         smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()
         return ids, dists
+
+    def predict(self, queries, lengths: Sequence[int], ids, ekv: Sequence[int], horizon: int, theta,
+                query_sensor=None):
+        """(ar_mean, ar_var, gp_mean, gp_var), each [n_mq, n_len, len(ekv)] float64."""
+        shape = (queries.shape[0], len(lengths), len(ekv))
+        outs = [np.empty(shape, np.float64) for _ in range(4)]
+        smiler_predict(self.handle, np.ascontiguousarray(queries), query_sensor, lengths,
+                       np.ascontiguousarray(ids, dtype=np.int64), ekv, horizon,
+                       np.ascontiguousarray(theta, dtype=np.float64), *outs)
+        return tuple(outs)
 
     def knn_step(self, queries, lengths: Sequence[int], k: int, prev_ids, shift: int = 1, query_sensor=None,
                  stats: bool = False, timing: bool = False):
@@ -339,6 +381,15 @@ class Index:
         lbw = np.empty((n_mq, len(lengths), n), vt)
         smiler_lower_bounds(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, post, lbw)
         return post, lbw
+
+    def lower_bounds_kind(self, queries, lengths, n: int, lb_kind: int, query_sensor=None):
+        """The per-candidate bound smiler_knn_ex filters with under `lb_kind`:
+        [n_mq][n_len][n] (entries with t > n - d_i unspecified)."""
+        n_mq = queries.shape[0]
+        vt = np.int32 if self.dtype == SMILER_I16 else np.float32
+        lb = np.empty((n_mq, len(lengths), n), vt)
+        smiler_lower_bounds_ex(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, lb_kind, lb)
+        return lb
 
     def dtw(self, sensor: int, q, rho: int, ts):
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32

@@ -27,7 +27,8 @@ def test_header_declares_the_boundary():
     # the three calls of the north star plus merge and the per-step entry points
     for f in ("smiler_index_build", "smiler_knn", "smiler_free", "smiler_merge_topk",
               "smiler_index_build_shard", "smiler_knn_ex", "smiler_lower_bounds", "smiler_dtw",
-              "smiler_index_envelope", "smiler_last_error", "smiler_abi_version"):
+              "smiler_index_envelope", "smiler_last_error", "smiler_abi_version", "smiler_lower_bounds_ex",
+              "smiler_predict"):
         assert f in fns, f
 
 
@@ -39,10 +40,10 @@ def test_library_exports_every_declared_symbol(built):
 
 def test_abi_version_and_stats_layout(built):
     import paper_conf_sigmod_zhout15_b200 as pkg
-    assert pkg.smiler_abi_version() == 1
+    assert pkg.smiler_abi_version() == 2
     # struct sizes match the header (8 x 8-byte counters, 2 int32, 8 doubles)
     assert ctypes.sizeof(pkg.KnnStats) == 8 * 8 + 2 * 4 + 8 * 8
-    assert ctypes.sizeof(pkg.KnnOpts) == 8 * 4
+    assert ctypes.sizeof(pkg.KnnOpts) == 10 * 4
 
 
 def test_no_gpu_means_error_not_fallback(built):

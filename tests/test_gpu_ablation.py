@@ -1,0 +1,95 @@
+"""Parity of the lower-bound ablations with the oracle (-m gpu).
+
+Table 3 compares filtering by LB_EQ, LB_EC and LB_en;
+Fig. 8 compares LB_en through the window-level
+index ("SMiLer-Idx") with LB_en computed directly per item query
+("SMiLer-Dir").  smiler_knn_opts.lb_kind selects the bound:
+
+  index      LB_w = max(EQ sum, EC sum) over the full disjoint windows (Eq. 5)
+  index_eq   the EQ sum alone;  index_ec  the EC sum alone
+  direct     LB_en = max(LB_EQ, LB_EC) over all d_i points (Thm 4.1), per IQ
+  direct_shared  the same LB_en from one end-aligned pass for all IQs
+
+Each bound is compared value by value with the oracle's plain loops (bit-exact
+in i16, rtol 2e-5 in f32), and the kNN found with it must equal the oracle's
+brute force (every kind is a valid DTW lower bound, so filtering is exact).
+"""
+import numpy as np
+import pytest
+
+import synth
+
+from test_gpu_parity import check_workload
+
+pytestmark = pytest.mark.gpu
+
+KINDS = {"index": 0, "index_eq": 1, "index_ec": 2, "direct": 3, "direct_shared": 4}
+ORACLE_KEY = {"index": "w", "index_eq": "weq", "index_ec": "wec", "direct": "en", "direct_shared": "en"}
+
+
+@pytest.fixture(scope="module")
+def pkg():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sigmod_zhout15_b200 import build
+    build.build()
+    import paper_conf_sigmod_zhout15_b200 as p
+    return p
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("cfg,n,lengths,window,band", [
+    ("C2", 9001, [16, 32, 64, 128], 8, 0.1),
+    ("C3", 7013, [32, 64, 96], 16, 8.0),
+    ("C1", 2500, [5, 13, 40], 5, 2.0),        # lengths not multiples of the 8-point chunk
+    ("C1", 3001, [3, 1000], 8, 0.02),          # long query (rho 20), a length inside the first chunk
+])
+def test_lower_bound_kinds(pkg, orc, dtype, cfg, n, lengths, window, band):
+    wl = synth.make_workload(cfg, dtype, n=n, n_sensors=1, mq_per_sensor=3, lengths=lengths,
+                             window=window, band=band)
+    rhos = wl.rhos()
+    got = {}
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        for name, kind in KINDS.items():
+            got[name] = idx.lower_bounds_kind(wl.queries, wl.lengths, n, kind)
+    for j in range(wl.n_mq):
+        res, _ = orc.mq_lower_bounds(wl.series, wl.queries[j], wl.lengths, rhos, window)
+        for i, d in enumerate(wl.lengths):
+            for name in KINDS:
+                exp = res[i][ORACLE_KEY[name]]
+                g = got[name][j, i, :n - d + 1]
+                if dtype == "i16":
+                    np.testing.assert_array_equal(g.astype(np.int64), exp, err_msg=name)
+                else:
+                    np.testing.assert_allclose(g, exp, rtol=2e-5, atol=1e-6, err_msg=name)
+            # the chain of the paper: LB_EQ,w / LB_EC,w <= LB_w <= LB_en (Thm 4.3 proof)
+            w_ = got["index"][j, i, :n - d + 1].astype(np.float64)
+            en = got["direct"][j, i, :n - d + 1].astype(np.float64)
+            assert (got["index_eq"][j, i, :n - d + 1] <= got["index"][j, i, :n - d + 1]).all()
+            tol = 0.0 if dtype == "i16" else 1e-4        # f32 sums of up to d = 1000 terms (R16)
+            assert (w_ <= en * (1 + tol) + tol).all()
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("kind", ["index_eq", "index_ec", "direct", "direct_shared"])
+def test_knn_with_each_bound_equals_oracle(pkg, orc, dtype, kind):
+    wl = synth.make_workload("C5", dtype, n=12001, n_sensors=3, mq_per_sensor=2, consecutive=True)
+    check_workload(pkg, orc, wl, lb_kind=KINDS[kind])
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_direct_uneven_sensors_and_c3_shape(pkg, orc, dtype):
+    """Sensors of different lengths: CTAs past a short sensor's end must leave
+    no stale tau-set entries; C3's w=16 index vs the direct bound."""
+    wl = synth.make_workload("C3", dtype, n=9001, n_sensors=3, mq_per_sensor=2)
+    cut = [9001, 4000, 7500]
+    parts, offs = [], [0]
+    for s in range(3):
+        x = wl.sensor_slice(s)[:cut[s]]
+        parts.append(x)
+        offs.append(offs[-1] + len(x))
+    wl.series = np.concatenate(parts)
+    wl.offsets = np.asarray(offs, np.int64)
+    for kind in ("direct", "direct_shared", "index"):
+        check_workload(pkg, orc, wl, lb_kind=KINDS[kind])
