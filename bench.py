@@ -234,9 +234,9 @@ class Runner:
         self.ids = torch.empty((wl.n_mq, self.n_len, self.k), dtype=torch.int64, device=dev)
         self.dd = torch.empty((wl.n_mq, self.n_len, self.k), dtype=vt, device=dev)
         self.op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=int(args.two_level))
-        self.op.reserved[2] = args.tau_mult
+        self.op.tau_mult = args.tau_mult
         self.op_fast = pkg.KnnOpts(no_prune=0, timing=0, mq_chunk=0, two_level=int(args.two_level))
-        self.op_fast.reserved[2] = args.tau_mult
+        self.op_fast.tau_mult = args.tau_mult
         # C5 is a continuous prediction stream: every step is one tick of all
         # streams (each MQ advances one point); after the first tick the previous
         # tick's neighbours seed the thresholds (smiler_knn_step)

@@ -85,7 +85,19 @@ typedef struct smiler_knn_opts {
                          c_{t+d-1+h} exists are candidates, i.e. t <= N - d - h (the
                          kNN data (X_{k,d}, Y_h) of the predictors);
                          0 = every segment (Def. 4.1).  Shards: N is the full series. */
-    int32_t reserved[4];
+    int32_t exact_postings; /* smiler_stream_create_ex: 1 keeps the stream's window-level
+                         postings in the index arithmetic type; 0 (default) stores them for
+                         F32 indices with window 4/8/16/32 as fp16 rounded toward zero --
+                         never above the exact value, so every sum of them is still a
+                         lower bound of DTW (Thm 4.3) and the kNN is unchanged, while the
+                         ring and the bytes the group scan reads per step halve */
+    int32_t tau_mult; /* size of the tile tau set (reading R8), in multiples of k per item
+                         query: 0 = default (16 one-shot, 0 in continuous steps, whose
+                         thresholds come from the previous step's neighbours),
+                         > 0 = that many, < 0 = none.  With no tile set in a continuous
+                         step the thresholds exist before the scan, and the LB kernel
+                         filters as it goes (a4+a6 fused, no LB_w array) */
+    int32_t reserved[3];
 } smiler_knn_opts;
 
 /* smiler_knn_opts.lb_kind.  The default is the paper's method; the others are
@@ -222,9 +234,12 @@ SMILER_API int smiler_knn_step(smiler_index *idx, const void *queries, const int
  * smiler_stream_create  queries [n_streams][D] (initial master queries),
  *                       query_sensor/lengths/k as smiler_knn; runs the first
  *                       search and writes its ids/dists ([n][n_len][k], host
- *                       or device).  Memory: 8 (D - w + 1) floor(N/w) bytes of
- *                       posting lists per stream, resident; ENOMEM if absent.
+ *                       or device).  Memory: 2 planes x (D - w + 1) floor(N/w)
+ *                       posting entries per stream, resident (2 bytes each for
+ *                       F32 indices with w in {4,8,16,32}, else 4; see
+ *                       smiler_knn_opts.exact_postings); ENOMEM if absent.
  *                       The index must outlive the stream.
+ * smiler_stream_create_ex  the same with opts (exact_postings; others ignored).
  * smiler_stream_step    new_points [n_streams] (one new point per stream, index
  *                       dtype, host or device); writes the step's results.
  * smiler_stream_free    NULL-safe.
@@ -233,6 +248,10 @@ typedef struct smiler_stream smiler_stream;
 SMILER_API int smiler_stream_create(smiler_index *idx, const void *queries, const int32_t *query_sensor,
                                     int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
                                     int64_t *ids, void *dists, smiler_stream **out);
+SMILER_API int smiler_stream_create_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                       int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
+                                       int64_t *ids, void *dists, const smiler_knn_opts *opts,
+                                       smiler_stream **out);
 SMILER_API int smiler_stream_step(smiler_stream *st, const void *new_points, int64_t *ids, void *dists,
                                   smiler_knn_stats *stats, const smiler_knn_opts *opts);
 SMILER_API void smiler_stream_free(smiler_stream *st);

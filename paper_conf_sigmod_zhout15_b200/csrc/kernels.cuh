@@ -1,6 +1,7 @@
 // kernels.cuh -- steps a1-a6, a8, a9 of the Search Step.
 // Included once, by smiler.cu.  DTW (a5/a7) is in dtw.cu.
 #pragma once
+#include <cuda_fp16.h>
 #include <stdint.h>
 
 #include <type_traits>

@@ -41,6 +41,18 @@ __device__ __forceinline__ void tau_clear(const QParams &P, int mq, int units_pe
     }
 }
 
+// Posting storage.  PV = V keeps the window-level postings exact; PV = __half
+// (continuous f32 streams) stores each P_EQ / P_EC rounded toward zero, i.e.
+// never above its value (saturating at 65504): a sum of such entries is still
+// a lower bound of LB_w, hence of DTW (Thm 4.3), so filtering stays exact while
+// the ring -- the bytes the group scan streams every step -- halves.
+template <typename PV, typename V> __device__ __forceinline__ void post_st(PV *p, V v) { *p = v; }
+template <> __device__ __forceinline__ void post_st<__half, float>(__half *p, float v) {
+    *p = __float2half_rz(v);
+}
+template <typename V, typename PV> __device__ __forceinline__ V post_cv(PV x) { return x; }
+template <> __device__ __forceinline__ float post_cv<float, __half>(__half x) { return __half2float(x); }
+
 // emission table: em[j*w + b] = lo | hi << 8, the IQ range [lo, hi) with
 // m_i(b) == j + 1 (contiguous in i because d_i increases).
 __device__ __forceinline__ void build_emit_table(uint16_t *em, int mmax, int w, const QParams &P) {
@@ -242,11 +254,11 @@ __device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], 
 // {q, U(Q), L(Q)} loaded once into registers (no shared-memory load per term).
 // 8 ALU ops per (b, r, j) term pair.  Output post[mq][b][r] = {P_EQ, P_EC}.
 // ---------------------------------------------------------------------------
-template <typename S, int W>
+template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
                                                        const MQMeta *meta,
                                                        const typename Tr<S>::V4 *qtab, int D,
-                                                       int w_rt, typename Tr<S>::V *post) {
+                                                       int w_rt, PV *post) {
     using V = typename Tr<S>::V;
     extern __shared__ __align__(16) unsigned char wl_smem[];
     V *sqq = reinterpret_cast<V *>(wl_smem);
@@ -265,7 +277,7 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= m.n_dw) return;
     const int64_t ndw = m.n_dw;
-    V *oe = post + m.post_off + r;  // P_EQ plane; P_EC plane `plane` further
+    PV *oe = post + m.post_off + r;  // P_EQ plane; P_EC plane `plane` further
     if constexpr (W > 0) {
         constexpr int BC = W < 8 ? W : 8;
         const int n_sw = D - W + 1;
@@ -280,19 +292,19 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
         }
         int b0 = 0;
         for (; b0 + BC <= n_sw; b0 += BC) {
-            V *o = oe + (int64_t)b0 * ndw;
+            PV *o = oe + (int64_t)b0 * ndw;
             posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
                                            [&](int bb, V eq, V ec) {
-                                               o[bb * ndw] = eq;
-                                               o[bb * ndw + plane] = ec;
+                                               post_st(o + bb * ndw, eq);
+                                               post_st(o + bb * ndw + plane, ec);
                                            });
         }
         if (b0 < n_sw) {
-            V *o = oe + (int64_t)b0 * ndw;
+            PV *o = oe + (int64_t)b0 * ndw;
             posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
                                           [&](int bb, V eq, V ec) {
-                                              o[bb * ndw] = eq;
-                                              o[bb * ndw + plane] = ec;
+                                              post_st(o + bb * ndw, eq);
+                                              post_st(o + bb * ndw + plane, ec);
                                           });
         }
     } else {
@@ -307,8 +319,8 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
                 lb_term((V)series[base + j], squ[p0 + j], sql[p0 + j], eq);
                 lb_term(sqq[p0 + j], (V)UC[base + j], (V)LC[base + j], ec);
             }
-            oe[(int64_t)b * ndw] = eq;
-            oe[(int64_t)b * ndw + plane] = ec;
+            post_st(oe + (int64_t)b * ndw, eq);
+            post_st(oe + (int64_t)b * ndw + plane, ec);
         }
     }
 }
@@ -321,11 +333,11 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
 // the EC terms are not even computed and the EQ plane takes full 4-byte
 // coalesced rows.
 // ---------------------------------------------------------------------------
-template <typename S, int W>
+template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, const S *UC, const S *LC,
                                                            const MQMeta *meta,
                                                            const typename Tr<S>::V4 *qtab, int D, int nrows,
-                                                           int cursor, typename Tr<S>::V *post) {
+                                                           int cursor, PV *post) {
     using V = typename Tr<S>::V;
     constexpr int BC = W < 8 ? W : 8;
     extern __shared__ __align__(16) unsigned char wi_smem[];
@@ -347,7 +359,7 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
     const int64_t ndw = m.n_dw;
     const int n_ring = D - W + 1;
     const int n_sw = min(n_ring, nrows);
-    V *oe = post + m.post_off + r;
+    PV *oe = post + m.post_off + r;
     const int64_t base = m.series_off + r * W;
     V c[W], U[W], L[W];
 #pragma unroll
@@ -363,18 +375,18 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
     };
     // SW_0: both lists
     posting_chunk<V, W, 1, false>(c, U, L, sqq, squ, sql, D - W, 1, [&](int, V eq, V ec) {
-        V *o = row_ptr(0);
-        o[0] = eq;
-        o[(int64_t)n_ring * ndw] = ec;
+        PV *o = row_ptr(0);
+        post_st(o, eq);
+        post_st(o + (int64_t)n_ring * ndw, ec);
     });
     int b0 = 1;
     for (; b0 + BC <= n_sw; b0 += BC)
         posting_chunk<V, W, BC, false, true>(
-            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC, [&](int bb, V eq, V) { *row_ptr(b0 + bb) = eq; });
+            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC, [&](int bb, V eq, V) { post_st(row_ptr(b0 + bb), eq); });
     if (b0 < n_sw)
         posting_chunk<V, W, BC, true, true>(
             c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-            [&](int bb, V eq, V) { *row_ptr(b0 + bb) = eq; });
+            [&](int bb, V eq, V) { post_st(row_ptr(b0 + bb), eq); });
 }
 
 // ---------------------------------------------------------------------------
@@ -645,6 +657,39 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
     V *out = lb + m.seg_off + (int64_t)i * m.n;
     const int64_t t0 = s0 - d;
+    if (P.fuse) {  // a6 here: keep LB <= thr (ties survive), warp-aggregated append
+        const int seg = mq * P.n_len + i;
+        const uint32_t th = P.thr[seg];
+        uint32_t keep = 0;
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            const int64_t t = t0 + b;
+            bool k_;
+            if constexpr (std::is_same<V, float>::value)
+                k_ = v[b] <= __uint_as_float(th);
+            else
+                k_ = v[b] <= (int32_t)th;
+            keep |= (uint32_t)(k_ && t >= tmin && t < tend) << b;
+        }
+        const int lane = threadIdx.x & 31;
+        const int cnt = __popc(keep);
+        int x = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        const int total = __shfl_sync(0xffffffffu, x, 31);
+        int base = 0;
+        if (lane == 31 && total) base = atomicAdd(&P.scount[seg], total);
+        base = __shfl_sync(0xffffffffu, base, 31);
+        int o = base + x - cnt;
+        int32_t *dst = P.surv + m.seg_off + (int64_t)i * m.n;
+#pragma unroll
+        for (int b = 0; b < W; b++)
+            if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
+        return;
+    }
     const bool all = t0 >= tmin && t0 + W <= tend;
     if (all && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
 #pragma unroll
@@ -900,8 +945,8 @@ constexpr int kScanThreads = 256;
 #define SMILER_GS_MINB(W) ((W) <= 8 ? 4 : (W) <= 16 ? 2 : 1)
 #endif
 
-template <typename V, int W, bool CHECK>
-__device__ __forceinline__ void gs_load_row(V (&pe)[W], V (&pc)[W], const V *pp, uint32_t off, int bw,
+template <int W, bool CHECK, typename PV>
+__device__ __forceinline__ void gs_load_row(PV (&pe)[W], PV (&pc)[W], const PV *pp, uint32_t off, int bw,
                                             uint32_t ndw, uint32_t wrap, int nrow, bool ok) {
 #pragma unroll
     for (int b = 0; b < W; b++) {
@@ -909,7 +954,7 @@ __device__ __forceinline__ void gs_load_row(V (&pe)[W], V (&pc)[W], const V *pp,
         // the P_EC plane sits `wrap` (= n_sw * n_dw) elements after P_EQ
         const uint32_t o = off + (uint32_t)b * ndw - (b >= bw ? wrap : 0u);
         if constexpr (CHECK) {
-            pe[b] = pc[b] = (V)0;
+            pe[b] = pc[b] = (PV)0;
             if (ok && b < nrow) {
                 pe[b] = __ldg(pp + o);
                 pc[b] = __ldg(pp + o + wrap);
@@ -921,9 +966,9 @@ __device__ __forceinline__ void gs_load_row(V (&pe)[W], V (&pc)[W], const V *pp,
     }
 }
 
-template <typename S, int W>
+template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_reg_kernel(
-    const typename Tr<S>::V *post, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
+    const PV *post, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
     using V = typename Tr<S>::V;
     const int D = P.D;
     const int nl = P.n_len;
@@ -944,7 +989,7 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
     const uint32_t wrap = (uint32_t)n_sw * ndw;
     const int64_t rc = r < 0 ? 0 : (r < m.n_dw ? r : m.n_dw - 1);
     // offsets count from pp - mmax so they stay non-negative across the ring wrap
-    const V *pp = post + m.post_off + rc - mmax;
+    const PV *pp = post + m.post_off + rc - mmax;
     // values saved after row q_i - 2 live in shared memory ([b][thread]: no
     // bank conflicts), keeping the registers for sums and loads in flight
     __shared__ V s_saved[W][kScanThreads];
@@ -966,22 +1011,34 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
     }
     // ring row of SW_{j w} (Remark 1): rr = (j w + cursor) mod n_sw,
     // advanced by w per row (mmax >= 2 implies n_sw > w)
+    // one row of look-ahead: row j + 1's loads are in flight while row j is summed
+    // (the fp16 ring moves half the bytes per load, so it needs the extra depth)
     int rr = P.ring_cursor;
-    for (int j = 0; j < mmax; j++) {
-        V pe[W], pc[W];
-        const uint32_t off = (uint32_t)rr * ndw + (uint32_t)(mmax - j);
-        const int nrow = n_sw - j * W;
+    PV ne[W], nc[W];
+    auto load = [&](int jj, int r_) {
+        const uint32_t off = (uint32_t)r_ * ndw + (uint32_t)(mmax - jj);
+        const int nrow = n_sw - jj * W;
         if (first || nrow < W)
-            gs_load_row<V, W, true>(pe, pc, pp, off, n_sw - rr, ndw, wrap, nrow, j < jall);
+            gs_load_row<W, true, PV>(ne, nc, pp, off, n_sw - r_, ndw, wrap, nrow, jj < jall);
         else
-            gs_load_row<V, W, false>(pe, pc, pp, off, n_sw - rr, ndw, wrap, nrow, true);
+            gs_load_row<W, false, PV>(ne, nc, pp, off, n_sw - r_, ndw, wrap, nrow, true);
+    };
+    load(0, rr);
+    for (int j = 0; j < mmax; j++) {
+        PV pe[W], pc[W];
+#pragma unroll
+        for (int b = 0; b < W; b++) pe[b] = ne[b], pc[b] = nc[b];
         rr += W;
         rr -= rr >= n_sw ? n_sw : 0;
+        // look-ahead only where registers allow (w = 8 at 64 registers spills)
+        constexpr bool LA = W >= 16;
+        if (LA && j + 1 < mmax) load(j + 1, rr);
 #pragma unroll
         for (int b = 0; b < W; b++) {
-            se[b] += pe[b];
-            sc[b] += pc[b];
+            se[b] += post_cv<V>(pe[b]);
+            sc[b] += post_cv<V>(pc[b]);
         }
+        if (!LA && j + 1 < mmax) load(j + 1, rr);
         if (emit_rows >> j & 1ull) {
             for (int i = 0; i < nl; i++) {
                 const int qi = P.len[i] / W, ri = P.len[i] % W;

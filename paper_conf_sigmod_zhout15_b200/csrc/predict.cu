@@ -11,36 +11,37 @@
 //              u0 = c0^T C^-1 Y,  s0^2 = th0^2 + th2^2 - c0^T C^-1 c0      (Eq. 16-17)
 //
 // All arithmetic in fp64 (the Gram of fp32/int16 inputs is exact in the
-// differences).  C^-1 is applied through its Cholesky factor L (C = L L^T):
-// with z = L^-1 c0 and w = L^-1 Y,  u0 = z.w and c0^T C^-1 c0 = z.z.  The
-// k x k factor lives in shared memory (k_j <= kMaxPredK); the Gram streams
-// the segments through shared memory 64 points at a time.  No tensor cores:
-// k_j^2 d / 2 + k_j^3 / 3 fp64 flops per predictor (at most ~1.8 MFLOP at
-// k = 128, d = 128), a latency-bound small dense problem per CTA.
+// differences).  C^-1 is applied through C = L D L^T (unit lower L): with
+// z = L^-1 c0 and w = L^-1 Y, u0 = sum z_a w_a / D_a and c0^T C^-1 c0 =
+// sum z_a^2 / D_a; the forward solves ride along the elimination (c0 and Y
+// are extra columns), one barrier per column.  The k x k matrix lives in
+// shared memory (k_j <= kMaxPredK); the Gram uses 4 x 4 register tiles of
+// pairs over points staged 32 at a time.  No tensor cores: 3 d k_j^2 / 2 +
+// k_j^3 / 3 fp64 flops per predictor (~3.9 MFLOP at k = 128, d = 128), a
+// small dense problem per CTA.
 #include <math.h>
 
 #include "internal.h"
 
 namespace smiler {
 
-constexpr int kPredThreads = 256;
-constexpr int kPredChunk = 64;  // segment points staged per Gram pass
+constexpr int kPredThreads = 512;
+constexpr int kPredChunk = 32;  // segment points staged per Gram pass
+constexpr int kPredTile = 4;    // Gram register tile (4 x 4 pairs per thread task)
 
 struct PredSensor {
     int64_t off, n;
 };
 
-// staged points [kmax + 1][kPredChunk + 1] floats, rounded up to 16 bytes (int64 follow)
-__host__ __device__ inline size_t pred_xs_bytes(int kmax) {
-    return ((size_t)(kmax + 1) * (kPredChunk + 1) * sizeof(float) + 15) & ~(size_t)15;
-}
+// padded row length (doubles) of the point-major staging Xs[pp][a]
+__host__ __device__ inline int pred_xs_stride(int kmax) { return ((kmax + 1 + kPredTile - 1) / kPredTile) * kPredTile + 2; }
 
 __host__ __device__ inline size_t pred_smem_bytes(int kmax) {
     const int kp = kmax + 1;
-    return (size_t)kp * kp * sizeof(double)                  // Gram / C / L (row-major, lower)
-           + (size_t)4 * kp * sizeof(double)                 // c0, Y, z, w
-           + pred_xs_bytes(kmax)                              // staged points (k_j segments + x0)
-           + (size_t)kp * sizeof(int64_t) + 64;              // neighbour starts, flags
+    return (size_t)kp * kp * sizeof(double)                            // Gram / C / LDL^T (row-major, lower)
+           + (size_t)3 * kp * sizeof(double)                           // c0, Y, D
+           + (size_t)kPredChunk * pred_xs_stride(kmax) * sizeof(double)  // staged points
+           + (size_t)kp * sizeof(int64_t) + 64;                        // neighbour starts, flag
 }
 
 template <typename S>
@@ -53,15 +54,16 @@ __global__ void __launch_bounds__(kPredThreads) predict_kernel(
     const int j = pred % n_k, i = (pred / n_k) % n_len, m = pred / (n_k * n_len);
     const int kj = ekv[j], d = lens[i];
     const int kp = kmax + 1;
+    const int XS = pred_xs_stride(kmax);
     double *G = reinterpret_cast<double *>(pr_smem);  // [kp][kp]
     double *c0 = G + (size_t)kp * kp;
     double *Yv = c0 + kp;
-    double *z = Yv + kp;
-    double *wv = z + kp;
-    float *Xs = reinterpret_cast<float *>(wv + kp);  // [kj + 1][kPredChunk + 1]
-    int64_t *ts = reinterpret_cast<int64_t *>(reinterpret_cast<unsigned char *>(Xs) + pred_xs_bytes(kmax));
+    double *Dg = Yv + kp;
+    double *Xs = Dg + kp;                                   // [kPredChunk][XS], point-major
+    int64_t *ts = reinterpret_cast<int64_t *>(Xs + (size_t)kPredChunk * XS);
     int *flag = reinterpret_cast<int *>(ts + kp);
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    constexpr int NW = kPredThreads / 32;
     const PredSensor sn = sens[qsens[m]];
     const S *c = series + sn.off;
     const S *x0 = queries + (int64_t)m * D + (D - d);  // IQ_i = last d points of the MQ
@@ -81,124 +83,120 @@ __global__ void __launch_bounds__(kPredThreads) predict_kernel(
         return;
     }
     // ---- AR (Eq. 12-13): two passes, warp 0 ----------------------------------
-    if (tid < 32) {
-        double s = 0;
-        for (int a = tid; a < kj; a += 32) s += Yv[a];
+    if (warp == 0) {
+        double sacc = 0;
+        for (int a = lane; a < kj; a += 32) sacc += Yv[a];
 #pragma unroll
-        for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-        const double u = s / kj;
+        for (int o = 16; o; o >>= 1) sacc += __shfl_xor_sync(0xffffffffu, sacc, o);
+        const double u = sacc / kj;
         double v = 0;
-        for (int a = tid; a < kj; a += 32) v += (Yv[a] - u) * (Yv[a] - u);
+        for (int a = lane; a < kj; a += 32) v += (Yv[a] - u) * (Yv[a] - u);
 #pragma unroll
         for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if (tid == 0) {
+        if (lane == 0) {
             ar_mean[out] = u;
             ar_var[out] = v / kj;
         }
     }
-    // ---- Gram: G[a][b] = |x_a - x_b|^2 (a >= b), row kj = x0 -----------------
+    // ---- Gram G[a][b] = |x_a - x_b|^2 (a > b; row kj is x0) in 4 x 4 register
+    // tiles of pairs, points staged 32 at a time as doubles (exact differences)
     const int np = kj + 1;
-    const int npairs = np * (np + 1) / 2;
-    for (int x = tid; x < npairs; x += kPredThreads) {
-        // pair x -> (a, b), a >= b: a = floor((sqrt(8x+1)-1)/2)
-        int a = (int)((sqrt(8.0 * x + 1.0) - 1.0) * 0.5);
-        while ((a + 1) * (a + 2) / 2 <= x) a++;
-        while (a * (a + 1) / 2 > x) a--;
-        G[a * kp + (x - a * (a + 1) / 2)] = 0.0;
-    }
+    const int R = (np + kPredTile - 1) / kPredTile;
+    const int T = R * (R + 1) / 2;  // lower-triangle tiles (ta >= tb)
+    for (int x = tid; x < np * kp; x += kPredThreads) G[x] = 0.0;
     for (int p0 = 0; p0 < d; p0 += kPredChunk) {
         const int pn = min(kPredChunk, d - p0);
         __syncthreads();
-        for (int x = tid; x < np * kPredChunk; x += kPredThreads) {
-            const int a = x / kPredChunk, pp = x % kPredChunk;
-            float v = 0.f;
-            if (pp < pn) v = (float)(a < kj ? c[ts[a] + p0 + pp] : x0[p0 + pp]);
-            Xs[a * (kPredChunk + 1) + pp] = v;
+        for (int x = tid; x < kPredChunk * R * kPredTile; x += kPredThreads) {
+            const int pp = x / (R * kPredTile), a = x % (R * kPredTile);
+            double v = 0.0;
+            if (pp < pn && a < np) v = (double)(a < kj ? c[ts[a] + p0 + pp] : x0[p0 + pp]);
+            Xs[pp * XS + a] = v;
         }
         __syncthreads();
-        for (int x = tid; x < npairs; x += kPredThreads) {
-            int a = (int)((sqrt(8.0 * x + 1.0) - 1.0) * 0.5);
-            while ((a + 1) * (a + 2) / 2 <= x) a++;
-            while (a * (a + 1) / 2 > x) a--;
-            const int b = x - a * (a + 1) / 2;
-            if (a == b) continue;
-            const float *xa = Xs + a * (kPredChunk + 1), *xb = Xs + b * (kPredChunk + 1);
-            double acc = 0.0;
+        for (int tt = tid; tt < T; tt += kPredThreads) {
+            // tile tt -> (ta, tb), ta >= tb (row-major over the lower triangle)
+            int ta = (int)((sqrt(8.0 * tt + 1.0) - 1.0) * 0.5);
+            while ((ta + 1) * (ta + 2) / 2 <= tt) ta++;
+            while (ta * (ta + 1) / 2 > tt) ta--;
+            const int tb = tt - ta * (ta + 1) / 2;
+            double acc[kPredTile][kPredTile];
+#pragma unroll
+            for (int u = 0; u < kPredTile; u++)
+#pragma unroll
+                for (int v = 0; v < kPredTile; v++) acc[u][v] = 0.0;
+            const double *xa = Xs + ta * kPredTile, *xb = Xs + tb * kPredTile;
             for (int pp = 0; pp < pn; pp++) {
-                const double df = (double)xa[pp] - (double)xb[pp];
-                acc = fma(df, df, acc);
+                const double2 a01 = *reinterpret_cast<const double2 *>(xa + pp * XS);
+                const double2 a23 = *reinterpret_cast<const double2 *>(xa + pp * XS + 2);
+                const double2 b01 = *reinterpret_cast<const double2 *>(xb + pp * XS);
+                const double2 b23 = *reinterpret_cast<const double2 *>(xb + pp * XS + 2);
+                const double av[4] = {a01.x, a01.y, a23.x, a23.y}, bv[4] = {b01.x, b01.y, b23.x, b23.y};
+#pragma unroll
+                for (int u = 0; u < kPredTile; u++)
+#pragma unroll
+                    for (int v = 0; v < kPredTile; v++) {
+                        const double df = av[u] - bv[v];
+                        acc[u][v] = fma(df, df, acc[u][v]);
+                    }
             }
-            G[a * kp + b] += acc;
+#pragma unroll
+            for (int u = 0; u < kPredTile; u++)
+#pragma unroll
+                for (int v = 0; v < kPredTile; v++) {
+                    const int a = ta * kPredTile + u, b = tb * kPredTile + v;
+                    if (a < np && b < a) G[a * kp + b] += acc[u][v];
+                }
         }
     }
     __syncthreads();
-    // ---- covariance (Eq. 18) ---------------------------------------------------
-    const double* th = theta + out * 3;
+    // ---- covariance (Eq. 18): C in the lower triangle, c0 = row kj ----------
+    const double *th = theta + out * 3;
     const double t0s = th[0] * th[0], inv2t1 = 0.5 / (th[1] * th[1]), t2s = th[2] * th[2];
-    for (int x = tid; x < npairs; x += kPredThreads) {
-        int a = (int)((sqrt(8.0 * x + 1.0) - 1.0) * 0.5);
-        while ((a + 1) * (a + 2) / 2 <= x) a++;
-        while (a * (a + 1) / 2 > x) a--;
-        const int b = x - a * (a + 1) / 2;
-        const double cv = t0s * exp(-G[a * kp + b] * inv2t1);
-        if (a == kj) {
-            if (b < kj) c0[b] = cv;  // c(x_b, x0): no delta term
-        } else {
-            G[a * kp + b] = cv + (a == b ? t2s : 0.0);
+    for (int a = warp; a < np; a += NW)
+        for (int b = lane; b <= a; b += 32) {
+            const double cv = t0s * exp(-G[a * kp + b] * inv2t1);
+            if (a == kj) {
+                if (b < kj) c0[b] = cv;  // c(x_b, x0): no delta term
+            } else {
+                G[a * kp + b] = cv + (a == b ? t2s : 0.0);
+            }
         }
-    }
     __syncthreads();
-    // ---- Cholesky C = L L^T (right-looking, lower, in place) ------------------
+    // ---- C = L D L^T with the forward solves folded in: eliminating column p
+    // also updates the right-hand sides c0 and Y, so afterwards c0 = L^-1 c0,
+    // Y = L^-1 Y and c0^T C^-1 Y = sum_a c0_a Y_a / D_a (one barrier per column)
     for (int p = 0; p < kj; p++) {
-        if (tid == 0) {
-            const double piv = G[p * kp + p];
-            if (!(piv > 0.0)) *flag = 1;
-            G[p * kp + p] = sqrt(piv > 0.0 ? piv : 1.0);
+        const double dp = G[p * kp + p];
+        if (!(dp > 0.0)) {
+            if (tid == 0) *flag = 1;
+            break;  // uniform: every thread reads the same pivot
         }
-        __syncthreads();
-        const double lpp = G[p * kp + p];
-        for (int r = p + 1 + tid; r < kj; r += kPredThreads) G[r * kp + p] /= lpp;
-        __syncthreads();
-        const int nr = kj - p - 1;
-        for (int x = tid; x < nr * nr; x += kPredThreads) {
-            const int r = p + 1 + x / nr, cc = p + 1 + x % nr;
-            if (cc <= r) G[r * kp + cc] -= G[r * kp + p] * G[cc * kp + p];
+        const double inv = 1.0 / dp;
+        for (int r = p + 1 + warp; r < kj; r += NW) {
+            const double lr = G[r * kp + p] * inv;
+            for (int cc = p + 1 + lane; cc <= r; cc += 32) G[r * kp + cc] -= lr * G[cc * kp + p];
+            if (lane == 0) {
+                c0[r] -= lr * c0[p];
+                Yv[r] -= lr * Yv[p];
+            }
         }
+        if (tid == 0) Dg[p] = dp;
         __syncthreads();
-    }
-    // ---- z = L^-1 c0, w = L^-1 Y (forward substitution, column-oriented) -------
-    for (int a = tid; a < kj; a += kPredThreads) {
-        z[a] = c0[a];
-        wv[a] = Yv[a];
     }
     __syncthreads();
-    for (int p = 0; p < kj; p++) {
-        const double lpp = G[p * kp + p];
-        const double zp = z[p] / lpp, wp = wv[p] / lpp;
-        for (int r = p + 1 + tid; r < kj; r += kPredThreads) {
-            const double l = G[r * kp + p];
-            z[r] -= l * zp;
-            wv[r] -= l * wp;
-        }
-        __syncthreads();
-        if (tid == 0) {
-            z[p] = zp;
-            wv[p] = wp;
-        }
-    }
-    __syncthreads();
-    if (tid < 32) {
+    if (warp == 0) {
         double uw = 0, zz = 0;
-        for (int a = tid; a < kj; a += 32) {
-            uw += z[a] * wv[a];
-            zz += z[a] * z[a];
+        for (int a = lane; a < kj; a += 32) {
+            uw += c0[a] * Yv[a] / Dg[a];
+            zz += c0[a] * c0[a] / Dg[a];
         }
 #pragma unroll
         for (int o = 16; o; o >>= 1) {
             uw += __shfl_xor_sync(0xffffffffu, uw, o);
             zz += __shfl_xor_sync(0xffffffffu, zz, o);
         }
-        if (tid == 0) {
+        if (lane == 0) {
             const bool bad = *flag != 0;
             gp_mean[out] = bad ? nan("") : uw;
             gp_var[out] = bad ? nan("") : t0s + t2s - zz;

@@ -7,6 +7,7 @@
 //   -> a8 topk -> copy out
 // Data-dependent sizes (survivors, finalists) stay on the device; buffers are
 // sized for the worst case (every candidate) and kernels read the counts.
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdarg.h>
@@ -572,6 +573,7 @@ struct StreamCtx {
     int mode;                  // 0: build every row; 1: incremental rows [0, nrows)
     int nrows;
     int64_t *d_prev_out;       // device copy of the results (next step's tau seeds)
+    bool post_half;            // ring entries are fp16 rounded toward zero (f32 index, static w)
 };
 
 template <typename S>
@@ -736,8 +738,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             // tau set ~ mult * k tile candidates per IQ (plus k shifted previous
             // neighbours in a continuous step, where a smaller tile set suffices)
             int mult = use_prev ? kTauMultCont : kTauMult;
-            if (o.reserved[2] > 0) mult = o.reserved[2];
-            if (o.reserved[2] < 0) mult = 0;
+            if (o.tau_mult > 0) mult = o.tau_mult;
+            if (o.tau_mult < 0) mult = 0;
             E = mult > 0 ? std::min(kTauEMax, std::max(1, (mult * pl.k + umin - 1) / umin)) : 0;
             // with previous neighbours the tau list must fit the sorting (dedupe) path
             while (use_prev && E > 0 && nblk_max * units_per_blk * E + pl.k > kSortCap) E--;
@@ -812,6 +814,53 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         CU(cudaEventRecord(idx->meta_ev[mslot], idx->stream));
         CU(cudaMemcpyAsync(idx->queries.p, (const char *)queries + (size_t)c0 * D * es, es * (size_t)B * D,
                            q_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, idx->stream));
+        int32_t *scount = idx->scount.as<int32_t>();
+        int32_t *fcount = idx->fcount.as<int32_t>();
+        uint64_t *taukey = idx->taukey.as<uint64_t>();
+        uint32_t *thr = idx->thr.as<uint32_t>();
+        if (!lb_only) {
+            CU(cudaMemsetAsync(scount, 0, 4 * (size_t)nseg, idx->stream));
+            CU(cudaMemsetAsync(fcount, 0, 4 * (size_t)nseg, idx->stream));
+        }
+        int32_t *taskoff = idx->taskoff.as<int32_t>();
+        auto do_a5 = [&]() -> int {
+            // ---- a5: tau ------------------------------------------------------
+            if (use_prev) {
+                const int64_t *pv = prev_ids + (size_t)c0 * nl * pl.k;
+                if (!is_device_ptr(prev_ids)) {
+                    TRY(idx->tmp2.ensure(8 * (size_t)nseg * pl.k));
+                    CU(cudaMemcpyAsync(idx->tmp2.p, pv, 8 * (size_t)nseg * pl.k, cudaMemcpyHostToDevice, idx->stream));
+                    pv = idx->tmp2.as<int64_t>();
+                }
+                prev_tau_kernel<<<nseg, 128, 0, idx->stream>>>(pv, shift, d_meta, P, LTt, idx->tauc.as<int32_t>());
+                CHECK_LAUNCH();
+                launches++;
+            }
+            if (!o.no_prune) {
+                TRY(side_fork(idx, nl));
+                for (int i = 0; i < nl; i++) {
+                    TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
+                                        taskoff + (size_t)i * (B + 1), idx->tauk.as<uint64_t>(), nullptr,
+                                        nullptr, nullptr, d_meta, idx->qv.as<V>(), D, idx->side[i]));
+                    launches += 2;
+                    tau_slots_total += (int64_t)B * LT;
+                    cells_acc += (double)B * LT * (double)dtw_cells(pl.len[i], pl.rho[i]);
+                }
+                TRY(side_join(idx, nl));
+                tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
+                CHECK_LAUNCH();
+                launches++;
+            } else {
+                CU(cudaMemsetAsync(taukey, 0xFF, 8 * (size_t)nseg, idx->stream));
+            }
+            return SMILER_OK;
+        };
+        // a4+a6 fused: with thresholds known before the scan (a continuous step
+        // seeded only by the previous neighbours, E = 0), the LB kernel compares
+        // each LB_w with tau_i as it is produced and appends the survivors; the
+        // LB_w array is never written or re-read (P:1437-1448 in one pass).
+        const bool fuse = use_prev && E == 0 && !lb_only && !o.no_prune &&
+                          (pl.direct || (pl.fused && pl.fused_kind == 0) || (!pl.fused && pl.scan_reg));
         TRY(tm.mark(0));
         // ---- a2 ----------------------------------------------------------
         query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env,
@@ -819,6 +868,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         CHECK_LAUNCH();
         launches++;
         TRY(tm.mark(1));
+        if (fuse) {
+            TRY(do_a5());
+            TRY(tm.mark(4));
+            P.fuse = 1;
+            P.thr = thr;
+            P.surv = idx->surv.as<int32_t>();
+            P.scount = scount;
+        }
         if (pl.direct) {
             // ---- SMiLer-Dir (ablation): LB_en per candidate, no window level --
             dim3 grid((unsigned)nblk_max, (unsigned)B);
@@ -880,17 +937,30 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 // continuous step, static w: SW_0 (EQ + EC) and SW_1..SW_rho (EQ only)
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
                 size_t smem = 3 * sizeof(V) * D;
-                auto go = [&](auto kern) {
+                auto go = [&](auto kern, auto *pb) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           sctx->nrows, sctx->cursor, postbuf);
+                                                           sctx->nrows, sctx->cursor, pb);
                 };
-                switch (w) {
-                    case 4: go(window_lb_inc_kernel<S, 4>); break;
-                    case 8: go(window_lb_inc_kernel<S, 8>); break;
-                    case 16: go(window_lb_inc_kernel<S, 16>); break;
-                    default: go(window_lb_inc_kernel<S, 32>); break;
+                if constexpr (std::is_same<S, float>::value) {
+                    if (sctx->post_half) {
+                        __half *hb = reinterpret_cast<__half *>(sctx->ring);
+                        switch (w) {
+                            case 4: go(window_lb_inc_kernel<S, 4, __half>, hb); break;
+                            case 8: go(window_lb_inc_kernel<S, 8, __half>, hb); break;
+                            case 16: go(window_lb_inc_kernel<S, 16, __half>, hb); break;
+                            default: go(window_lb_inc_kernel<S, 32, __half>, hb); break;
+                        }
+                    }
+                }
+                if (!sctx->post_half) {
+                    switch (w) {
+                        case 4: go(window_lb_inc_kernel<S, 4>, postbuf); break;
+                        case 8: go(window_lb_inc_kernel<S, 8>, postbuf); break;
+                        case 16: go(window_lb_inc_kernel<S, 16>, postbuf); break;
+                        default: go(window_lb_inc_kernel<S, 32>, postbuf); break;
+                    }
                 }
                 CHECK_LAUNCH();
                 launches++;
@@ -898,37 +968,63 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 // every row (ring cursor 0 when a stream is created)
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
                 size_t smem = 3 * sizeof(V) * D;
-                auto go = [&](auto kern) {
+                auto go = [&](auto kern, auto *pb) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           w, postbuf);
+                                                           w, pb);
                 };
-                switch (w) {
-                    case 4: go(window_lb_kernel<S, 4>); break;
-                    case 8: go(window_lb_kernel<S, 8>); break;
-                    case 16: go(window_lb_kernel<S, 16>); break;
-                    case 32: go(window_lb_kernel<S, 32>); break;
-                    default: go(window_lb_kernel<S, 0>); break;
+                bool done_half = false;
+                if constexpr (std::is_same<S, float>::value) {
+                    if (sctx && sctx->post_half) {
+                        __half *hb = reinterpret_cast<__half *>(sctx->ring);
+                        done_half = true;
+                        switch (w) {
+                            case 4: go(window_lb_kernel<S, 4, __half>, hb); break;
+                            case 8: go(window_lb_kernel<S, 8, __half>, hb); break;
+                            case 16: go(window_lb_kernel<S, 16, __half>, hb); break;
+                            default: go(window_lb_kernel<S, 32, __half>, hb); break;
+                        }
+                    }
+                }
+                if (!done_half) switch (w) {
+                    case 4: go(window_lb_kernel<S, 4>, postbuf); break;
+                    case 8: go(window_lb_kernel<S, 8>, postbuf); break;
+                    case 16: go(window_lb_kernel<S, 16>, postbuf); break;
+                    case 32: go(window_lb_kernel<S, 32>, postbuf); break;
+                    default: go(window_lb_kernel<S, 0>, postbuf); break;
                 }
                 CHECK_LAUNCH();
                 launches++;
             }
-            post_bytes += post_tot * (int64_t)sizeof(V);
+            post_bytes += post_tot * (int64_t)((sctx && sctx->post_half) ? 2 : sizeof(V));
             TRY(tm.mark(2));
             // ---- a4 ----------------------------------------------------------
             dim3 grid((unsigned)nblk_max, (unsigned)B);
-            auto go4 = [&](auto kern) {
+            auto go4 = [&](auto kern, auto *pb) {
                 set_smem((const void *)kern, pl.smem_gs);
-                kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(postbuf, d_meta, P, idx->lb.as<V>(),
+                kern<<<grid, pl.RT, pl.smem_gs, idx->stream>>>(pb, d_meta, P, idx->lb.as<V>(),
                                                                idx->tauc.as<int32_t>());
             };
-            switch (pl.scan_reg ? w : 0) {
-                case 4: go4(group_scan_reg_kernel<S, 4>); break;
-                case 8: go4(group_scan_reg_kernel<S, 8>); break;
-                case 16: go4(group_scan_reg_kernel<S, 16>); break;
-                case 32: go4(group_scan_reg_kernel<S, 32>); break;
-                default: go4(group_scan_kernel<S, 0>); break;
+            bool done4 = false;
+            if constexpr (std::is_same<S, float>::value) {
+                if (sctx && sctx->post_half) {
+                    __half *hb = reinterpret_cast<__half *>(sctx->ring);
+                    done4 = true;
+                    switch (w) {
+                        case 4: go4(group_scan_reg_kernel<S, 4, __half>, hb); break;
+                        case 8: go4(group_scan_reg_kernel<S, 8, __half>, hb); break;
+                        case 16: go4(group_scan_reg_kernel<S, 16, __half>, hb); break;
+                        default: go4(group_scan_reg_kernel<S, 32, __half>, hb); break;
+                    }
+                }
+            }
+            if (!done4) switch (pl.scan_reg ? w : 0) {
+                case 4: go4(group_scan_reg_kernel<S, 4>, postbuf); break;
+                case 8: go4(group_scan_reg_kernel<S, 8>, postbuf); break;
+                case 16: go4(group_scan_reg_kernel<S, 16>, postbuf); break;
+                case 32: go4(group_scan_reg_kernel<S, 32>, postbuf); break;
+                default: go4(group_scan_kernel<S, 0>, postbuf); break;
             }
             CHECK_LAUNCH();
             launches++;
@@ -949,48 +1045,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             c0 = c1;
             continue;
         }
-        int32_t *scount = idx->scount.as<int32_t>();
-        int32_t *fcount = idx->fcount.as<int32_t>();
-        uint64_t *taukey = idx->taukey.as<uint64_t>();
-        uint32_t *thr = idx->thr.as<uint32_t>();
-        CU(cudaMemsetAsync(scount, 0, 4 * (size_t)nseg, idx->stream));
-        CU(cudaMemsetAsync(fcount, 0, 4 * (size_t)nseg, idx->stream));
-        int32_t *taskoff = idx->taskoff.as<int32_t>();
-        // ---- a5: tau ------------------------------------------------------
-        if (use_prev) {
-            const int64_t *pv = prev_ids + (size_t)c0 * nl * pl.k;
-            if (!is_device_ptr(prev_ids)) {
-                TRY(idx->tmp2.ensure(8 * (size_t)nseg * pl.k));
-                CU(cudaMemcpyAsync(idx->tmp2.p, pv, 8 * (size_t)nseg * pl.k, cudaMemcpyHostToDevice, idx->stream));
-                pv = idx->tmp2.as<int64_t>();
-            }
-            prev_tau_kernel<<<nseg, 128, 0, idx->stream>>>(pv, shift, d_meta, P, LTt, idx->tauc.as<int32_t>());
-            CHECK_LAUNCH();
-            launches++;
-        }
-        if (!o.no_prune) {
-            TRY(side_fork(idx, nl));
-            for (int i = 0; i < nl; i++) {
-                TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
-                                    taskoff + (size_t)i * (B + 1), idx->tauk.as<uint64_t>(), nullptr,
-                                    nullptr, nullptr, d_meta, idx->qv.as<V>(), D, idx->side[i]));
-                launches += 2;
-                tau_slots_total += (int64_t)B * LT;
-                cells_acc += (double)B * LT * (double)dtw_cells(pl.len[i], pl.rho[i]);
-            }
-            TRY(side_join(idx, nl));
-            tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
-            CHECK_LAUNCH();
-            launches++;
-        } else {
-            CU(cudaMemsetAsync(taukey, 0xFF, 8 * (size_t)nseg, idx->stream));
-        }
+        if (!fuse) TRY(do_a5());
         TRY(tm.mark(4));
         // ---- a6 ----------------------------------------------------------
         {
             int64_t nmax = 0;
             for (int j = 0; j < B; j++) nmax = std::max(nmax, meta[j].n);
-            if (!o.no_prune) {
+            if (fuse) {
+                // survivors were appended by the LB kernel
+            } else if (!o.no_prune) {
                 dim3 grid((unsigned)((nmax + kFiltThreads * kFiltItems - 1) / (kFiltThreads * kFiltItems)),
                           (unsigned)nseg);
                 filter_kernel<S><<<grid, kFiltThreads, 0, idx->stream>>>(idx->lb.as<V>(), d_meta, P, thr,
@@ -999,8 +1062,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 dim3 grid((unsigned)std::min<int64_t>((nmax + 255) / 256, 1024), (unsigned)nseg);
                 all_candidates_kernel<<<grid, 256, 0, idx->stream>>>(d_meta, P, idx->surv.as<int32_t>(), scount);
             }
-            CHECK_LAUNCH();
-            launches++;
+            if (!fuse) {
+                CHECK_LAUNCH();
+                launches++;
+            }
         }
         TRY(tm.mark(5));
         // ---- a7 ----------------------------------------------------------
@@ -1116,6 +1181,7 @@ struct smiler_stream {
     void *d_new = nullptr;     // [n] staging for new points
     void *ring = nullptr;      // posting-list rings
     int64_t *d_prev = nullptr; // [n][n_len][k] last results
+    bool post_half = false;    // ring entries fp16 rounded toward zero (see post_st in lb.cuh)
     int cursor = 0;
     int64_t steps = 0;
 };
@@ -1141,13 +1207,15 @@ static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_s
     sc.mode = mode;
     sc.nrows = st->nrows;
     sc.d_prev_out = st->d_prev;
+    sc.post_half = st->post_half;
     return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
                        stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
 }
 
-extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, const int32_t *query_sensor,
-                                    int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
-                                    int64_t *ids, void *dists, smiler_stream **out) {
+extern "C" int smiler_stream_create_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                       int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
+                                       int64_t *ids, void *dists, const smiler_knn_opts *opts,
+                                       smiler_stream **out) {
     if (!out) return fail(SMILER_EINVAL, "out is NULL");
     *out = nullptr;
     if (!idx || !queries || !lengths || !ids || !dists) return fail(SMILER_EINVAL, "NULL argument");
@@ -1178,6 +1246,8 @@ extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, cons
     st->D = pl.D;
     st->n_sw = pl.D - pl.w + 1;
     st->nrows = std::min(pl.rho_env + 1, st->n_sw);
+    // fp16 ring (rounded toward zero) for f32 indices on the register group scan
+    st->post_half = idx->dtype == SMILER_F32 && pl.scan_reg && !(opts && opts->exact_postings);
     st->qsens.assign(n_streams, 0);
     if (query_sensor) {
         if (is_device_ptr(query_sensor)) cudaMemcpy(st->qsens.data(), query_sensor, 4 * (size_t)n_streams, cudaMemcpyDeviceToHost);
@@ -1194,7 +1264,7 @@ extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, cons
         tot += 2 * (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
     }
     const size_t es = esize(idx->dtype);
-    cudaError_t e = cudaMalloc(&st->ring, 4 * (size_t)std::max<int64_t>(tot, 1));
+    cudaError_t e = cudaMalloc(&st->ring, (st->post_half ? 2 : 4) * (size_t)std::max<int64_t>(tot, 1));
     if (e == cudaSuccess) e = cudaMalloc(&st->d_mq, es * (size_t)n_streams * pl.D);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_new, es * (size_t)n_streams);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_prev, 8 * (size_t)n_streams * n_len * k);
@@ -1216,6 +1286,13 @@ extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, cons
     }
     *out = st;
     return SMILER_OK;
+}
+
+extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, const int32_t *query_sensor,
+                                    int32_t n_streams, const int32_t *lengths, int32_t n_len, int32_t k,
+                                    int64_t *ids, void *dists, smiler_stream **out) {
+    return smiler_stream_create_ex(idx, queries, query_sensor, n_streams, lengths, n_len, k, ids, dists, nullptr,
+                                   out);
 }
 
 extern "C" int smiler_stream_step(smiler_stream *st, const void *new_points, int64_t *ids, void *dists,

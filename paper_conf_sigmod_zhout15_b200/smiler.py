@@ -46,7 +46,8 @@ class KnnStats(ctypes.Structure):
 class KnnOpts(ctypes.Structure):
     _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
                 ("mq_chunk", ctypes.c_int32), ("two_level", ctypes.c_int32),
-                ("lb_kind", ctypes.c_int32), ("horizon", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+                ("lb_kind", ctypes.c_int32), ("horizon", ctypes.c_int32),
+                ("exact_postings", ctypes.c_int32), ("tau_mult", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
@@ -73,6 +74,7 @@ def lib():
         L.smiler_knn_ex.argtypes = [P, P, P, i32, P, i32, i32, P, P, P, P]
         L.smiler_knn_step.argtypes = [P, P, P, i32, P, i32, i32, P, i32, P, P, P, P]
         L.smiler_stream_create.argtypes = [P, P, P, i32, P, i32, i32, P, P, ctypes.POINTER(P)]
+        L.smiler_stream_create_ex.argtypes = [P, P, P, i32, P, i32, i32, P, P, P, ctypes.POINTER(P)]
         L.smiler_stream_step.argtypes = [P, P, P, P, P, P]
         L.smiler_stream_free.argtypes = [P]
         L.smiler_stream_free.restype = None
@@ -87,7 +89,7 @@ def lib():
         L.smiler_last_error.restype = ctypes.c_char_p
         L.smiler_abi_version.restype = i32
         for f in ("smiler_index_build", "smiler_index_build_shard", "smiler_knn", "smiler_knn_ex", "smiler_knn_step",
-                  "smiler_stream_create", "smiler_stream_step",
+                  "smiler_stream_create", "smiler_stream_create_ex", "smiler_stream_step",
                   "smiler_merge_topk", "smiler_index_envelope", "smiler_lower_bounds", "smiler_lower_bounds_ex",
                   "smiler_dtw", "smiler_predict"):
             getattr(L, f).restype = i32
@@ -183,14 +185,16 @@ def smiler_knn_step(handle: int, queries, query_sensor, lengths, k: int, prev_id
                                  ctypes.byref(opts) if opts is not None else None))
 
 
-def smiler_stream_create(handle: int, queries, query_sensor, lengths, k: int, ids, dists) -> int:
+def smiler_stream_create(handle: int, queries, query_sensor, lengths, k: int, ids, dists,
+                         opts: Optional[KnnOpts] = None) -> int:
     """Create a batch of continuous streams (Remark 1) and run their first search."""
     h = ctypes.c_void_p()
     lens = np.ascontiguousarray(lengths, dtype=np.int32)
     qs = None if query_sensor is None else np.ascontiguousarray(query_sensor, np.int32)
     _check("smiler_stream_create",
-           lib().smiler_stream_create(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens), len(lens),
-                                      k, _ptr(ids), _ptr(dists), ctypes.byref(h)))
+           lib().smiler_stream_create_ex(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens),
+                                         len(lens), k, _ptr(ids), _ptr(dists),
+                                         ctypes.byref(opts) if opts is not None else None, ctypes.byref(h)))
     return h.value
 
 
@@ -276,21 +280,23 @@ def smiler_abi_version() -> int:
 class Stream:
     """A batch of continuous master-query streams over one Index (host numpy I/O)."""
 
-    def __init__(self, index: "Index", queries, lengths: Sequence[int], k: int, query_sensor=None):
+    def __init__(self, index: "Index", queries, lengths: Sequence[int], k: int, query_sensor=None,
+                 exact_postings: bool = False):
         self.index, self.lengths, self.k = index, list(lengths), k
         self.n = int(queries.shape[0])
         self.vt = np.int32 if index.dtype == SMILER_I16 else np.float32
         ids = np.empty((self.n, len(lengths), k), np.int64)
         dists = np.empty((self.n, len(lengths), k), self.vt)
         self.handle = smiler_stream_create(index.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
-                                           ids, dists)
+                                           ids, dists, KnnOpts(exact_postings=int(exact_postings)))
         self.first = (ids, dists)
 
-    def step(self, new_points, stats: bool = False, timing: bool = False):
+    def step(self, new_points, stats: bool = False, timing: bool = False, tau_mult: int = 0):
         ids = np.empty((self.n, len(self.lengths), self.k), np.int64)
         dists = np.empty((self.n, len(self.lengths), self.k), self.vt)
         st = KnnStats() if stats else None
-        smiler_stream_step(self.handle, np.ascontiguousarray(new_points), ids, dists, st, KnnOpts(timing=int(timing)))
+        smiler_stream_step(self.handle, np.ascontiguousarray(new_points), ids, dists, st,
+                           KnnOpts(timing=int(timing), tau_mult=int(tau_mult)))
         if stats:
             return ids, dists, st.as_dict()
         return ids, dists
@@ -353,12 +359,12 @@ class Index:
         return tuple(outs)
 
     def knn_step(self, queries, lengths: Sequence[int], k: int, prev_ids, shift: int = 1, query_sensor=None,
-                 stats: bool = False, timing: bool = False):
+                 stats: bool = False, timing: bool = False, tau_mult: int = 0):
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
-        op = KnnOpts(timing=int(timing))
+        op = KnnOpts(timing=int(timing), tau_mult=int(tau_mult))
         smiler_knn_step(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
                         np.ascontiguousarray(prev_ids, dtype=np.int64), shift, ids, dists, st, op)
         if stats:

@@ -28,7 +28,7 @@ def test_header_declares_the_boundary():
     for f in ("smiler_index_build", "smiler_knn", "smiler_free", "smiler_merge_topk",
               "smiler_index_build_shard", "smiler_knn_ex", "smiler_lower_bounds", "smiler_dtw",
               "smiler_index_envelope", "smiler_last_error", "smiler_abi_version", "smiler_lower_bounds_ex",
-              "smiler_predict"):
+              "smiler_predict", "smiler_stream_create_ex"):
         assert f in fns, f
 
 
@@ -43,7 +43,7 @@ def test_abi_version_and_stats_layout(built):
     assert pkg.smiler_abi_version() == 2
     # struct sizes match the header (8 x 8-byte counters, 2 int32, 8 doubles)
     assert ctypes.sizeof(pkg.KnnStats) == 8 * 8 + 2 * 4 + 8 * 8
-    assert ctypes.sizeof(pkg.KnnOpts) == 10 * 4
+    assert ctypes.sizeof(pkg.KnnOpts) == 11 * 4
 
 
 def test_no_gpu_means_error_not_fallback(built):

@@ -357,7 +357,10 @@ def test_c2_full_size_sampled(pkg, orc, dtype):
 # continuous steps (Def. 4.1; threshold method 2, P:1452-1458 / R9)
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
-def test_continuous_steps(pkg, orc, dtype):
+@pytest.mark.parametrize("tau_mult", [0, -1, 2])
+def test_continuous_steps(pkg, orc, dtype, tau_mult):
+    """tau_mult -1: thresholds from the previous neighbours only, so the LB
+    kernel filters as it scans (a4+a6 fused); 2: plus a tile tau set."""
     kw = dict(n=12001, n_sensors=3, mq_per_sensor=2)
     wl = synth.make_workload("C5", dtype, step=0, **kw)
     with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
@@ -365,7 +368,8 @@ def test_continuous_steps(pkg, orc, dtype):
         for s in range(1, 4):
             ws = synth.make_workload("C5", dtype, step=s, **kw)
             assert (ws.series == wl.series).all()
-            ids, dists, st = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 1, ws.query_sensor, stats=True)
+            ids, dists, st = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 1, ws.query_sensor, stats=True,
+                                          tau_mult=tau_mult)
             # the k previous neighbours are part of every item query's tau list
             assert st["tau_verified"] >= ws.n_mq * len(ws.lengths) * ws.k
             if dtype == "i16":
@@ -378,11 +382,11 @@ def test_continuous_steps(pkg, orc, dtype):
                 np.testing.assert_array_equal(dists, od)
         # useless previous neighbours (all padding): tau = +inf, still exact
         bad = np.full_like(ids, -1)
-        i2, d2 = idx.knn_step(ws.queries, ws.lengths, ws.k, bad, 1, ws.query_sensor)
+        i2, d2 = idx.knn_step(ws.queries, ws.lengths, ws.k, bad, 1, ws.query_sensor, tau_mult=tau_mult)
         np.testing.assert_array_equal(i2, ids)
         np.testing.assert_array_equal(d2, dists)
         # stale neighbours from far away still give a valid (loose) threshold
-        i3, d3 = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 50, ws.query_sensor)
+        i3, d3 = idx.knn_step(ws.queries, ws.lengths, ws.k, ids, 50, ws.query_sensor, tau_mult=tau_mult)
         np.testing.assert_array_equal(i3, ids)
         np.testing.assert_array_equal(d3, dists)
 
@@ -478,18 +482,18 @@ def test_device_buffers_and_streams(pkg):
 # ---------------------------------------------------------------------------
 # continuous streams with the reused window-level index (Remark 1)
 # ---------------------------------------------------------------------------
-def _stream_case(pkg, orc, dtype, name, steps, **kw):
+def _stream_case(pkg, orc, dtype, name, steps, exact_postings=False, tau_mult=0, **kw):
     wl = synth.make_workload(name, dtype, step=0, **kw)
     D = wl.D
     with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
-        with pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor) as st:
+        with pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor, exact_postings=exact_postings) as st:
             ids, dists = st.first
             for s in range(steps + 1):
                 ws = wl if s == 0 else synth.make_workload(name, dtype, step=s, **kw)
                 if s > 0:
                     newp = np.ascontiguousarray(ws.queries[:, D - 1])   # the point appended at step s
                     assert (ws.queries[:, :D - 1] == prev_q[:, 1:]).all()
-                    ids, dists, stt = st.step(newp, stats=True)
+                    ids, dists, stt = st.step(newp, stats=True, tau_mult=tau_mult)
                     assert stt["posting_bytes"] > 0
                 prev_q = ws.queries
                 if s % 3 and s != steps:
@@ -504,12 +508,32 @@ def _stream_case(pkg, orc, dtype, name, steps, **kw):
                     np.testing.assert_array_equal(dists, od)
 
 
-@pytest.mark.parametrize("dtype", ["i16", "f32"])
-def test_stream_steps_c5_shape(pkg, orc, dtype):
-    _stream_case(pkg, orc, dtype, "C5", 6, n=12001, n_sensors=3, mq_per_sensor=2)
+# f32 streams store their postings as fp16 rounded toward zero unless
+# exact_postings (a valid, slightly looser bound: the kNN must not change)
+@pytest.mark.parametrize("tau_mult", [0, -1, 2])
+@pytest.mark.parametrize("dtype,exact", [("i16", False), ("f32", False), ("f32", True)])
+def test_stream_steps_c5_shape(pkg, orc, dtype, exact, tau_mult):
+    _stream_case(pkg, orc, dtype, "C5", 6, exact_postings=exact, tau_mult=tau_mult, n=12001, n_sensors=3,
+                 mq_per_sensor=2)
 
 
-@pytest.mark.parametrize("dtype", ["i16", "f32"])
-def test_stream_ring_wraps(pkg, orc, dtype):
+@pytest.mark.parametrize("tau_mult", [0, -1])
+@pytest.mark.parametrize("dtype,exact", [("i16", False), ("f32", False), ("f32", True)])
+def test_stream_ring_wraps(pkg, orc, dtype, exact, tau_mult):
     """D = 32, w = 8: 25 sliding windows, so 30 steps wrap the ring cursor."""
-    _stream_case(pkg, orc, dtype, "C1", 30, n=3000, lengths=[16, 32], window=8, band=3.0, k=6, mq_per_sensor=3)
+    _stream_case(pkg, orc, dtype, "C1", 30, exact_postings=exact, tau_mult=tau_mult, n=3000, lengths=[16, 32],
+                 window=8, band=3.0, k=6, mq_per_sensor=3)
+
+
+def test_stream_fp16_postings_saturate(pkg, orc):
+    """Values whose posting sums exceed fp16's range (65504): rounding toward
+    zero saturates, the bound stays valid, the kNN stays exact."""
+    wl = synth.make_workload("C1", "f32", n=3000, lengths=[16, 32], window=8, band=3.0, k=6, mq_per_sensor=3)
+    wl.series = (wl.series * 300.0).astype(np.float32)
+    wl.queries = (wl.queries * 300.0).astype(np.float32)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        with pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor) as st:
+            ids, dists = st.first
+    oid, od = orc.knn(wl, mode="f32", threads=THREADS)
+    np.testing.assert_array_equal(ids, oid)
+    np.testing.assert_array_equal(dists, od)

@@ -15,7 +15,8 @@ steps = int(sys.argv[4]) if len(sys.argv) > 4 else 4
 wl = synth.make_workload(cfg, dtype, n_sensors=ns, consecutive=True)
 nxt = synth.make_workload(cfg, dtype, n_sensors=ns, consecutive=True, step=steps)
 idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band)
-st = pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor)
+exact = len(sys.argv) > 5 and sys.argv[5] == "exact"
+st = pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor, exact_postings=exact)
 D = wl.D
 acc = {}
 for s in range(steps):

@@ -25,7 +25,7 @@ cont = len(sys.argv) > 3 and sys.argv[3] == "cont"
 prev = None
 for mult in ((-1, 2, 4, 8, 16) if cont else (8, 16, 32, 64, 128)):
     op = pkg.KnnOpts(no_prune=0, timing=1, mq_chunk=0, two_level=0)
-    op.reserved[2] = mult
+    op.tau_mult = mult
     s = pkg.KnnStats()
     for it in range(2):
         if cont:
