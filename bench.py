@@ -223,6 +223,9 @@ class Runner:
                                        device=local, stream=stream)
             self.index_points = len(sl)
             self.global_mq = wl.n_mq              # every rank serves the same MQs
+            # NEXT-2: a running threshold shared by the ranks' shards (opt-in)
+            self.tau_bufs = sdist.shared_tau_buffers(wl.n_mq * len(wl.lengths), dev) if args.shared_tau else None
+            self.step_no = 0
         else:
             self.idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band, device=local, stream=stream)
             self.index_points = len(wl.series)
@@ -296,10 +299,23 @@ class Runner:
                                stats, op)
                 self.have_prev = True
             return
+        self._arm_shared_tau(op)
         pkg.smiler_knn(self.idx.handle, self.qd, self.qs, self.wl.lengths, self.k, self.ids, self.dd, stats, op)
         if self.sharded_window:
             with self.torch.cuda.stream(self.stream):
                 self._merge(self.ids, self.dd)
+
+    def _arm_shared_tau(self, op):
+        """Step s uses shared buffer s % 2; rank 0 resets the other one first (it is
+        next used after this step's all-gather, which orders the reset before it)."""
+        if not (self.sharded_window and self.tau_bufs):
+            return
+        s = self.step_no
+        self.step_no += 1
+        if self.rank == 0:
+            with self.torch.cuda.stream(self.stream):
+                self.sdist.reset_shared_tau(self.tau_bufs[(s + 1) % 2])
+        op.shared_tau = self.tau_bufs[s % 2].data_ptr()
 
     def e2e_buffers(self):
         torch = self.torch
@@ -342,7 +358,9 @@ class Runner:
             return
         with torch.cuda.stream(self.stream):
             self.qd.copy_(self.qh, non_blocking=True)
-        pkg.smiler_knn(self.idx.handle, self.qd, None, self.wl.lengths, self.k, self.ids, self.dd)
+        self._arm_shared_tau(self.op_fast)
+        pkg.smiler_knn(self.idx.handle, self.qd, None, self.wl.lengths, self.k, self.ids, self.dd, None,
+                       self.op_fast)
         with torch.cuda.stream(self.stream):
             oi, od = self._merge(self.ids, self.dd)
             self.ih.copy_(oi, non_blocking=True)
@@ -367,6 +385,8 @@ def main():
                     help="C3/C5: do not use the reused window-level index (smiler_stream_step); C5 then uses "
                          "smiler_knn_step, C3 independent searches")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--shared-tau", action="store_true",
+                    help="C4: ranks share a running threshold through CUDA IPC / NVLink atomics (NEXT-2)")
     ap.add_argument("--two-level", action="store_true", help="time the paper's two-level path (a3 -> HBM -> a4)")
     ap.add_argument("--two-level-steps", type=int, default=3,
                     help="extra steps of the two-level path for the LB-scan (a4) HBM figure; 0 = skip")
@@ -543,7 +563,10 @@ def main():
         pts = [int(wl.offsets[s + 1] - wl.offsets[s]) for s in wl.query_sensor.tolist()]
     # algorithmic work: (SW, DW, j) term pairs = n_sw * n_dw * w per MQ
     win_terms = n_sw * sum(p // wl.window * wl.window for p in pts)
-    post_bytes_step = 8 * n_sw * sum(p // wl.window for p in pts)
+    # bytes per (P_EQ, P_EC) pair as stored: f32 streams keep fp16 entries rounded
+    # toward zero (smiler_knn_opts.exact_postings = 0), otherwise 2 x 4 bytes
+    pair_bytes = 4 if (R.streaming and args.dtype == "f32" and wl.window in (4, 8, 16, 32)) else 8
+    post_bytes_step = pair_bytes * n_sw * sum(p // wl.window for p in pts)
     lb_bytes_step = 4 * n_len * sum(pts)
 
     # continuous streams recompute only SW_0 (EQ + EC) and SW_1..SW_rho_max (EQ):

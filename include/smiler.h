@@ -98,6 +98,17 @@ typedef struct smiler_knn_opts {
                          step the thresholds exist before the scan, and the LB kernel
                          filters as it goes (a4+a6 fused, no LB_w array) */
     int32_t reserved[3];
+    uint64_t *shared_tau; /* NULL, or a running threshold shared by calls that split ONE
+                         search (window-range shards of the same series and master
+                         queries): [n_mq][n_len] keys
+                         (float/int dist bits << 32 | global t), device memory of this
+                         GPU or of a peer reachable over NVLink, set to all ones before
+                         the first call.  Each call atomically lowers entry (m, i) to its
+                         own threshold key (a5) and prunes with the minimum it reads
+                         back -- every key written is an upper bound of the k-th NN key
+                         of the whole search, so the merged top-k is unchanged while later
+                         shards verify fewer candidates; a shard's own list may then hold
+                         fewer than k entries (padded) */
 } smiler_knn_opts;
 
 /* smiler_knn_opts.lb_kind.  The default is the paper's method; the others are

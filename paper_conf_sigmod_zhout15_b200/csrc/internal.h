@@ -39,7 +39,11 @@ struct MQMeta {
     int64_t origin;      // global id of local t = 0
     int64_t t_lo, t_hi;  // owned candidate starts, local coordinates
     int64_t n_dw;        // floor(N / w) disjoint windows
-    int64_t post_off;    // element offset of this MQ's P_EQ plane [n_sw][n_dw]; P_EC plane follows
+    int64_t post_off;    // element offset of this MQ's P_EQ plane [prows][pstride]; P_EC plane follows
+    int64_t pstride;     // posting row stride (elements): n_dw, or n_dw rounded up to 8 (TMA ring)
+    int32_t prows;       // posting rows per plane: n_sw, or n_sw + w - 1 (TMA ring: physical rows
+                         // 0 .. w-2 mirrored after row n_sw - 1, so any w consecutive ring rows
+                         // are contiguous)
     int64_t seg_off;     // offset of this MQ's per-candidate segments; (mq,i) at seg_off + i*n
     int64_t hz;          // prediction horizon h (local): candidates must end by n - hz (C_{t,d} with
                          // c_{t+d-1+h} in the series); 0 = every segment

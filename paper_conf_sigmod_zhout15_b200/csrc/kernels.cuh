@@ -1,6 +1,7 @@
 // kernels.cuh -- steps a1-a6, a8, a9 of the Search Step.
 // Included once, by smiler.cu.  DTW (a5/a7) is in dtw.cu.
 #pragma once
+#include <cuda.h>
 #include <cuda_fp16.h>
 #include <stdint.h>
 
@@ -237,6 +238,17 @@ __global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D
 // int: dist; f32: dist * (1 + 2^-10) rounded up (R16 rounding slack).
 // no candidates enough -> key max / thr = +inf (no pruning).
 // ---------------------------------------------------------------------------
+// LB admission bound of a threshold key: int: the distance; f32: distance x
+// (1 + 2^-10) rounded up (R16 rounding slack); no key -> no pruning.
+template <typename V> __device__ __forceinline__ uint32_t thr_from_key(uint64_t key) {
+    if (key == kKeyMax) return std::is_same<V, float>::value ? 0x7f800000u : 0x7FFFFFFFu;
+    const uint32_t db = (uint32_t)(key >> 32);
+    if constexpr (std::is_same<V, float>::value)
+        return __float_as_uint(__fmul_ru(__uint_as_float(db), 1.0f + 1.0f / 1024.0f));
+    else
+        return db;
+}
+
 template <typename S>
 __global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, int LT, int k,
                                                         uint64_t *tau_key, uint32_t *thr) {
@@ -281,17 +293,43 @@ __global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, i
     }
     if (threadIdx.x == 0) {
         tau_key[seg] = kth;
-        if (kth == kKeyMax) {
-            thr[seg] = std::is_same<V, float>::value ? 0x7f800000u : 0x7FFFFFFFu;
-        } else {
-            uint32_t db = (uint32_t)(kth >> 32);
-            if constexpr (std::is_same<V, float>::value) {
-                float tf = __uint_as_float(db);
-                thr[seg] = __float_as_uint(__fmul_ru(tf, 1.0f + 1.0f / 1024.0f));
-            } else {
-                thr[seg] = db;
-            }
-        }
+        thr[seg] = thr_from_key<V>(kth);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// NEXT-2: running threshold shared by the shards of one search (smiler_knn_opts
+// .shared_tau).  Each segment's local threshold key becomes global (t + origin),
+// is atomically min'ed into the shared entry (system scope: the entry may live
+// on a peer GPU), and the minimum read back -- an upper bound of the k-th NN
+// key of the whole search, since every shard's key is one -- is converted back
+// to this shard's local coordinates: local key <= result  <=>  global key <= g.
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void tau_share_kernel(uint64_t *tau_key, uint32_t *thr, unsigned long long *shared, const MQMeta *meta,
+                                 int n_len, int nseg) {
+    using V = typename Tr<S>::V;
+    const int seg = blockIdx.x * blockDim.x + threadIdx.x;
+    if (seg >= nseg) return;
+    const int64_t origin = meta[seg / n_len].origin;
+    const uint64_t k = tau_key[seg];
+    uint64_t g;
+    if (k != kKeyMax) {
+        const uint64_t kg = (k & 0xFFFFFFFF00000000ull) | (uint32_t)((k & 0xFFFFFFFFull) + (uint64_t)origin);
+        const uint64_t old = atomicMin_system(shared + seg, (unsigned long long)kg);
+        g = old < kg ? old : kg;
+    } else {
+        g = atomicMin_system(shared + seg, (unsigned long long)kKeyMax);  // read
+    }
+    uint64_t loc = g;
+    if (g != kKeyMax) {
+        const uint64_t gt = g & 0xFFFFFFFFull;
+        if (gt >= (uint64_t)origin) loc = (g & 0xFFFFFFFF00000000ull) | (gt - (uint64_t)origin);
+        else loc = (g & 0xFFFFFFFF00000000ull) - 1;  // same distance, smaller global t: none of ours ties
+    }
+    if (loc < k) {
+        tau_key[seg] = loc;
+        thr[seg] = thr_from_key<V>(loc);
     }
 }
 

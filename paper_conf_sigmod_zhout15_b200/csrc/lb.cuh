@@ -278,10 +278,12 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
     if (r >= m.n_dw) return;
     const int64_t ndw = m.n_dw;
     PV *oe = post + m.post_off + r;  // P_EQ plane; P_EC plane `plane` further
+    const int64_t pst = m.pstride;
     if constexpr (W > 0) {
         constexpr int BC = W < 8 ? W : 8;
         const int n_sw = D - W + 1;
-        const int64_t plane = (int64_t)n_sw * ndw;
+        const int64_t plane = (int64_t)m.prows * pst;
+        const int nmir = m.prows - n_sw;  // mirrored leading rows (TMA ring)
         const int64_t base = m.series_off + r * W;
         V c[W], U[W], L[W];
 #pragma unroll
@@ -291,26 +293,25 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
             L[j] = (V)LC[base + j];
         }
         int b0 = 0;
-        for (; b0 + BC <= n_sw; b0 += BC) {
-            PV *o = oe + (int64_t)b0 * ndw;
+        auto put = [&](int b, V eq, V ec) {  // ring cursor 0 at a full build: row b
+            PV *o = oe + (int64_t)b * pst;
+            post_st(o, eq);
+            post_st(o + plane, ec);
+            if (b < nmir) {
+                post_st(o + (int64_t)n_sw * pst, eq);
+                post_st(o + (int64_t)n_sw * pst + plane, ec);
+            }
+        };
+        for (; b0 + BC <= n_sw; b0 += BC)
             posting_chunk<V, W, BC, false>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
-                                           [&](int bb, V eq, V ec) {
-                                               post_st(o + bb * ndw, eq);
-                                               post_st(o + bb * ndw + plane, ec);
-                                           });
-        }
-        if (b0 < n_sw) {
-            PV *o = oe + (int64_t)b0 * ndw;
+                                           [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
+        if (b0 < n_sw)
             posting_chunk<V, W, BC, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-                                          [&](int bb, V eq, V ec) {
-                                              post_st(o + bb * ndw, eq);
-                                              post_st(o + bb * ndw + plane, ec);
-                                          });
-        }
+                                          [&](int bb, V eq, V ec) { put(b0 + bb, eq, ec); });
     } else {
         const int w = w_rt;
         const int n_sw = D - w + 1;
-        const int64_t plane = (int64_t)n_sw * ndw;
+        const int64_t plane = (int64_t)m.prows * pst;
         const int64_t base = m.series_off + r * w;
         for (int b = 0; b < n_sw; b++) {
             const int p0 = D - w - b;
@@ -319,8 +320,8 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
                 lb_term((V)series[base + j], squ[p0 + j], sql[p0 + j], eq);
                 lb_term(sqq[p0 + j], (V)UC[base + j], (V)LC[base + j], ec);
             }
-            post_st(oe + (int64_t)b * ndw, eq);
-            post_st(oe + (int64_t)b * ndw + plane, ec);
+            post_st(oe + (int64_t)b * pst, eq);
+            post_st(oe + (int64_t)b * pst + plane, ec);
         }
     }
 }
@@ -368,25 +369,29 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
         U[j] = (V)UC[base + j];
         L[j] = (V)LC[base + j];
     }
-    auto row_ptr = [&](int b) {
+    const int64_t pst = m.pstride;
+    const int64_t plane = (int64_t)m.prows * pst;
+    const int nmir = m.prows - n_ring;  // mirrored leading physical rows (TMA ring)
+    // store one entry of logical row b (physical (b + cursor) mod n_sw, and its mirror)
+    auto put = [&](int b, int pl, V v) {
         int row = b + cursor;
         row -= row >= n_ring ? n_ring : 0;
-        return oe + (int64_t)row * ndw;
+        PV *o = oe + (int64_t)pl * plane + (int64_t)row * pst;
+        post_st(o, v);
+        if (row < nmir) post_st(o + (int64_t)n_ring * pst, v);
     };
     // SW_0: both lists
     posting_chunk<V, W, 1, false>(c, U, L, sqq, squ, sql, D - W, 1, [&](int, V eq, V ec) {
-        PV *o = row_ptr(0);
-        post_st(o, eq);
-        post_st(o + (int64_t)n_ring * ndw, ec);
+        put(0, 0, eq);
+        put(0, 1, ec);
     });
     int b0 = 1;
     for (; b0 + BC <= n_sw; b0 += BC)
-        posting_chunk<V, W, BC, false, true>(
-            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC, [&](int bb, V eq, V) { post_st(row_ptr(b0 + bb), eq); });
+        posting_chunk<V, W, BC, false, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                             [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
     if (b0 < n_sw)
-        posting_chunk<V, W, BC, true, true>(
-            c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-            [&](int bb, V eq, V) { post_st(row_ptr(b0 + bb), eq); });
+        posting_chunk<V, W, BC, true, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
+                                            [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
 }
 
 // ---------------------------------------------------------------------------
@@ -1046,6 +1051,145 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
                     V v[W];
 #pragma unroll
                     for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
+                    diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
+                }
+            }
+        }
+        if (save_rows >> j & 1ull) {
+#pragma unroll
+            for (int b = 0; b < W; b++) s_saved[b][x] = lbpick(P, se[b], sc[b]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a4 over the continuous-stream ring, TMA-staged (the HBM-bound "LB scan").
+// The ring of every stream is one 2-D tensor: rows = (stream, plane, physical
+// SW row) with the first w-1 physical rows mirrored after the last (so the w
+// ring rows of one CSG row are contiguous for any cursor), columns = disjoint
+// windows (row stride padded to 16 bytes).  For CSG row j the CTA's 256
+// rightmost DWs r = Rb .. Rb+255 need columns r - j of the w rows
+// (j w + cursor) mod n_sw + b: one w x 256 TMA box per plane (columns < 0 or
+// >= n_dw arrive zero-filled), landing in a 4-stage shared-memory ring armed
+// with mbarriers; thread x then reads its column x of each row (conflict-free
+// 2- or 4-byte loads) -- no per-element address arithmetic, whole 512-byte
+// rows per request.  Sums, emission and the tau set are group_scan_reg's.
+// ---------------------------------------------------------------------------
+constexpr int kTmaStages = 4;
+template <int W, typename PV> constexpr size_t tma_scan_smem() { return (size_t)kTmaStages * 2 * W * kScanThreads * sizeof(PV); }
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int c0, int c1, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
+            "r"(smem_u32(dst)),
+        "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+
+template <typename S, int W, typename PV>
+__global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tma_kernel(
+    const __grid_constant__ CUtensorMap tmap, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb,
+    int32_t *tauc) {
+    using V = typename Tr<S>::V;
+    constexpr int NT = kScanThreads;
+    constexpr int PLANE = W * NT;                 // PV per plane per stage
+    constexpr uint32_t STAGE_BYTES = 2 * PLANE * sizeof(PV);
+    extern __shared__ __align__(128) unsigned char tma_smem[];
+    PV (*s_tile)[2][W][NT] = reinterpret_cast<PV (*)[2][W][NT]>(tma_smem);  // [kTmaStages]
+    __shared__ __align__(8) uint64_t s_full[kTmaStages];
+    __shared__ V s_saved[W][NT];
+    const int D = P.D;
+    const int nl = P.n_len;
+    const int n_sw = D - W + 1;
+    const int mmax = D / W;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, NT / 32, 0, P.n_len, tauc);
+        return;
+    }
+    const int x = threadIdx.x;
+    const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
+    const int64_t r = Rb + x;
+    const int64_t s0 = (r + 1) * W;  // e of slot b = 0
+    const int row_base = (int)(m.post_off / m.pstride);  // tensor row of this stream's P_EQ row 0
+    auto issue = [&](int j) {         // CSG row j -> stage j % kTmaStages
+        int pr = j * W + P.ring_cursor;
+        pr -= pr >= n_sw ? n_sw : 0;
+        pr -= pr >= n_sw ? n_sw : 0;
+        const int st = j % kTmaStages;
+        mbar_expect_tx(&s_full[st], STAGE_BYTES);
+        const int col = (int)(Rb - j);
+        tma_load_2d(&s_tile[st][0][0][0], &tmap, col, row_base + pr, &s_full[st]);
+        tma_load_2d(&s_tile[st][1][0][0], &tmap, col, row_base + m.prows + pr, &s_full[st]);
+    };
+    if (x == 0) {
+        for (int st = 0; st < kTmaStages; st++) mbar_init(&s_full[st], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (x == 0)
+        for (int j = 0; j < kTmaStages && j < mmax; j++) issue(j);
+    V se[W], sc[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
+    uint64_t emit_rows = 0, save_rows = 0;
+    for (int i = 0; i < nl; i++) {
+        const int qi = P.len[i] / W;
+        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
+        if (qi >= 2) save_rows |= 1ull << (qi - 2);
+    }
+    if (nl > 0 && P.len[0] < W) {
+        V z[W];
+#pragma unroll
+        for (int b = 0; b < W; b++) z[b] = (V)0;
+        for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq);
+    }
+    for (int j = 0; j < mmax; j++) {
+        const int st = j % kTmaStages;
+        mbar_wait(&s_full[st], (uint32_t)(j / kTmaStages) & 1u);
+        const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
+#pragma unroll
+        for (int b = 0; b < W; b++) {
+            if (b < nrow) {
+                se[b] += post_cv<V>(s_tile[st][0][b][x]);
+                sc[b] += post_cv<V>(s_tile[st][1][b][x]);
+            }
+        }
+        __syncthreads();  // every thread has read stage st
+        if (x == 0 && j + kTmaStages < mmax) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            issue(j + kTmaStages);
+        }
+        if (emit_rows >> j & 1ull) {
+            for (int i = 0; i < nl; i++) {
+                const int qi = P.len[i] / W, ri = P.len[i] % W;
+                if (j == qi - 1) {
+                    V v[W];
+#pragma unroll
+                    for (int b = 0; b < W; b++)
+                        v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
                     diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }

@@ -7,6 +7,8 @@
 //   -> a8 topk -> copy out
 // Data-dependent sizes (survivors, finalists) stay on the device; buffers are
 // sized for the worst case (every candidate) and kernels read the counts.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <math.h>
@@ -141,6 +143,8 @@ struct smiler_index {
     cudaEvent_t fork_ev = nullptr;
     cudaEvent_t join_ev[kMaxLen] = {};
 };
+
+static inline int64_t m_ndw_of(const SensorInfo &si, int w) { return si.n / w; }
 
 static int side_fork(smiler_index *idx, int n) {
     if (!idx->fork_ev) CU(cudaEventCreateWithFlags(&idx->fork_ev, cudaEventDisableTiming));
@@ -574,6 +578,10 @@ struct StreamCtx {
     int nrows;
     int64_t *d_prev_out;       // device copy of the results (next step's tau seeds)
     bool post_half;            // ring entries are fp16 rounded toward zero (f32 index, static w)
+    bool tma;                  // ring laid out for group_scan_tma_kernel (padded stride, mirrored rows)
+    int64_t pstride;           // ring row stride (elements)
+    int prows;                 // ring rows per plane
+    const CUtensorMap *tmap;   // the ring as one 2-D tensor (tma)
 };
 
 template <typename S>
@@ -710,6 +718,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             m.hz = std::max<int64_t>(0, (int64_t)o.horizon - (si.n_global - (si.slice_begin + si.n)));
             m.n_dw = si.n / w;
             m.post_off = sctx ? sctx->ring_off[c0 + j] : post_tot;
+            m.pstride = (sctx && sctx->tma) ? sctx->pstride : m_ndw_of(si, pl.w);
+            m.prows = (sctx && sctx->tma) ? sctx->prows : pl.D - pl.w + 1;
             m.seg_off = seg_tot;
             m.nblk = pl.direct ? (int)(m.n / kDirEnds + 1) : (int)(m.n_dw / (pl.fused ? pl.RTf : pl.RT) + 1);
             m.sensor = qsens[c0 + j];
@@ -850,6 +860,13 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
                 CHECK_LAUNCH();
                 launches++;
+                if (o.shared_tau) {  // NEXT-2: running threshold shared across the shards
+                    tau_share_kernel<S><<<(nseg + 255) / 256, 256, 0, idx->stream>>>(
+                        taukey, thr, reinterpret_cast<unsigned long long *>(o.shared_tau) + (size_t)c0 * nl, d_meta,
+                        nl, nseg);
+                    CHECK_LAUNCH();
+                    launches++;
+                }
             } else {
                 CU(cudaMemsetAsync(taukey, 0xFF, 8 * (size_t)nseg, idx->stream));
             }
@@ -1007,8 +1024,37 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                                                                idx->tauc.as<int32_t>());
             };
             bool done4 = false;
+            if (sctx && sctx->tma) {  // TMA-staged ring scan
+                done4 = true;
+                auto go5 = [&](auto kern, size_t smem) {
+                    set_smem((const void *)kern, smem);
+                    kern<<<grid, kScanThreads, smem, idx->stream>>>(*sctx->tmap, d_meta, P, idx->lb.as<V>(),
+                                                                    idx->tauc.as<int32_t>());
+                };
+                if constexpr (std::is_same<S, float>::value) {
+                    if (sctx->post_half) {
+                        switch (w) {
+                            case 4: go5(group_scan_tma_kernel<S, 4, __half>, tma_scan_smem<4, __half>()); break;
+                            case 8: go5(group_scan_tma_kernel<S, 8, __half>, tma_scan_smem<8, __half>()); break;
+                            default: go5(group_scan_tma_kernel<S, 16, __half>, tma_scan_smem<16, __half>()); break;
+                        }
+                    } else {
+                        switch (w) {
+                            case 4: go5(group_scan_tma_kernel<S, 4, float>, tma_scan_smem<4, float>()); break;
+                            case 8: go5(group_scan_tma_kernel<S, 8, float>, tma_scan_smem<8, float>()); break;
+                            default: go5(group_scan_tma_kernel<S, 16, float>, tma_scan_smem<16, float>()); break;
+                        }
+                    }
+                } else {
+                    switch (w) {
+                        case 4: go5(group_scan_tma_kernel<S, 4, V>, tma_scan_smem<4, V>()); break;
+                        case 8: go5(group_scan_tma_kernel<S, 8, V>, tma_scan_smem<8, V>()); break;
+                        default: go5(group_scan_tma_kernel<S, 16, V>, tma_scan_smem<16, V>()); break;
+                    }
+                }
+            }
             if constexpr (std::is_same<S, float>::value) {
-                if (sctx && sctx->post_half) {
+                if (!done4 && sctx && sctx->post_half) {
                     __half *hb = reinterpret_cast<__half *>(sctx->ring);
                     done4 = true;
                     switch (w) {
@@ -1182,6 +1228,10 @@ struct smiler_stream {
     void *ring = nullptr;      // posting-list rings
     int64_t *d_prev = nullptr; // [n][n_len][k] last results
     bool post_half = false;    // ring entries fp16 rounded toward zero (see post_st in lb.cuh)
+    bool tma = false;          // ring as one TMA tensor (group_scan_tma_kernel)
+    int64_t pstride = 0;       // ring row stride (elements)
+    int prows = 0;             // ring rows per plane
+    CUtensorMap tmap;
     int cursor = 0;
     int64_t steps = 0;
 };
@@ -1208,6 +1258,10 @@ static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_s
     sc.nrows = st->nrows;
     sc.d_prev_out = st->d_prev;
     sc.post_half = st->post_half;
+    sc.tma = st->tma;
+    sc.pstride = st->pstride;
+    sc.prows = st->prows;
+    sc.tmap = &st->tmap;
     return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
                        stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
 }
@@ -1255,16 +1309,71 @@ extern "C" int smiler_stream_create_ex(smiler_index *idx, const void *queries, c
     }
     int64_t tot = 0;
     st->ring_off.resize(n_streams);
+    int64_t ndw0 = -1;
+    bool same_ndw = true;
     for (int j = 0; j < n_streams; j++) {
         if (st->qsens[j] < 0 || st->qsens[j] >= (int)idx->sensors.size()) {
             stream_release(st);
             return fail(SMILER_EINVAL, "query_sensor[%d] out of range", j);
         }
+        const int64_t ndw = idx->sensors[st->qsens[j]].n / pl.w;
+        if (ndw0 < 0) ndw0 = ndw;
+        same_ndw = same_ndw && ndw == ndw0;
+    }
+    // TMA ring (group_scan_tma_kernel): every stream's sensor has the same n_dw,
+    // row stride padded to 8 entries (16-byte rows), first w-1 rows mirrored
+    const int pbytes = st->post_half ? 2 : 4;
+    st->tma = pl.scan_reg && (pl.w == 4 || pl.w == 8 || pl.w == 16) && same_ndw && ndw0 >= 1 &&
+              !(opts && opts->reserved[0] == 7);  // reserved[0] == 7: A/B without TMA
+    st->pstride = st->tma ? (ndw0 + 7) / 8 * 8 : 0;
+    st->prows = st->tma ? st->n_sw + pl.w - 1 : st->n_sw;
+    for (int j = 0; j < n_streams; j++) {
         st->ring_off[j] = tot;
-        tot += 2 * (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
+        const int64_t ndw = idx->sensors[st->qsens[j]].n / pl.w;
+        tot += st->tma ? 2 * (int64_t)st->prows * st->pstride : 2 * (int64_t)st->n_sw * ndw;
+    }
+    if (st->tma && tot / st->pstride > INT32_MAX) st->tma = false;  // TMA row coordinates are int32
+    if (!st->tma) {  // plain layout
+        tot = 0;
+        st->prows = st->n_sw;
+        for (int j = 0; j < n_streams; j++) {
+            st->ring_off[j] = tot;
+            tot += 2 * (int64_t)st->n_sw * (idx->sensors[st->qsens[j]].n / pl.w);
+        }
     }
     const size_t es = esize(idx->dtype);
-    cudaError_t e = cudaMalloc(&st->ring, (st->post_half ? 2 : 4) * (size_t)std::max<int64_t>(tot, 1));
+    cudaError_t e = cudaMalloc(&st->ring, (size_t)pbytes * (size_t)std::max<int64_t>(tot, 1));
+    if (e == cudaSuccess && st->tma) {
+        // the mirror rows and the row padding are never read as valid data, but
+        // start them at zero so the ring holds no uninitialised bytes
+        e = cudaMemsetAsync(st->ring, 0, (size_t)pbytes * (size_t)tot, idx->stream);
+        static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+        if (!encode) {
+            void *fn = nullptr;
+            cudaDriverEntryPointQueryResult q;
+            if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+                q == cudaDriverEntryPointSuccess)
+                encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+        }
+        if (!encode) {
+            stream_release(st);
+            return fail(SMILER_ECUDA, "cuTensorMapEncodeTiled unavailable");
+        }
+        const CUtensorMapDataType dt = st->post_half ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                       : idx->dtype == SMILER_F32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                                                  : CU_TENSOR_MAP_DATA_TYPE_INT32;
+        const cuuint64_t gdim[2] = {(cuuint64_t)ndw0, (cuuint64_t)(tot / st->pstride)};
+        const cuuint64_t gstride[1] = {(cuuint64_t)st->pstride * pbytes};
+        const cuuint32_t box[2] = {(cuuint32_t)kScanThreads, (cuuint32_t)pl.w};
+        const cuuint32_t estr[2] = {1, 1};
+        CUresult cr = encode(&st->tmap, dt, 2, st->ring, gdim, gstride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (cr != CUDA_SUCCESS) {
+            stream_release(st);
+            return fail(SMILER_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
+        }
+    }
     if (e == cudaSuccess) e = cudaMalloc(&st->d_mq, es * (size_t)n_streams * pl.D);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_new, es * (size_t)n_streams);
     if (e == cudaSuccess) e = cudaMalloc(&st->d_prev, 8 * (size_t)n_streams * n_len * k);

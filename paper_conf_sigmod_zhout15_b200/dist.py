@@ -98,3 +98,36 @@ def window_sharded_knn(series_slice, shard: WindowShard, n_global: int, queries,
         return oi.view(n_mq, nl, k), od.view(n_mq, nl, k)
     finally:
         idx.close()
+
+
+def shared_tau_buffers(rows: int, device, n: int = 2, group=None):
+    """NEXT-2: `n` device buffers of `rows` threshold keys
+    (smiler_knn_opts.shared_tau), allocated on rank 0's GPU and mapped into every
+    rank through CUDA IPC, so each rank's atomicMin reaches them over NVLink.
+    All ones (-1) = no threshold yet.  Use buffer s % n for step s and reset the
+    next one (rank 0, `reset_shared_tau`) before the step's collective, so no
+    rank can see a previous batch's minima."""
+    import torch
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    handles = None
+    bufs = None
+    if rank == 0:
+        bufs = [torch.full((rows,), -1, dtype=torch.int64, device=device) for _ in range(n)]
+        handles = [b.untyped_storage()._share_cuda_() for b in bufs]
+        torch.cuda.synchronize(device)
+    obj = [handles]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    if rank != 0:
+        bufs = []
+        for h in obj[0]:
+            st = torch.UntypedStorage._new_shared_cuda(*h)
+            t = torch.empty(0, dtype=torch.int64, device=st.device)
+            t.set_(st, 0, (rows,), (1,))
+            bufs.append(t)
+    return bufs
+
+
+def reset_shared_tau(buf) -> None:
+    """Back to 'no threshold' (all ones); rank 0 only, on its stream."""
+    buf.fill_(-1)

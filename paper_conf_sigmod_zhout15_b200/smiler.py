@@ -47,7 +47,8 @@ class KnnOpts(ctypes.Structure):
     _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
                 ("mq_chunk", ctypes.c_int32), ("two_level", ctypes.c_int32),
                 ("lb_kind", ctypes.c_int32), ("horizon", ctypes.c_int32),
-                ("exact_postings", ctypes.c_int32), ("tau_mult", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+                ("exact_postings", ctypes.c_int32), ("tau_mult", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3),
+                ("shared_tau", ctypes.c_void_p)]
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
@@ -336,13 +337,17 @@ class Index:
 
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
             no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False,
-            lb_kind: int = 0, horizon: int = 0):
+            lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0):
+        """kNN of every item query (smiler_knn_ex).  shared_tau: optional device
+        buffer (torch int64 tensor of n_mq * n_len entries, all ones = -1 at start)
+        shared by the window-range shards of one search (NEXT-2)."""
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
         op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level),
-                     lb_kind=int(lb_kind), horizon=int(horizon))
+                     lb_kind=int(lb_kind), horizon=int(horizon), tau_mult=int(tau_mult),
+                     shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
         smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()

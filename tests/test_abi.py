@@ -43,7 +43,7 @@ def test_abi_version_and_stats_layout(built):
     assert pkg.smiler_abi_version() == 2
     # struct sizes match the header (8 x 8-byte counters, 2 int32, 8 doubles)
     assert ctypes.sizeof(pkg.KnnStats) == 8 * 8 + 2 * 4 + 8 * 8
-    assert ctypes.sizeof(pkg.KnnOpts) == 11 * 4
+    assert ctypes.sizeof(pkg.KnnOpts) == 11 * 4 + 4 + 8   # + padding + shared_tau
 
 
 def test_no_gpu_means_error_not_fallback(built):

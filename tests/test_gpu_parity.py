@@ -292,6 +292,46 @@ def test_shards_merge_equals_unsharded(pkg, orc, dtype):
         np.testing.assert_array_equal(md.reshape(full_d.shape), full_d)
 
 
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+@pytest.mark.parametrize("tau_mult", [0, 1])
+def test_shards_shared_running_tau(pkg, orc, dtype, tau_mult):
+    """NEXT-2: shards of one search share a running threshold (atomicMin of
+    global keys): the merged top-k is unchanged, later shards verify no more
+    candidates than alone, and shards that hold none of the global top-k may
+    return padded lists."""
+    import torch
+    wl = synth.make_workload("C4", dtype, n=40009, mq_per_sensor=2)
+    full_ids, full_d = check_workload(pkg, orc, wl)
+    N, D, w = len(wl.series), wl.D, wl.window
+    rho_env = max(wl.rhos())
+    rows = wl.n_mq * len(wl.lengths)
+    for G in (2, 4, 8):
+        bounds = [((N * g) // G) // w * w for g in range(G)] + [N]
+        shared = torch.full((rows,), -1, dtype=torch.int64, device="cuda")
+        outs_i, outs_d, surv_sh, surv_alone = [], [], 0, 0
+        for g in range(G):
+            t0, t1 = bounds[g], bounds[g + 1]
+            s0 = max(0, t0 - rho_env) // w * w
+            s1 = min(N, t1 + D - 1 + rho_env)
+            sl = np.ascontiguousarray(wl.series[s0:s1])
+            with pkg.Index.shard(sl, s0, N, t0, t1, w, wl.band) as idx:
+                i_, d_, st = idx.knn(wl.queries, wl.lengths, wl.k, stats=True, shared_tau=shared,
+                                     tau_mult=tau_mult)
+                _, _, st0 = idx.knn(wl.queries, wl.lengths, wl.k, stats=True, tau_mult=tau_mult)
+            surv_sh += st["survivors"]
+            surv_alone += st0["survivors"]
+            outs_i.append(i_)
+            outs_d.append(d_)
+        I = np.ascontiguousarray(np.stack(outs_i))
+        Dd = np.ascontiguousarray(np.stack(outs_d))
+        mi = np.empty((rows, wl.k), np.int64)
+        md = np.empty((rows, wl.k), Dd.dtype)
+        pkg.smiler_merge_topk(I, Dd, G, rows, wl.k, mi, md)
+        np.testing.assert_array_equal(mi.reshape(full_ids.shape), full_ids)
+        np.testing.assert_array_equal(md.reshape(full_d.shape), full_d)
+        assert surv_sh <= surv_alone, (G, surv_sh, surv_alone)
+
+
 def test_errors_on_gpu(pkg):
     x = np.zeros(100, np.int16)
     x[5] = 2000
