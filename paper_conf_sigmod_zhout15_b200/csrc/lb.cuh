@@ -1069,14 +1069,31 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
 // ring rows of one CSG row are contiguous for any cursor), columns = disjoint
 // windows (row stride padded to 16 bytes).  For CSG row j the CTA's 256
 // rightmost DWs r = Rb .. Rb+255 need columns r - j of the w rows
-// (j w + cursor) mod n_sw + b: one w x 256 TMA box per plane (columns < 0 or
-// >= n_dw arrive zero-filled), landing in a 4-stage shared-memory ring armed
-// with mbarriers; thread x then reads its column x of each row (conflict-free
-// 2- or 4-byte loads) -- no per-element address arithmetic, whole 512-byte
-// rows per request.  Sums, emission and the tau set are group_scan_reg's.
+// (j w + cursor) mod n_sw + b.  A tiled TMA box must start on a 16-byte
+// boundary of the innermost dimension (a misaligned start coordinate traps
+// with "illegal instruction", measured: tools/tma_probe.cu), so per plane the
+// CTA loads a w x 256 box at the aligned column ca = floor((Rb - j) / A) A
+// (A = 16 bytes / entry) and, through a second tensor map, a w x A tail box
+// at ca + 256; columns < 0 or
+// >= n_dw arrive zero-filled.  Both land in a 4-stage shared-memory ring armed
+// with mbarriers; thread x then reads column x + (Rb - j - ca) of each row
+// (from the main box, or the tail for the last few threads) -- conflict-free
+// 2- or 4-byte loads, no per-element address arithmetic, whole 512-byte rows
+// per request.  Sums, emission and the tau set are group_scan_reg's.
 // ---------------------------------------------------------------------------
 constexpr int kTmaStages = 4;
-template <int W, typename PV> constexpr size_t tma_scan_smem() { return (size_t)kTmaStages * 2 * W * kScanThreads * sizeof(PV); }
+template <typename PV> constexpr int tma_align_elems() { return 16 / (int)sizeof(PV); }
+// one stage: per plane a [W][256] main box and a [W][A] tail box, every box at
+// a 128-byte aligned shared-memory offset
+template <int W, typename PV> constexpr int tma_tail_pitch() {  // elements per tail box incl. padding
+    return (int)((W * 16 + 127) / 128 * 128 / sizeof(PV));
+}
+template <int W, typename PV> constexpr size_t tma_stage_elems() {
+    return (size_t)2 * W * kScanThreads + 2 * tma_tail_pitch<W, PV>();
+}
+template <int W, typename PV> constexpr size_t tma_scan_smem() {
+    return (size_t)kTmaStages * tma_stage_elems<W, PV>() * sizeof(PV);
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -1109,14 +1126,17 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
 
 template <typename S, int W, typename PV>
 __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tma_kernel(
-    const __grid_constant__ CUtensorMap tmap, const MQMeta *meta, const QParams P, typename Tr<S>::V *lb,
-    int32_t *tauc) {
+    const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_tail, const MQMeta *meta,
+    const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
     using V = typename Tr<S>::V;
     constexpr int NT = kScanThreads;
-    constexpr int PLANE = W * NT;                 // PV per plane per stage
-    constexpr uint32_t STAGE_BYTES = 2 * PLANE * sizeof(PV);
+    constexpr int A = tma_align_elems<PV>();      // TMA start-column granule (16 bytes)
+    constexpr int STAGE = (int)tma_stage_elems<W, PV>();
+    constexpr int TP = tma_tail_pitch<W, PV>();
+    constexpr uint32_t STAGE_BYTES = 2 * W * (NT + A) * sizeof(PV);  // bytes the four boxes deliver
     extern __shared__ __align__(128) unsigned char tma_smem[];
-    PV (*s_tile)[2][W][NT] = reinterpret_cast<PV (*)[2][W][NT]>(tma_smem);  // [kTmaStages]
+    // stage st: [plane 0 main W x NT][plane 1 main W x NT][plane 0 tail W x A][plane 1 tail W x A]
+    PV *s_ring = reinterpret_cast<PV *>(tma_smem);
     __shared__ __align__(8) uint64_t s_full[kTmaStages];
     __shared__ V s_saved[W][NT];
     const int D = P.D;
@@ -1141,8 +1161,12 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
         const int st = j % kTmaStages;
         mbar_expect_tx(&s_full[st], STAGE_BYTES);
         const int col = (int)(Rb - j);
-        tma_load_2d(&s_tile[st][0][0][0], &tmap, col, row_base + pr, &s_full[st]);
-        tma_load_2d(&s_tile[st][1][0][0], &tmap, col, row_base + m.prows + pr, &s_full[st]);
+        const int ca = col - (((col % A) + A) % A);  // floor to the 16-byte granule
+        PV *sb = s_ring + (size_t)st * STAGE;
+        tma_load_2d(sb, &tmap, ca, row_base + pr, &s_full[st]);
+        tma_load_2d(sb + W * NT, &tmap, ca, row_base + m.prows + pr, &s_full[st]);
+        tma_load_2d(sb + 2 * W * NT, &tmap_tail, ca + NT, row_base + pr, &s_full[st]);
+        tma_load_2d(sb + 2 * W * NT + TP, &tmap_tail, ca + NT, row_base + m.prows + pr, &s_full[st]);
     };
     if (x == 0) {
         for (int st = 0; st < kTmaStages; st++) mbar_init(&s_full[st], 1);
@@ -1170,11 +1194,18 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
         const int st = j % kTmaStages;
         mbar_wait(&s_full[st], (uint32_t)(j / kTmaStages) & 1u);
         const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
+        const int col = (int)(Rb - j);
+        const int xo = x + (((col % A) + A) % A);  // this thread's column within the aligned boxes
+        const PV *sb = s_ring + (size_t)st * STAGE;
+        const bool main_box = xo < NT;
+        const PV *pe = main_box ? sb + xo : sb + 2 * W * NT + (xo - NT);
+        const int rs = main_box ? NT : A;       // row pitch of the box the column lies in
+        const int ps = main_box ? W * NT : TP;  // offset of the P_EC box
 #pragma unroll
         for (int b = 0; b < W; b++) {
             if (b < nrow) {
-                se[b] += post_cv<V>(s_tile[st][0][b][x]);
-                sc[b] += post_cv<V>(s_tile[st][1][b][x]);
+                se[b] += post_cv<V>(pe[b * rs]);
+                sc[b] += post_cv<V>(pe[ps + b * rs]);
             }
         }
         __syncthreads();  // every thread has read stage st

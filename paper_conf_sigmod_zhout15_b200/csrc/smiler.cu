@@ -581,7 +581,8 @@ struct StreamCtx {
     bool tma;                  // ring laid out for group_scan_tma_kernel (padded stride, mirrored rows)
     int64_t pstride;           // ring row stride (elements)
     int prows;                 // ring rows per plane
-    const CUtensorMap *tmap;   // the ring as one 2-D tensor (tma)
+    const CUtensorMap *tmap;   // the ring as one 2-D tensor (tma): w x 256 boxes
+    const CUtensorMap *tmap_tail;  // the same tensor, w x (16 bytes) boxes
 };
 
 template <typename S>
@@ -1028,7 +1029,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 done4 = true;
                 auto go5 = [&](auto kern, size_t smem) {
                     set_smem((const void *)kern, smem);
-                    kern<<<grid, kScanThreads, smem, idx->stream>>>(*sctx->tmap, d_meta, P, idx->lb.as<V>(),
+                    kern<<<grid, kScanThreads, smem, idx->stream>>>(*sctx->tmap, *sctx->tmap_tail, d_meta, P, idx->lb.as<V>(),
                                                                     idx->tauc.as<int32_t>());
                 };
                 if constexpr (std::is_same<S, float>::value) {
@@ -1231,7 +1232,7 @@ struct smiler_stream {
     bool tma = false;          // ring as one TMA tensor (group_scan_tma_kernel)
     int64_t pstride = 0;       // ring row stride (elements)
     int prows = 0;             // ring rows per plane
-    CUtensorMap tmap;
+    CUtensorMap tmap, tmap_tail;
     int cursor = 0;
     int64_t steps = 0;
 };
@@ -1262,6 +1263,7 @@ static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_s
     sc.pstride = st->pstride;
     sc.prows = st->prows;
     sc.tmap = &st->tmap;
+    sc.tmap_tail = &st->tmap_tail;
     return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
                        stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
 }
@@ -1366,9 +1368,14 @@ extern "C" int smiler_stream_create_ex(smiler_index *idx, const void *queries, c
         const cuuint64_t gstride[1] = {(cuuint64_t)st->pstride * pbytes};
         const cuuint32_t box[2] = {(cuuint32_t)kScanThreads, (cuuint32_t)pl.w};
         const cuuint32_t estr[2] = {1, 1};
+        // tail boxes: 16 bytes wide (group_scan_tma_kernel loads from 16-byte aligned columns)
+        const cuuint32_t box_tail[2] = {(cuuint32_t)(16 / pbytes), (cuuint32_t)pl.w};
         CUresult cr = encode(&st->tmap, dt, 2, st->ring, gdim, gstride, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (cr == CUDA_SUCCESS)
+            cr = encode(&st->tmap_tail, dt, 2, st->ring, gdim, gstride, box_tail, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         if (cr != CUDA_SUCCESS) {
             stream_release(st);
             return fail(SMILER_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)cr);
