@@ -97,7 +97,8 @@ typedef struct smiler_knn_opts {
                          > 0 = that many, < 0 = none.  With no tile set in a continuous
                          step the thresholds exist before the scan, and the LB kernel
                          filters as it goes (a4+a6 fused, no LB_w array) */
-    int32_t reserved[3];
+    int32_t reserved[3];  /* 0; reserved[0] selects internal A/B variants in experiments (7: stream
+                             ring without TMA, 8: one tile per group-scan CTA) */
     uint64_t *shared_tau; /* NULL, or a running threshold shared by calls that split ONE
                          search (window-range shards of the same series and master
                          queries): [n_mq][n_len] keys

@@ -32,11 +32,12 @@ template <typename V> __device__ __forceinline__ V lbpick(const QParams &P, V eq
 // chunk) still own tau-list slots: mark them empty (-1) so the tau DTW pass
 // never reads a stale t from an earlier call.
 __device__ __forceinline__ void tau_clear(const QParams &P, int mq, int units_per_blk, int li0, int li1,
-                                          int32_t *tauc) {
+                                          int32_t *tauc, int bx = -1) {
     if (P.E <= 0 || P.k < 0) return;
     const int n = units_per_blk * P.E;
+    const int64_t tile = bx >= 0 ? bx : (int)blockIdx.x;
     for (int i = li0; i < li1; i++) {
-        int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)blockIdx.x * n;
+        int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + tile * n;
         for (int x = threadIdx.x; x < n; x += blockDim.x) dst[x] = -1;
     }
 }
@@ -656,7 +657,7 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 // t = e - d_i contiguous) and emit its warp's tau candidates.
 template <typename V, int W>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
-                                          V *lb, int32_t *tauc, int mq) {
+                                          V *lb, int32_t *tauc, int mq, int bx = -1) {
     const int d = P.len[i];
     const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
     const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
@@ -715,7 +716,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     }
     if (P.E <= 0) return;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const int unit = blockIdx.x * nw + warp;  // tau units are warps
+    const int unit = (bx >= 0 ? bx : (int)blockIdx.x) * nw + warp;  // tau units are warps of tile bx
     int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)unit * P.E;
     // The E smallest (LB_w, t) keys of the warp with 32-bit compares only: t
     // grows with the slot b inside a thread and with the lane across the warp,
@@ -1076,7 +1077,8 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
 // (A = 16 bytes / entry) and, through a second tensor map, a w x A tail box
 // at ca + 256; columns < 0 or
 // >= n_dw arrive zero-filled.  Both land in a 4-stage shared-memory ring armed
-// with mbarriers; thread x then reads column x + (Rb - j - ca) of each row
+// with mbarriers (persistent CTAs: the ring runs ahead across tiles); thread x
+// then reads column x + (Rb - j - ca) of each row
 // (from the main box, or the tail for the last few threads) -- conflict-free
 // 2- or 4-byte loads, no per-element address arithmetic, whole 512-byte rows
 // per request.  Sums, emission and the tau set are group_scan_reg's.
@@ -1124,10 +1126,29 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
         : "memory");
 }
 
+// One CSG row of the TMA scan for one thread's column: the W P_EQ entries at
+// pe[b RS] and the W P_EC entries at pe[PS + b RS]; all 2W loads first, then the
+// adds (rows b >= nrow, only in the last CSG row, add zero).
+template <typename V, typename PV, int W, int RS, int PS, bool FULL>
+__device__ __forceinline__ void tma_row_add(const PV *pe, int nrow, V (&se)[W], V (&sc)[W]) {
+    PV ve[W], vc[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) {
+        ve[b] = pe[b * RS];
+        vc[b] = pe[PS + b * RS];
+    }
+#pragma unroll
+    for (int b = 0; b < W; b++) {
+        const V e = post_cv<V>(ve[b]), c = post_cv<V>(vc[b]);
+        se[b] += (FULL || b < nrow) ? e : (V)0;
+        sc[b] += (FULL || b < nrow) ? c : (V)0;
+    }
+}
+
 template <typename S, int W, typename PV>
 __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tma_kernel(
     const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_tail, const MQMeta *meta,
-    const QParams P, typename Tr<S>::V *lb, int32_t *tauc) {
+    const QParams P, typename Tr<S>::V *lb, int32_t *tauc, int nb, int n_mq, int row0, int prows) {
     using V = typename Tr<S>::V;
     constexpr int NT = kScanThreads;
     constexpr int A = tma_align_elems<PV>();      // TMA start-column granule (16 bytes)
@@ -1143,30 +1164,33 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
     const int nl = P.n_len;
     const int n_sw = D - W + 1;
     const int mmax = D / W;
-    const int mq = blockIdx.y;
-    const MQMeta m = meta[mq];
-    if ((int)blockIdx.x >= m.nblk) {
-        tau_clear(P, mq, NT / 32, 0, P.n_len, tauc);
-        return;
-    }
     const int x = threadIdx.x;
-    const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
-    const int64_t r = Rb + x;
-    const int64_t s0 = (r + 1) * W;  // e of slot b = 0
-    const int row_base = (int)(m.post_off / m.pstride);  // tensor row of this stream's P_EQ row 0
-    auto issue = [&](int j) {         // CSG row j -> stage j % kTmaStages
+    // Persistent: this CTA scans tiles blockIdx.x, blockIdx.x + gridDim.x, ...
+    // (tile = mq * nb + bx); CSG rows are numbered g = k mmax + j over the CTA's
+    // k-th tile, and the TMA ring runs ahead across tile boundaries, so the next
+    // tile's rows stream in while this one emits.
+    const int ntiles = n_mq * nb;
+    const int my_tiles = (int)blockIdx.x < ntiles ? (ntiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+    const int64_t g_end = (int64_t)my_tiles * mmax;
+    auto issue = [&](int64_t g) {  // global row g -> stage g % kTmaStages
+        const int k = (int)(g / mmax), j = (int)(g - (int64_t)k * mmax);
+        const int tile = (int)blockIdx.x + k * (int)gridDim.x;
+        const int mq = tile / nb, bx = tile - mq * nb;
+        // tensor row of this stream's P_EQ row 0: the streams' rings are
+        // consecutive [2][prows] row blocks (no memory access on the issue path)
+        const int row_base = row0 + mq * 2 * prows;
         int pr = j * W + P.ring_cursor;
         pr -= pr >= n_sw ? n_sw : 0;
         pr -= pr >= n_sw ? n_sw : 0;
-        const int st = j % kTmaStages;
+        const int st = (int)(g % kTmaStages);
         mbar_expect_tx(&s_full[st], STAGE_BYTES);
-        const int col = (int)(Rb - j);
+        const int col = bx * NT - 1 - j;
         const int ca = col - (((col % A) + A) % A);  // floor to the 16-byte granule
         PV *sb = s_ring + (size_t)st * STAGE;
         tma_load_2d(sb, &tmap, ca, row_base + pr, &s_full[st]);
-        tma_load_2d(sb + W * NT, &tmap, ca, row_base + m.prows + pr, &s_full[st]);
+        tma_load_2d(sb + W * NT, &tmap, ca, row_base + prows + pr, &s_full[st]);
         tma_load_2d(sb + 2 * W * NT, &tmap_tail, ca + NT, row_base + pr, &s_full[st]);
-        tma_load_2d(sb + 2 * W * NT + TP, &tmap_tail, ca + NT, row_base + m.prows + pr, &s_full[st]);
+        tma_load_2d(sb + 2 * W * NT + TP, &tmap_tail, ca + NT, row_base + prows + pr, &s_full[st]);
     };
     if (x == 0) {
         for (int st = 0; st < kTmaStages; st++) mbar_init(&s_full[st], 1);
@@ -1174,60 +1198,71 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
     }
     __syncthreads();
     if (x == 0)
-        for (int j = 0; j < kTmaStages && j < mmax; j++) issue(j);
-    V se[W], sc[W];
-#pragma unroll
-    for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
+        for (int64_t g = 0; g < kTmaStages && g < g_end; g++) issue(g);
     uint64_t emit_rows = 0, save_rows = 0;
     for (int i = 0; i < nl; i++) {
         const int qi = P.len[i] / W;
         if (qi >= 1) emit_rows |= 1ull << (qi - 1);
         if (qi >= 2) save_rows |= 1ull << (qi - 2);
     }
-    if (nl > 0 && P.len[0] < W) {
-        V z[W];
+    int64_t g = 0;
+    for (int k = 0; k < my_tiles; k++) {
+        const int tile = (int)blockIdx.x + k * (int)gridDim.x;
+        const int mq = tile / nb, bx = tile - mq * nb;
+        // first used at the first emission row: the load overlaps the row loop
+        const MQMeta m = meta[mq];
+        const int64_t Rb = (int64_t)bx * NT - 1;
+        const int64_t r = Rb + x;
+        const int64_t s0 = (r + 1) * W;  // e of slot b = 0
+        V se[W], sc[W];
 #pragma unroll
-        for (int b = 0; b < W; b++) z[b] = (V)0;
-        for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq);
-    }
-    for (int j = 0; j < mmax; j++) {
-        const int st = j % kTmaStages;
-        mbar_wait(&s_full[st], (uint32_t)(j / kTmaStages) & 1u);
-        const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
-        const int col = (int)(Rb - j);
-        const int xo = x + (((col % A) + A) % A);  // this thread's column within the aligned boxes
-        const PV *sb = s_ring + (size_t)st * STAGE;
-        const bool main_box = xo < NT;
-        const PV *pe = main_box ? sb + xo : sb + 2 * W * NT + (xo - NT);
-        const int rs = main_box ? NT : A;       // row pitch of the box the column lies in
-        const int ps = main_box ? W * NT : TP;  // offset of the P_EC box
-#pragma unroll
-        for (int b = 0; b < W; b++) {
-            if (b < nrow) {
-                se[b] += post_cv<V>(pe[b * rs]);
-                sc[b] += post_cv<V>(pe[ps + b * rs]);
+        for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
+        for (int j = 0; j < mmax; j++, g++) {
+            const int st = (int)(g % kTmaStages);
+            mbar_wait(&s_full[st], (uint32_t)(g / kTmaStages) & 1u);
+            const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
+            const int col = (int)(Rb - j);
+            const int xo = x + (((col % A) + A) % A);  // this thread's column within the aligned boxes
+            const PV *sb = s_ring + (size_t)st * STAGE;
+            // main-box columns (all but at most A-1 threads of the last warp) use
+            // compile-time row pitches, so the 2W loads take immediate offsets
+            if (xo < NT) {
+                if (nrow >= W) tma_row_add<V, PV, W, NT, W * NT, true>(sb + xo, nrow, se, sc);
+                else tma_row_add<V, PV, W, NT, W * NT, false>(sb + xo, nrow, se, sc);
+            } else {
+                tma_row_add<V, PV, W, A, TP, false>(sb + 2 * W * NT + (xo - NT), nrow, se, sc);
             }
-        }
-        __syncthreads();  // every thread has read stage st
-        if (x == 0 && j + kTmaStages < mmax) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            issue(j + kTmaStages);
-        }
-        if (emit_rows >> j & 1ull) {
-            for (int i = 0; i < nl; i++) {
-                const int qi = P.len[i] / W, ri = P.len[i] % W;
-                if (j == qi - 1) {
-                    V v[W];
+            __syncthreads();  // every thread has read stage st
+            if (x == 0 && g + kTmaStages < g_end) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                issue(g + kTmaStages);
+            }
+            const bool live = bx < m.nblk;  // grids are sized for the longest sensor of the chunk
+            if (!live) continue;
+            if (emit_rows >> j & 1ull) {
+                for (int i = 0; i < nl; i++) {
+                    const int qi = P.len[i] / W, ri = P.len[i] % W;
+                    if (j == qi - 1) {
+                        V v[W];
 #pragma unroll
-                    for (int b = 0; b < W; b++)
-                        v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
-                    diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
+                        for (int b = 0; b < W; b++)
+                            v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
+                        diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq, bx);
+                    }
                 }
             }
-        }
-        if (save_rows >> j & 1ull) {
+            if (save_rows >> j & 1ull) {
 #pragma unroll
-            for (int b = 0; b < W; b++) s_saved[b][x] = lbpick(P, se[b], sc[b]);
+                for (int b = 0; b < W; b++) s_saved[b][x] = lbpick(P, se[b], sc[b]);
+            }
+        }
+        if (bx >= m.nblk) {
+            tau_clear(P, mq, NT / 32, 0, P.n_len, tauc, bx);
+        } else if (nl > 0 && P.len[0] < W) {  // IQs shorter than W: no full DW (R6), LB_w = 0
+            V z[W];
+#pragma unroll
+            for (int b = 0; b < W; b++) z[b] = (V)0;
+            for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq, bx);
         }
     }
 }

@@ -1027,10 +1027,18 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             bool done4 = false;
             if (sctx && sctx->tma) {  // TMA-staged ring scan
                 done4 = true;
-                auto go5 = [&](auto kern, size_t smem) {
+                auto go5 = [&](auto kern, size_t smem) {  // persistent: ~ one wave of CTAs over B x nblk tiles
                     set_smem((const void *)kern, smem);
-                    kern<<<grid, kScanThreads, smem, idx->stream>>>(*sctx->tmap, *sctx->tmap_tail, d_meta, P, idx->lb.as<V>(),
-                                                                    idx->tauc.as<int32_t>());
+                    int occ = 0;
+                    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kScanThreads, smem);
+                    const int64_t tiles = (int64_t)nblk_max * B;
+                    // opts.reserved[0] == 8: one tile per CTA (A/B against the persistent grid)
+                    const int g5 = o.reserved[0] == 8 ? (int)tiles
+                                   : (int)std::min<int64_t>(tiles, (int64_t)idx->num_sms * std::max(occ, 1));
+                    kern<<<g5, kScanThreads, smem, idx->stream>>>(*sctx->tmap, *sctx->tmap_tail, d_meta, P,
+                                                                  idx->lb.as<V>(), idx->tauc.as<int32_t>(),
+                                                                  nblk_max, B, (int)(sctx->ring_off[c0] / sctx->pstride),
+                                                                  sctx->prows);
                 };
                 if constexpr (std::is_same<S, float>::value) {
                     if (sctx->post_half) {
