@@ -244,6 +244,9 @@ class Runner:
         ab = int(os.environ.get("SMILER_AB", "0"))
         self.op.reserved[0] = ab
         self.op_fast.reserved[0] = ab
+        keep = int(os.environ.get("SMILER_TAU_KEEP", "0"))   # reserved[2]: tau-set trim multiple (A/B)
+        self.op.reserved[2] = keep
+        self.op_fast.reserved[2] = keep
         # C5 is a continuous prediction stream: every step is one tick of all
         # streams (each MQ advances one point); after the first tick the previous
         # tick's neighbours seed the thresholds (smiler_knn_step)

@@ -92,13 +92,15 @@ typedef struct smiler_knn_opts {
                          lower bound of DTW (Thm 4.3) and the kNN is unchanged, while the
                          ring and the bytes the group scan reads per step halve */
     int32_t tau_mult; /* size of the tile tau set (reading R8), in multiples of k per item
-                         query: 0 = default (16 one-shot, 0 in continuous steps, whose
-                         thresholds come from the previous step's neighbours),
+                         query: 0 = default (16 one-shot; 2 in continuous steps, which also
+                         verify the previous step's k neighbours shifted),
                          > 0 = that many, < 0 = none.  With no tile set in a continuous
                          step the thresholds exist before the scan, and the LB kernel
                          filters as it goes (a4+a6 fused, no LB_w array) */
     int32_t reserved[3];  /* 0; reserved[0] selects internal A/B variants in experiments (7: stream
-                             ring without TMA, 8: one tile per group-scan CTA) */
+                             ring without TMA, 8: one tile per group-scan CTA, 9: radix-select tau-set trim); reserved[2]: tau-set trim
+                             (kept tile candidates per item query, in multiples of k; 0 = default
+                             8 one-shot / 1 continuous, < 0 = verify every tile candidate) */
     uint64_t *shared_tau; /* NULL, or a running threshold shared by calls that split ONE
                          search (window-range shards of the same series and master
                          queries): [n_mq][n_len] keys

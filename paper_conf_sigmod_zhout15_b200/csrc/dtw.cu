@@ -77,8 +77,11 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
     }
 }
 
+#ifndef SMILER_DTW_MINB_WIDE
+#define SMILER_DTW_MINB_WIDE 1  // CTAs per SM the compiler must fit for rho > 12 (register cap)
+#endif
 template <typename S, int RHO>
-__global__ void __launch_bounds__(kDtwThreads) dtw_kernel(const DtwParams<S> p) {
+__global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE : 1)) dtw_kernel(const DtwParams<S> p) {
     using V = typename Tr<S>::V;
     constexpr int W = 2 * RHO + 1;
     constexpr bool IS_F = std::is_same<S, float>::value;
@@ -109,7 +112,7 @@ __global__ void __launch_bounds__(kDtwThreads) dtw_kernel(const DtwParams<S> p) 
         int cnt;
         int64_t lbase;
         if (p.mode == 0) {
-            cnt = p.LT;
+            cnt = p.LTc;
             lbase = (int64_t)seg * p.LT;
         } else {
             cnt = p.counts[seg];

@@ -14,6 +14,7 @@ constexpr int kMaxK = 1024;      // max k
 constexpr int kMaxWindow = 64;   // max omega
 constexpr int kMaxRhoFast = 32;  // rho handled by the register-band DTW kernels
 constexpr int kSortCap = 4096;   // keys sorted in shared memory by one CTA
+constexpr int kTrimBigCap = 55296;  // tau-set trim: 32-bit keys in shared memory (216 KB)
 constexpr int kMaxPredK = 128;   // neighbours per GP predictor (k x k fp64 factor in shared memory)
 constexpr uint64_t kKeyMax = ~0ull;
 
@@ -73,6 +74,7 @@ template <typename S> struct DtwParams {
     int mode;                     // 0 = tau list -> keys_out; 1 = survivors -> finalists
     const int32_t *list;          // candidate t values
     int LT;                       // tau mode: list stride per segment
+    int LTc;                      // tau mode: entries per segment to verify (<= LT)
     const int32_t *counts;        // survivors mode: per-segment counts
     const int32_t *task_off;      // [n_mq + 1] prefix of warp tasks
     uint64_t *keys_out;           // tau mode

@@ -250,15 +250,16 @@ template <typename V> __device__ __forceinline__ uint32_t thr_from_key(uint64_t 
 }
 
 template <typename S>
-__global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, int LT, int k,
+__global__ void __launch_bounds__(256) tau_select_kernel(const uint64_t *tauk, int LTs, int LT, int k,
                                                         uint64_t *tau_key, uint32_t *thr) {
+    // LTs: list stride per segment; LT: entries in use (the verified tau list)
     using V = typename Tr<S>::V;
     __shared__ int s_hist[256];
     __shared__ uint64_t s_b[2];
     __shared__ uint64_t s_keys[kSortCap];
     __shared__ int s_scan[32];
     const int seg = blockIdx.x;
-    const uint64_t *src = tauk + (int64_t)seg * LT;
+    const uint64_t *src = tauk + (int64_t)seg * LTs;
     uint64_t kth;
     if (LT <= kSortCap) {
         // sort, then the k-th DISTINCT key: the tau list may hold a candidate twice
@@ -518,6 +519,138 @@ __global__ void __launch_bounds__(512) merge_topk_kernel(const int64_t *ids_in, 
             const uint32_t db = (uint32_t)(key >> 32);
             d_out[o] = *reinterpret_cast<const V *>(&db);
         }
+    }
+}
+
+// a5 tau-set trim (reading R8): of the LTt tile candidates of a segment (each
+// scan unit's smallest-LB_w candidates), keep the `keep` smallest (LB_w, t) and
+// move the previous step's k neighbours (continuous step, at [LTt, LTt + kprev))
+// right after them, so the tau DTW pass verifies keep + kprev candidates.  Any
+// subset of verified candidates gives a valid tau (the k-th distinct key of k
+// verified candidates bounds the k-th NN key); the trim only trades a slightly
+// looser tau for fewer DTWs.  One CTA per segment; keys sorted in dynamic
+// shared memory (n2 = next power of two >= LTt).
+template <typename S>
+__global__ void __launch_bounds__(256) tau_trim_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
+                                                      const typename Tr<S>::V *lb, const MQMeta *meta,
+                                                      int n_len) {
+    extern __shared__ __align__(16) uint64_t s_tk[];
+    const int seg = blockIdx.x;
+    const int mq = seg / n_len, i = seg % n_len;
+    const MQMeta m = meta[mq];
+    int32_t *row = tauc + (int64_t)seg * LT;
+    const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
+    int n2 = 1;
+    while (n2 < LTt) n2 <<= 1;
+    for (int x = threadIdx.x; x < n2; x += blockDim.x) {
+        uint64_t key = kKeyMax;
+        if (x < LTt) {
+            const int t = row[x];
+            if (t >= 0) key = ((uint64_t)key_bits(lbi[t]) << 32) | (uint32_t)t;
+        }
+        s_tk[x] = key;
+    }
+    int32_t *s_prev = reinterpret_cast<int32_t *>(s_tk + n2);
+    for (int j = threadIdx.x; j < kprev; j += blockDim.x) s_prev[j] = row[LTt + j];
+    bitonic_sort_smem(s_tk, n2);  // ends with a barrier
+    for (int x = threadIdx.x; x < keep; x += blockDim.x)
+        row[x] = s_tk[x] != kKeyMax ? (int32_t)(uint32_t)s_tk[x] : -1;
+    for (int j = threadIdx.x; j < kprev; j += blockDim.x) row[keep + j] = s_prev[j];
+}
+
+// tau_trim_kernel for tile lists too long for a 64-bit key sort (window-range
+// scale, C4: ~49k per item query): only the 32-bit LB_w bits are kept in shared
+// memory (<= kTrimBigCap entries), the keep-th smallest is radix-selected (four
+// 8-bit MSB passes over shared memory), and the candidates below it, then those
+// equal to it up to `keep`, are compacted to the front in any order (any subset
+// of verified candidates gives a valid tau).
+template <typename S>
+__global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
+                                                          const typename Tr<S>::V *lb, const MQMeta *meta,
+                                                          int n_len) {
+    extern __shared__ __align__(16) uint32_t s_lbk[];
+    __shared__ int s_hist[256];
+    __shared__ uint32_t s_sel[2];
+    __shared__ int s_cnt;
+    const int seg = blockIdx.x;
+    const int mq = seg / n_len, i = seg % n_len;
+    const MQMeta m = meta[mq];
+    int32_t *row = tauc + (int64_t)seg * LT;
+    const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
+    for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
+        const int t = row[x];
+        s_lbk[x] = t >= 0 ? key_bits(lbi[t]) : 0xFFFFFFFFu;
+    }
+    // keep-th smallest valid value (MSB radix select over shared memory)
+    uint32_t prefix = 0, mask = 0;
+    int krem = keep;
+    bool few = false;
+    for (int shift = 24; shift >= 0; shift -= 8) {
+        for (int h = threadIdx.x; h < 256; h += blockDim.x) s_hist[h] = 0;
+        __syncthreads();
+        for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
+            const uint32_t v = s_lbk[x];
+            if (v != 0xFFFFFFFFu && (v & mask) == prefix) atomicAdd(&s_hist[(v >> shift) & 255], 1);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int acc = 0, dsel = -1;
+            for (int dg = 0; dg < 256; dg++) {
+                if (acc + s_hist[dg] >= krem) {
+                    dsel = dg;
+                    break;
+                }
+                acc += s_hist[dg];
+            }
+            s_sel[0] = dsel < 0 ? 0xFFFFFFFFu : (prefix | ((uint32_t)dsel << shift));
+            s_sel[1] = (uint32_t)(krem - acc);
+        }
+        __syncthreads();
+        if (s_sel[0] == 0xFFFFFFFFu) {  // fewer than keep valid candidates: keep them all
+            few = true;
+            break;
+        }
+        prefix = s_sel[0];
+        krem = (int)s_sel[1];
+        mask |= 255u << shift;
+        __syncthreads();
+    }
+    const uint32_t thr = few ? 0xFFFFFFFEu : prefix;
+    // previous neighbours [LTt, LTt + kprev) -> [keep, keep + kprev): read them first
+    int32_t pv[2];  // kprev <= 2 * 512 = kMaxK
+#pragma unroll
+    for (int r = 0; r < 2; r++) {
+        const int j = threadIdx.x + r * 512;
+        pv[r] = j < kprev ? row[LTt + j] : -1;
+    }
+    int32_t tl[kTrimBigCap / 512];  // this thread's tile t values (row is rewritten below)
+#pragma unroll
+    for (int r = 0; r < kTrimBigCap / 512; r++) {
+        const int x = threadIdx.x + r * 512;
+        tl[r] = x < LTt ? row[x] : -1;
+    }
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kTrimBigCap / 512; r++) {
+        const int x = threadIdx.x + r * 512;
+        if (x < LTt && s_lbk[x] < thr) row[atomicAdd(&s_cnt, 1)] = tl[r];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kTrimBigCap / 512; r++) {
+        const int x = threadIdx.x + r * 512;
+        if (x < LTt && s_lbk[x] == thr && s_lbk[x] != 0xFFFFFFFFu) {
+            const int o = atomicAdd(&s_cnt, 1);
+            if (o < keep) row[o] = tl[r];
+        }
+    }
+    __syncthreads();
+    for (int x = min(s_cnt, keep) + threadIdx.x; x < keep; x += blockDim.x) row[x] = -1;
+#pragma unroll
+    for (int r = 0; r < 2; r++) {
+        const int j = threadIdx.x + r * 512;
+        if (j < kprev) row[keep + j] = pv[r];
     }
 }
 

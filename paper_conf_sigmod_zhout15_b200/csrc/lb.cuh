@@ -22,6 +22,14 @@
 #pragma once
 // (included inside namespace smiler by kernels.cuh)
 
+// Build-time A/B switches (tools/build_variants.sh)
+#ifndef SMILER_LB_FOLD
+#define SMILER_LB_FOLD 1
+#endif
+#ifndef SMILER_DIAG_UNROLL2
+#define SMILER_DIAG_UNROLL2 0
+#endif
+
 // The bound of a candidate from its EQ and EC sums: LB = max(EQ, EC) (Eq. 5,
 // Thm 4.1), or one of the two sums alone (the Table 3 ablation).
 template <typename V> __device__ __forceinline__ V lbpick(const QParams &P, V eq, V ec) {
@@ -203,6 +211,25 @@ __device__ __forceinline__ void posting_chunk_w(const V (&c)[W], const V (&U)[W]
                 lb_term(wq[k], U[j], L[j], ec);
             }
             store(bb, eq, ec);
+        }
+    }
+}
+
+// posting_chunk_w with the terms accumulated straight into the running CSG
+// sums (se/sc slot bb): LB_w is the same sum of the same terms (Eq. 5 summed
+// over the CSG's postings), one add per posting element shorter.  f32 rounding
+// differs only in association; the filter's slack covers any order (R16).
+template <typename V, int W, int BC, int WL, int NS>
+__device__ __forceinline__ void posting_chunk_w_fold(const V (&c)[W], const V (&U)[W], const V (&L)[W],
+                                                     const V (&wq)[WL], const V (&wu)[WL], const V (&wl)[WL],
+                                                     V (&se)[NS], V (&sc)[NS]) {
+#pragma unroll
+    for (int bb = 0; bb < BC; bb++) {
+#pragma unroll
+        for (int j = 0; j < W; j++) {
+            const int k = BC - 1 - bb + j;
+            lb_term(c[j], wu[k], wl[k], se[bb]);
+            lb_term(wq[k], U[j], L[j], sc[bb]);
         }
     }
 }
@@ -848,6 +875,9 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
     // IQs shorter than W have no full DW anywhere (m = 0, R6): LB_w = 0
     for (int i = 0; i < nl && P.len[i] < W; i++)
         if (P.k >= 0) diag_emit<V, W>(saved, i, s0, m, P, lb, tauc, mq);
+#if SMILER_DIAG_UNROLL2
+#pragma unroll 2
+#endif
     for (int j = 0; j < mmax; j++) {
         const int col = x + HALO - j;  // DW r - j
         V c[W], U[W], L[W];
@@ -888,7 +918,11 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                     wu[k] = u.x, wu[k + 1] = u.y, wu[k + 2] = u.z, wu[k + 3] = u.w;
                     wl[k] = l.x, wl[k + 1] = l.y, wl[k + 2] = l.z, wl[k + 3] = l.w;
                 }
+#if SMILER_LB_FOLD
+                posting_chunk_w_fold<V, W, BC, WL, W>(c, U, L, wq, wu, wl, se, sc);
+#else
                 posting_chunk_w<V, W, BC, false, WL>(c, U, L, wq, wu, wl, BC, acc);
+#endif
             } else if (nv > 0) {
                 posting_chunk<V, W, BC, true>(c, U, L, sqq + qshift, squ + qshift, sql + qshift, pb, nv, acc);
             }

@@ -29,6 +29,18 @@ using namespace smiler;
 
 constexpr int kTauMult = 16;  // tau-set size target, multiples of k (R8 reading)
 constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previous neighbours)
+// Tile tau-set trim (tau_trim_kernel): keep the kTauKeep* x k smallest-LB_w tile
+// candidates of the scan units' picks (0 = verify them all).  smiler_knn_opts
+// .reserved[2] > 0 overrides the multiple (A/B experiments), < 0 disables.
+constexpr int kTauKeepOneShot = 8;
+constexpr int kTauKeepCont = 1;
+constexpr int kTrimCap = 16384;  // longer tile lists are trimmed by radix select (tau_trim_big_kernel)
+static int tau_keep(const smiler_knn_opts &o, int k, bool cont) {
+    int mult = cont ? kTauKeepCont : kTauKeepOneShot;
+    if (o.reserved[2] > 0) mult = o.reserved[2];
+    if (o.reserved[2] < 0) mult = 0;
+    return mult * k;
+}
 constexpr int kTauEMax = 8;   // candidates per tau unit (CTA or warp)
 
 // ---------------------------------------------------------------------------
@@ -523,9 +535,10 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
                         const int32_t *list, int LT, const int32_t *counts, int32_t *task_off,
                         uint64_t *keys_out, const uint64_t *tau_key, uint64_t *fin,
                         int32_t *fin_count, const MQMeta *d_meta, const typename Tr<S>::V *qv,
-                        int D, cudaStream_t st = nullptr) {
+                        int D, cudaStream_t st = nullptr, int LTc = -1) {
     if (!st) st = idx->stream;
-    task_prefix_kernel<<<1, 1024, 0, st>>>(counts, mode == 0 ? LT : -1, n_mq, pl.n_len, li, task_off);
+    if (LTc < 0) LTc = LT;  // tau mode: verify the first LTc entries of each stride-LT list
+    task_prefix_kernel<<<1, 1024, 0, st>>>(counts, mode == 0 ? LTc : -1, n_mq, pl.n_len, li, task_off);
     CHECK_LAUNCH();
     DtwParams<S> p;
     p.series = (const S *)idx->d_series;
@@ -539,6 +552,7 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
     p.mode = mode;
     p.list = list;
     p.LT = LT;
+    p.LTc = LTc;
     p.counts = counts;
     p.task_off = task_off;
     p.keys_out = keys_out;
@@ -848,17 +862,40 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 launches++;
             }
             if (!o.no_prune) {
+                // trim the tile tau set to its `keep` smallest-LB_w candidates
+                int LTc = LT;
+                const int keep = tau_keep(o, pl.k, use_prev);
+                if (keep > 0 && LTt > keep && LTt <= kTrimBigCap) {
+                    if (LTt <= kTrimCap && o.reserved[0] != 9) {  // reserved[0] == 9: test the radix path
+                        int n2 = 1;
+                        while (n2 < LTt) n2 <<= 1;
+                        const size_t sm = (size_t)8 * n2 + (size_t)4 * (use_prev ? pl.k : 0);
+                        set_smem((const void *)tau_trim_kernel<S>, sm);
+                        tau_trim_kernel<S><<<nseg, 256, sm, idx->stream>>>(idx->tauc.as<int32_t>(), LT, LTt, keep,
+                                                                           use_prev ? pl.k : 0, idx->lb.as<V>(),
+                                                                           d_meta, nl);
+                    } else {  // 32-bit LB keys, radix select in shared memory
+                        const size_t sm = (size_t)4 * LTt;
+                        set_smem((const void *)tau_trim_big_kernel<S>, sm);
+                        tau_trim_big_kernel<S><<<nseg, 512, sm, idx->stream>>>(
+                            idx->tauc.as<int32_t>(), LT, LTt, keep, use_prev ? pl.k : 0, idx->lb.as<V>(), d_meta, nl);
+                    }
+                    CHECK_LAUNCH();
+                    launches++;
+                    LTc = keep + (use_prev ? pl.k : 0);
+                }
                 TRY(side_fork(idx, nl));
                 for (int i = 0; i < nl; i++) {
                     TRY(run_dtw_list<S>(idx, pl, i, B, 0, idx->tauc.as<int32_t>(), LT, nullptr,
                                         taskoff + (size_t)i * (B + 1), idx->tauk.as<uint64_t>(), nullptr,
-                                        nullptr, nullptr, d_meta, idx->qv.as<V>(), D, idx->side[i]));
+                                        nullptr, nullptr, d_meta, idx->qv.as<V>(), D, idx->side[i], LTc));
                     launches += 2;
-                    tau_slots_total += (int64_t)B * LT;
-                    cells_acc += (double)B * LT * (double)dtw_cells(pl.len[i], pl.rho[i]);
+                    tau_slots_total += (int64_t)B * LTc;
+                    cells_acc += (double)B * LTc * (double)dtw_cells(pl.len[i], pl.rho[i]);
                 }
                 TRY(side_join(idx, nl));
-                tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, pl.k, taukey, thr);
+                tau_select_kernel<S><<<nseg, 256, 0, idx->stream>>>(idx->tauk.as<uint64_t>(), LT, LTc, pl.k, taukey,
+                                                                    thr);
                 CHECK_LAUNCH();
                 launches++;
                 if (o.shared_tau) {  // NEXT-2: running threshold shared across the shards

@@ -337,7 +337,7 @@ class Index:
 
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
             no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False,
-            lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0):
+            lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0, reserved=None):
         """kNN of every item query (smiler_knn_ex).  shared_tau: optional device
         buffer (torch int64 tensor of n_mq * n_len entries, all ones = -1 at start)
         shared by the window-range shards of one search (NEXT-2)."""
@@ -348,6 +348,9 @@ class Index:
         op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level),
                      lb_kind=int(lb_kind), horizon=int(horizon), tau_mult=int(tau_mult),
                      shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
+        if reserved is not None:   # experiment / test switches (include/smiler.h)
+            for j, v in enumerate(reserved):
+                op.reserved[j] = int(v)
         smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()

@@ -193,6 +193,20 @@ def test_c4_reduced(pkg, orc, dtype):
     check_workload(pkg, orc, wl)
 
 
+# a5 tau-set trim (tau_trim_kernel / tau_trim_big_kernel): any kept subset of
+# verified candidates gives a valid tau, so the kNN must not change; keep = 1 x k
+# is the tightest trim, (9, 0, m) forces the radix-select path, -1 disables it
+@pytest.mark.parametrize("reserved", [(0, 0, 1), (9, 0, 1), (9, 0, 3), (0, 0, -1), (0, 0, 64)])
+@pytest.mark.parametrize("cfg,kw", [("C2", dict(n=20011, mq_per_sensor=4)),
+                                    ("C4", dict(n=60013, mq_per_sensor=2))])
+def test_tau_trim(pkg, orc, cfg, kw, reserved):
+    wl = synth.make_workload(cfg, "i16", **kw)
+    ids, dists, st = gpu_knn(pkg, wl, stats=True, reserved=reserved)
+    oid, od = orc.knn(wl, threads=THREADS)
+    np.testing.assert_array_equal(ids, oid)
+    np.testing.assert_array_equal(dists.astype(np.int64), od)
+
+
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
 def test_c5_reduced(pkg, orc, dtype):
     wl = synth.make_workload("C5", dtype, n=12001, n_sensors=4, mq_per_sensor=2, consecutive=True)
