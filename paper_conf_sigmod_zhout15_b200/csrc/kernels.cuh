@@ -530,8 +530,11 @@ __global__ void __launch_bounds__(512) merge_topk_kernel(const int64_t *ids_in, 
 // verified candidates bounds the k-th NN key); the trim only trades a slightly
 // looser tau for fewer DTWs.  One CTA per segment; keys sorted in dynamic
 // shared memory (n2 = next power of two >= LTt).
+// src: the candidate list of each segment (stride sstride, nsrc entries): the
+// tile list itself, or the per-chunk winners of tau_trim_chunk_kernel.
 template <typename S>
-__global__ void __launch_bounds__(256) tau_trim_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
+__global__ void __launch_bounds__(256) tau_trim_kernel(const int32_t *src, int sstride, int nsrc, int32_t *tauc,
+                                                      int LT, int LTt, int keep, int kprev,
                                                       const typename Tr<S>::V *lb, const MQMeta *meta,
                                                       int n_len) {
     extern __shared__ __align__(16) uint64_t s_tk[];
@@ -539,13 +542,14 @@ __global__ void __launch_bounds__(256) tau_trim_kernel(int32_t *tauc, int LT, in
     const int mq = seg / n_len, i = seg % n_len;
     const MQMeta m = meta[mq];
     int32_t *row = tauc + (int64_t)seg * LT;
+    const int32_t *srow = src + (int64_t)seg * sstride;
     const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
     int n2 = 1;
-    while (n2 < LTt) n2 <<= 1;
+    while (n2 < nsrc) n2 <<= 1;
     for (int x = threadIdx.x; x < n2; x += blockDim.x) {
         uint64_t key = kKeyMax;
-        if (x < LTt) {
-            const int t = row[x];
+        if (x < nsrc) {
+            const int t = srow[x];
             if (t >= 0) key = ((uint64_t)key_bits(lbi[t]) << 32) | (uint32_t)t;
         }
         s_tk[x] = key;
@@ -556,6 +560,37 @@ __global__ void __launch_bounds__(256) tau_trim_kernel(int32_t *tauc, int LT, in
     for (int x = threadIdx.x; x < keep; x += blockDim.x)
         row[x] = s_tk[x] != kKeyMax ? (int32_t)(uint32_t)s_tk[x] : -1;
     for (int j = threadIdx.x; j < kprev; j += blockDim.x) row[keep + j] = s_prev[j];
+}
+
+// First level of the trim for very long tile lists (window-range scale): chunk
+// c of segment seg (kTrimChunk entries) keeps its `keep` smallest (LB_w, t) in
+// out[seg][c keep ..); tau_trim_kernel then trims the chunk winners.
+constexpr int kTrimChunk = 8192;
+template <typename S>
+__global__ void __launch_bounds__(256) tau_trim_chunk_kernel(const int32_t *tauc, int LT, int LTt, int keep,
+                                                            const typename Tr<S>::V *lb, const MQMeta *meta,
+                                                            int n_len, int32_t *out, int ostride) {
+    extern __shared__ __align__(16) uint64_t s_tk[];
+    const int c = blockIdx.x, seg = blockIdx.y;
+    const int mq = seg / n_len, i = seg % n_len;
+    const MQMeta m = meta[mq];
+    const int32_t *row = tauc + (int64_t)seg * LT + (int64_t)c * kTrimChunk;
+    const int n = min(kTrimChunk, LTt - c * kTrimChunk);
+    const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
+    int n2 = 1;
+    while (n2 < n) n2 <<= 1;
+    for (int x = threadIdx.x; x < n2; x += blockDim.x) {
+        uint64_t key = kKeyMax;
+        if (x < n) {
+            const int t = row[x];
+            if (t >= 0) key = ((uint64_t)key_bits(lbi[t]) << 32) | (uint32_t)t;
+        }
+        s_tk[x] = key;
+    }
+    bitonic_sort_smem(s_tk, n2);
+    int32_t *o = out + (int64_t)seg * ostride + (int64_t)c * keep;
+    for (int x = threadIdx.x; x < keep; x += blockDim.x)
+        o[x] = x < n2 && s_tk[x] != kKeyMax ? (int32_t)(uint32_t)s_tk[x] : -1;
 }
 
 // tau_trim_kernel for tile lists too long for a 64-bit key sort (window-range

@@ -865,24 +865,42 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 // trim the tile tau set to its `keep` smallest-LB_w candidates
                 int LTc = LT;
                 const int keep = tau_keep(o, pl.k, use_prev);
-                if (keep > 0 && LTt > keep && LTt <= kTrimBigCap) {
-                    if (LTt <= kTrimCap && o.reserved[0] != 9) {  // reserved[0] == 9: test the radix path
+                const int kpv = use_prev ? pl.k : 0;
+                const int nch = (LTt + kTrimChunk - 1) / kTrimChunk;
+                const bool two_stage = keep > 0 && nch > 1 && (int64_t)nch * keep <= kTrimCap;
+                if (keep > 0 && LTt > keep && (LTt <= kTrimCap || two_stage || LTt <= kTrimBigCap)) {
+                    auto trim1 = [&](const int32_t *src, int sstride, int nsrc) {
                         int n2 = 1;
-                        while (n2 < LTt) n2 <<= 1;
-                        const size_t sm = (size_t)8 * n2 + (size_t)4 * (use_prev ? pl.k : 0);
+                        while (n2 < nsrc) n2 <<= 1;
+                        const size_t sm = (size_t)8 * n2 + (size_t)4 * kpv;
                         set_smem((const void *)tau_trim_kernel<S>, sm);
-                        tau_trim_kernel<S><<<nseg, 256, sm, idx->stream>>>(idx->tauc.as<int32_t>(), LT, LTt, keep,
-                                                                           use_prev ? pl.k : 0, idx->lb.as<V>(),
+                        tau_trim_kernel<S><<<nseg, 256, sm, idx->stream>>>(src, sstride, nsrc, idx->tauc.as<int32_t>(),
+                                                                           LT, LTt, keep, kpv, idx->lb.as<V>(),
                                                                            d_meta, nl);
+                    };
+                    if (LTt <= kTrimCap && o.reserved[0] != 9) {  // reserved[0] == 9: test the other paths
+                        trim1(idx->tauc.as<int32_t>(), LT, LTt);
+                    } else if (two_stage && (o.reserved[0] != 9 || LTt > kTrimBigCap || o.reserved[1] == 9)) {
+                        // chunk winners into the survivor buffer (unused until a6), then one more trim
+                        const int ostride = nch * keep;
+                        TRY(idx->surv.ensure(4 * (size_t)nseg * ostride));
+                        const size_t sm = (size_t)8 * kTrimChunk;
+                        set_smem((const void *)tau_trim_chunk_kernel<S>, sm);
+                        tau_trim_chunk_kernel<S><<<dim3(nch, nseg), 256, sm, idx->stream>>>(
+                            idx->tauc.as<int32_t>(), LT, LTt, keep, idx->lb.as<V>(), d_meta, nl,
+                            idx->surv.as<int32_t>(), ostride);
+                        CHECK_LAUNCH();
+                        launches++;
+                        trim1(idx->surv.as<int32_t>(), ostride, ostride);
                     } else {  // 32-bit LB keys, radix select in shared memory
                         const size_t sm = (size_t)4 * LTt;
                         set_smem((const void *)tau_trim_big_kernel<S>, sm);
                         tau_trim_big_kernel<S><<<nseg, 512, sm, idx->stream>>>(
-                            idx->tauc.as<int32_t>(), LT, LTt, keep, use_prev ? pl.k : 0, idx->lb.as<V>(), d_meta, nl);
+                            idx->tauc.as<int32_t>(), LT, LTt, keep, kpv, idx->lb.as<V>(), d_meta, nl);
                     }
                     CHECK_LAUNCH();
                     launches++;
-                    LTc = keep + (use_prev ? pl.k : 0);
+                    LTc = keep + kpv;
                 }
                 TRY(side_fork(idx, nl));
                 for (int i = 0; i < nl; i++) {

@@ -207,6 +207,18 @@ def test_tau_trim(pkg, orc, cfg, kw, reserved):
     np.testing.assert_array_equal(dists.astype(np.int64), od)
 
 
+# tile lists longer than one chunk (> 8192 scan units per item query): the
+# single bitonic trim (default), the two-stage chunked trim (9, 9, m) and the
+# shared-memory radix trim (9, 0, m)
+@pytest.mark.parametrize("reserved", [(0, 0, 0), (9, 9, 1), (9, 9, 4), (9, 0, 2)])
+def test_tau_trim_long_lists(pkg, orc, reserved):
+    wl = synth.make_workload("C2", "i16", n=2_200_003, mq_per_sensor=1, lengths=[16, 32])
+    ids, dists = gpu_knn(pkg, wl, reserved=reserved)
+    oid, od = orc.knn(wl, threads=THREADS)
+    np.testing.assert_array_equal(ids, oid)
+    np.testing.assert_array_equal(dists.astype(np.int64), od)
+
+
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
 def test_c5_reduced(pkg, orc, dtype):
     wl = synth.make_workload("C5", dtype, n=12001, n_sensors=4, mq_per_sensor=2, consecutive=True)
