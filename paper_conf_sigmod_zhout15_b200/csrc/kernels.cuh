@@ -623,9 +623,15 @@ __global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT
     for (int shift = 24; shift >= 0; shift -= 8) {
         for (int h = threadIdx.x; h < 256; h += blockDim.x) s_hist[h] = 0;
         __syncthreads();
-        for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
-            const uint32_t v = s_lbk[x];
-            if (v != 0xFFFFFFFFu && (v & mask) == prefix) atomicAdd(&s_hist[(v >> shift) & 255], 1);
+        // LB_w values share their top bits: aggregate equal digits per warp
+        // (one shared atomic per distinct digit) instead of one per element
+        for (int x0 = threadIdx.x & ~31; x0 < LTt; x0 += blockDim.x) {
+            const int x = x0 + (threadIdx.x & 31);
+            const uint32_t v = x < LTt ? s_lbk[x] : 0xFFFFFFFFu;
+            const bool in = v != 0xFFFFFFFFu && (v & mask) == prefix;
+            const int dg = in ? (int)((v >> shift) & 255) : 256;
+            const unsigned peers = __match_any_sync(0xffffffffu, dg);
+            if (in && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&s_hist[dg], __popc(peers));
         }
         __syncthreads();
         if (threadIdx.x == 0) {

@@ -29,6 +29,9 @@
 #ifndef SMILER_DIAG_UNROLL2
 #define SMILER_DIAG_UNROLL2 0
 #endif
+#ifndef SMILER_TMA_EMPTYBAR
+#define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower)
+#endif
 
 // The bound of a candidate from its EQ and EC sums: LB = max(EQ, EC) (Eq. 5,
 // Thm 4.1), or one of the two sums alone (the Table 3 ablation).
@@ -1141,6 +1144,9 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                  : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     asm volatile(
         "{\n"
@@ -1193,6 +1199,7 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
     // stage st: [plane 0 main W x NT][plane 1 main W x NT][plane 0 tail W x A][plane 1 tail W x A]
     PV *s_ring = reinterpret_cast<PV *>(tma_smem);
     __shared__ __align__(8) uint64_t s_full[kTmaStages];
+    __shared__ __align__(8) uint64_t s_empty[kTmaStages];  // SMILER_TMA_EMPTYBAR: one arrival per warp
     __shared__ V s_saved[W][NT];
     const int D = P.D;
     const int nl = P.n_len;
@@ -1227,7 +1234,10 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
         tma_load_2d(sb + 2 * W * NT + TP, &tmap_tail, ca + NT, row_base + prows + pr, &s_full[st]);
     };
     if (x == 0) {
-        for (int st = 0; st < kTmaStages; st++) mbar_init(&s_full[st], 1);
+        for (int st = 0; st < kTmaStages; st++) {
+            mbar_init(&s_full[st], 1);
+            mbar_init(&s_empty[st], NT / 32);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -1266,11 +1276,23 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
             } else {
                 tma_row_add<V, PV, W, A, TP, false>(sb + 2 * W * NT + (xo - NT), nrow, se, sc);
             }
+#if SMILER_TMA_EMPTYBAR
+            // each warp releases stage st once its reads are done; thread 0 alone
+            // waits for all of them before refilling it (no CTA-wide barrier)
+            __syncwarp();
+            if ((x & 31) == 0) mbar_arrive(&s_empty[st]);
+            if (x == 0 && g + kTmaStages < g_end) {
+                mbar_wait(&s_empty[st], (uint32_t)(g / kTmaStages) & 1u);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                issue(g + kTmaStages);
+            }
+#else
             __syncthreads();  // every thread has read stage st
             if (x == 0 && g + kTmaStages < g_end) {
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 issue(g + kTmaStages);
             }
+#endif
             const bool live = bx < m.nblk;  // grids are sized for the longest sensor of the chunk
             if (!live) continue;
             if (emit_rows >> j & 1ull) {

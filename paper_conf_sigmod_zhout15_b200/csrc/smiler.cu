@@ -34,7 +34,8 @@ constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previou
 // .reserved[2] > 0 overrides the multiple (A/B experiments), < 0 disables.
 constexpr int kTauKeepOneShot = 8;
 constexpr int kTauKeepCont = 1;
-constexpr int kTrimCap = 16384;  // longer tile lists are trimmed by radix select (tau_trim_big_kernel)
+constexpr int kTrimCap = 16384;   // chunk winners a second bitonic trim may take (two-stage)
+constexpr int kTrimSmall = 1024;  // tile lists sorted whole; longer: radix select (tau_trim_big_kernel)
 static int tau_keep(const smiler_knn_opts &o, int k, bool cont) {
     int mult = cont ? kTauKeepCont : kTauKeepOneShot;
     if (o.reserved[2] > 0) mult = o.reserved[2];
@@ -868,7 +869,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 const int kpv = use_prev ? pl.k : 0;
                 const int nch = (LTt + kTrimChunk - 1) / kTrimChunk;
                 const bool two_stage = keep > 0 && nch > 1 && (int64_t)nch * keep <= kTrimCap;
-                if (keep > 0 && LTt > keep && (LTt <= kTrimCap || two_stage || LTt <= kTrimBigCap)) {
+                if (keep > 0 && LTt > keep && (LTt <= kTrimBigCap || two_stage)) {
                     auto trim1 = [&](const int32_t *src, int sstride, int nsrc) {
                         int n2 = 1;
                         while (n2 < nsrc) n2 <<= 1;
@@ -878,9 +879,13 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                                                                            LT, LTt, keep, kpv, idx->lb.as<V>(),
                                                                            d_meta, nl);
                     };
-                    if (LTt <= kTrimCap && o.reserved[0] != 9) {  // reserved[0] == 9: test the other paths
+                    // <= kTrimSmall: one bitonic sort; <= kTrimBigCap: radix select in shared
+                    // memory; longer: two-stage (chunk bitonic sorts, then one more trim).
+                    // reserved[0] == 9 (tests): radix, or two-stage with reserved[1] == 9
+                    const bool test_alt = o.reserved[0] == 9;
+                    if (LTt <= kTrimSmall && !test_alt) {
                         trim1(idx->tauc.as<int32_t>(), LT, LTt);
-                    } else if (two_stage && (o.reserved[0] != 9 || LTt > kTrimBigCap || o.reserved[1] == 9)) {
+                    } else if (two_stage && (LTt > kTrimBigCap || (test_alt && o.reserved[1] == 9))) {
                         // chunk winners into the survivor buffer (unused until a6), then one more trim
                         const int ostride = nch * keep;
                         TRY(idx->surv.ensure(4 * (size_t)nseg * ostride));
