@@ -61,6 +61,7 @@ struct QParams {
     const uint32_t *thr;  // fuse: per-segment admission bound (tau_select_kernel)
     int32_t *surv;        // fuse: survivor t lists (segment layout)
     int32_t *scount;      // fuse: survivors per segment
+    uint32_t *taulb;      // LB_w bits of every tile tau candidate (same layout as the tau list), or null
     int len[kMaxLen];
     int rho[kMaxLen];
 };

@@ -536,13 +536,15 @@ template <typename S>
 __global__ void __launch_bounds__(256) tau_trim_kernel(const int32_t *src, int sstride, int nsrc, int32_t *tauc,
                                                       int LT, int LTt, int keep, int kprev,
                                                       const typename Tr<S>::V *lb, const MQMeta *meta,
-                                                      int n_len) {
+                                                      int n_len, const uint32_t *slb) {
+    // slb: LB_w bits beside src (same layout), or null: gather them from LB_w
     extern __shared__ __align__(16) uint64_t s_tk[];
     const int seg = blockIdx.x;
     const int mq = seg / n_len, i = seg % n_len;
     const MQMeta m = meta[mq];
     int32_t *row = tauc + (int64_t)seg * LT;
     const int32_t *srow = src + (int64_t)seg * sstride;
+    const uint32_t *slrow = slb ? slb + (int64_t)seg * sstride : nullptr;
     const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
     int n2 = 1;
     while (n2 < nsrc) n2 <<= 1;
@@ -550,7 +552,7 @@ __global__ void __launch_bounds__(256) tau_trim_kernel(const int32_t *src, int s
         uint64_t key = kKeyMax;
         if (x < nsrc) {
             const int t = srow[x];
-            if (t >= 0) key = ((uint64_t)key_bits(lbi[t]) << 32) | (uint32_t)t;
+            if (t >= 0) key = ((uint64_t)(slrow ? slrow[x] : key_bits(lbi[t])) << 32) | (uint32_t)t;
         }
         s_tk[x] = key;
     }
@@ -569,12 +571,14 @@ constexpr int kTrimChunk = 8192;
 template <typename S>
 __global__ void __launch_bounds__(256) tau_trim_chunk_kernel(const int32_t *tauc, int LT, int LTt, int keep,
                                                             const typename Tr<S>::V *lb, const MQMeta *meta,
-                                                            int n_len, int32_t *out, int ostride) {
+                                                            int n_len, int32_t *out, int ostride,
+                                                            const uint32_t *tlb, uint32_t *olb) {
     extern __shared__ __align__(16) uint64_t s_tk[];
     const int c = blockIdx.x, seg = blockIdx.y;
     const int mq = seg / n_len, i = seg % n_len;
     const MQMeta m = meta[mq];
     const int32_t *row = tauc + (int64_t)seg * LT + (int64_t)c * kTrimChunk;
+    const uint32_t *lrow = tlb ? tlb + (int64_t)seg * LT + (int64_t)c * kTrimChunk : nullptr;
     const int n = min(kTrimChunk, LTt - c * kTrimChunk);
     const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
     int n2 = 1;
@@ -583,14 +587,18 @@ __global__ void __launch_bounds__(256) tau_trim_chunk_kernel(const int32_t *tauc
         uint64_t key = kKeyMax;
         if (x < n) {
             const int t = row[x];
-            if (t >= 0) key = ((uint64_t)key_bits(lbi[t]) << 32) | (uint32_t)t;
+            if (t >= 0) key = ((uint64_t)(lrow ? lrow[x] : key_bits(lbi[t])) << 32) | (uint32_t)t;
         }
         s_tk[x] = key;
     }
     bitonic_sort_smem(s_tk, n2);
     int32_t *o = out + (int64_t)seg * ostride + (int64_t)c * keep;
-    for (int x = threadIdx.x; x < keep; x += blockDim.x)
-        o[x] = x < n2 && s_tk[x] != kKeyMax ? (int32_t)(uint32_t)s_tk[x] : -1;
+    uint32_t *ol = olb ? olb + (int64_t)seg * ostride + (int64_t)c * keep : nullptr;
+    for (int x = threadIdx.x; x < keep; x += blockDim.x) {
+        const bool ok = x < n2 && s_tk[x] != kKeyMax;
+        o[x] = ok ? (int32_t)(uint32_t)s_tk[x] : -1;
+        if (ol) ol[x] = ok ? (uint32_t)(s_tk[x] >> 32) : 0xFFFFFFFFu;
+    }
 }
 
 // tau_trim_kernel for tile lists too long for a 64-bit key sort (window-range
@@ -602,7 +610,7 @@ __global__ void __launch_bounds__(256) tau_trim_chunk_kernel(const int32_t *tauc
 template <typename S>
 __global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
                                                           const typename Tr<S>::V *lb, const MQMeta *meta,
-                                                          int n_len) {
+                                                          int n_len, const uint32_t *tlb) {
     extern __shared__ __align__(16) uint32_t s_lbk[];
     __shared__ int s_hist[256];
     __shared__ uint32_t s_sel[2];
@@ -612,9 +620,10 @@ __global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT
     const MQMeta m = meta[mq];
     int32_t *row = tauc + (int64_t)seg * LT;
     const typename Tr<S>::V *lbi = lb + m.seg_off + (int64_t)i * m.n;
+    const uint32_t *lrow = tlb ? tlb + (int64_t)seg * LT : nullptr;
     for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
         const int t = row[x];
-        s_lbk[x] = t >= 0 ? key_bits(lbi[t]) : 0xFFFFFFFFu;
+        s_lbk[x] = t >= 0 ? (lrow ? lrow[x] : key_bits(lbi[t])) : 0xFFFFFFFFu;
     }
     // keep-th smallest valid value (MSB radix select over shared memory)
     uint32_t prefix = 0, mask = 0;

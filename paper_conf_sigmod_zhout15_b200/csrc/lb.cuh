@@ -132,7 +132,10 @@ __device__ void lb_tile_epilogue(V *tile, int RT, int64_t e0, const MQMeta &m, c
                 uint32_t allones = 0xFFFFFFFFu;   // "taken": not a valid LB >= 0
                 row[bs] = *reinterpret_cast<V *>(&allones);
             }
-            if (threadIdx.x == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+            if (threadIdx.x == 0) {
+                dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+                if (P.taulb) P.taulb[dst - tauc + e] = (uint32_t)(win >> 32);
+            }
             __syncthreads();
         }
     }
@@ -194,7 +197,10 @@ __device__ void lb_tile_epilogue_warp(V *tile, int RT, int64_t e0, const MQMeta 
                 uint32_t allones = 0xFFFFFFFFu;
                 row[bs] = *reinterpret_cast<V *>(&allones);
             }
-            if (lane == 0) dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+            if (lane == 0) {
+                dst[e] = win != kKeyMax ? (int32_t)(uint32_t)win : -1;
+                if (P.taulb) P.taulb[dst - tauc + e] = (uint32_t)(win >> 32);
+            }
         }
     }
 }
@@ -776,7 +782,10 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
             for (int b = 0; b < W; b++)
                 if (b == bs) kb[b] = 0xFFFFFFFFu;
         }
-        if (lane == 0) dst[e] = win != 0xFFFFFFFFu ? tw : -1;
+        if (lane == 0) {
+            dst[e] = win != 0xFFFFFFFFu ? tw : -1;
+            if (P.taulb) P.taulb[dst - tauc + e] = win;  // the trim reads the bound here, not from LB_w
+        }
     }
 }
 

@@ -141,7 +141,7 @@ struct smiler_index {
     std::map<int, std::pair<void *, void *>> env;  // rho -> (U, L)
     int num_sms = 148;
     // workspace
-    DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, tauk, taukey, thr, scount, fcount,
+    DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, taulb, tauk, taukey, thr, scount, fcount,
         taskoff, out_ids, out_d, tmp, tmp2, pred;
     std::vector<cudaEvent_t> events;
     size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
@@ -318,7 +318,7 @@ static void destroy(smiler_index *idx) {
         cudaFree(kv.second.second);
     }
     DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
-                      &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->tauk,
+                      &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->taulb,  &idx->tauk,
                       &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
                       &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred};
     for (DevBuf *b : bufs) b->release();
@@ -809,6 +809,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             ENS(idx->surv.ensure(4 * (size_t)seg_tot));
             ENS(idx->fin.ensure(8 * (size_t)seg_tot));
             ENS(idx->tauc.ensure(4 * (size_t)nseg * LT));
+            ENS(idx->taulb.ensure(4 * (size_t)nseg * LT));
             ENS(idx->tauk.ensure(8 * (size_t)nseg * LT));
             ENS(idx->taukey.ensure(8 * (size_t)nseg));
             ENS(idx->thr.ensure(4 * (size_t)nseg));
@@ -834,6 +835,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
             TRY(rc_);
         }
+        if (!lb_only) P.taulb = idx->taulb.as<uint32_t>();  // tile tau candidates' LB_w bits (trim keys)
         V *postbuf = sctx ? reinterpret_cast<V *>(sctx->ring) : idx->post.as<V>();
         MQMeta *d_meta = idx->meta.as<MQMeta>();
         CU(cudaMemcpyAsync(d_meta, meta, sizeof(MQMeta) * B, cudaMemcpyHostToDevice, idx->stream));
@@ -870,38 +872,42 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 const int nch = (LTt + kTrimChunk - 1) / kTrimChunk;
                 const bool two_stage = keep > 0 && nch > 1 && (int64_t)nch * keep <= kTrimCap;
                 if (keep > 0 && LTt > keep && (LTt <= kTrimBigCap || two_stage)) {
-                    auto trim1 = [&](const int32_t *src, int sstride, int nsrc) {
+                    const uint32_t *tlb = idx->taulb.as<uint32_t>();
+                    auto trim1 = [&](const int32_t *src, int sstride, int nsrc, const uint32_t *slb) {
                         int n2 = 1;
                         while (n2 < nsrc) n2 <<= 1;
                         const size_t sm = (size_t)8 * n2 + (size_t)4 * kpv;
                         set_smem((const void *)tau_trim_kernel<S>, sm);
                         tau_trim_kernel<S><<<nseg, 256, sm, idx->stream>>>(src, sstride, nsrc, idx->tauc.as<int32_t>(),
                                                                            LT, LTt, keep, kpv, idx->lb.as<V>(),
-                                                                           d_meta, nl);
+                                                                           d_meta, nl, slb);
                     };
                     // <= kTrimSmall: one bitonic sort; <= kTrimBigCap: radix select in shared
                     // memory; longer: two-stage (chunk bitonic sorts, then one more trim).
                     // reserved[0] == 9 (tests): radix, or two-stage with reserved[1] == 9
                     const bool test_alt = o.reserved[0] == 9;
                     if (LTt <= kTrimSmall && !test_alt) {
-                        trim1(idx->tauc.as<int32_t>(), LT, LTt);
+                        trim1(idx->tauc.as<int32_t>(), LT, LTt, tlb);
                     } else if (two_stage && (LTt > kTrimBigCap || (test_alt && o.reserved[1] == 9))) {
                         // chunk winners into the survivor buffer (unused until a6), then one more trim
+                        // (t in the survivor buffer, their LB_w bits in the finalist buffer:
+                        // both unused until a6/a7)
                         const int ostride = nch * keep;
                         TRY(idx->surv.ensure(4 * (size_t)nseg * ostride));
+                        TRY(idx->fin.ensure(4 * (size_t)nseg * ostride));
                         const size_t sm = (size_t)8 * kTrimChunk;
                         set_smem((const void *)tau_trim_chunk_kernel<S>, sm);
                         tau_trim_chunk_kernel<S><<<dim3(nch, nseg), 256, sm, idx->stream>>>(
                             idx->tauc.as<int32_t>(), LT, LTt, keep, idx->lb.as<V>(), d_meta, nl,
-                            idx->surv.as<int32_t>(), ostride);
+                            idx->surv.as<int32_t>(), ostride, tlb, reinterpret_cast<uint32_t *>(idx->fin.p));
                         CHECK_LAUNCH();
                         launches++;
-                        trim1(idx->surv.as<int32_t>(), ostride, ostride);
+                        trim1(idx->surv.as<int32_t>(), ostride, ostride, reinterpret_cast<const uint32_t *>(idx->fin.p));
                     } else {  // 32-bit LB keys, radix select in shared memory
                         const size_t sm = (size_t)4 * LTt;
                         set_smem((const void *)tau_trim_big_kernel<S>, sm);
                         tau_trim_big_kernel<S><<<nseg, 512, sm, idx->stream>>>(
-                            idx->tauc.as<int32_t>(), LT, LTt, keep, kpv, idx->lb.as<V>(), d_meta, nl);
+                            idx->tauc.as<int32_t>(), LT, LTt, keep, kpv, idx->lb.as<V>(), d_meta, nl, tlb);
                     }
                     CHECK_LAUNCH();
                     launches++;
