@@ -694,25 +694,32 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 template <typename V, int W>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
                                           V *lb, int32_t *tauc, int mq, int bx = -1) {
+    static_assert(W <= 32, "slot mask is 32-bit");
     const int d = P.len[i];
     const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
     const int64_t tend = min(m.t_hi, m.n - m.hz - d + 1);
     V *out = lb + m.seg_off + (int64_t)i * m.n;
     const int64_t t0 = s0 - d;
+    // valid slots b: tmin <= t0 + b < tend, as one bit mask (two 64-bit
+    // compares per emission instead of two per slot)
+    const int blo = (int)max((int64_t)0, min((int64_t)W, tmin - t0));
+    const int bhi = (int)max((int64_t)0, min((int64_t)W, tend - t0));
+    const uint32_t vmask = (uint32_t)(((1ull << bhi) - 1ull) & ~((1ull << blo) - 1ull));
+    constexpr uint32_t kAll = (uint32_t)((1ull << W) - 1ull);
     if (P.fuse) {  // a6 here: keep LB <= thr (ties survive), warp-aggregated append
         const int seg = mq * P.n_len + i;
         const uint32_t th = P.thr[seg];
         uint32_t keep = 0;
 #pragma unroll
         for (int b = 0; b < W; b++) {
-            const int64_t t = t0 + b;
             bool k_;
             if constexpr (std::is_same<V, float>::value)
                 k_ = v[b] <= __uint_as_float(th);
             else
                 k_ = v[b] <= (int32_t)th;
-            keep |= (uint32_t)(k_ && t >= tmin && t < tend) << b;
+            keep |= (uint32_t)k_ << b;
         }
+        keep &= vmask;
         const int lane = threadIdx.x & 31;
         const int cnt = __popc(keep);
         int x = cnt;
@@ -732,8 +739,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
             if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
         return;
     }
-    const bool all = t0 >= tmin && t0 + W <= tend;
-    if (all && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
+    if (vmask == kAll && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
 #pragma unroll
         for (int b = 0; b < W; b += 4) {
             typename Tr<int16_t>::V4 pk;  // 4 x 32-bit lanes (int or float bits)
@@ -745,10 +751,8 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
         }
     } else {
 #pragma unroll
-        for (int b = 0; b < W; b++) {
-            const int64_t t = t0 + b;
-            if (t >= tmin && t < tend) out[t] = v[b];
-        }
+        for (int b = 0; b < W; b++)
+            if (vmask >> b & 1u) out[t0 + b] = v[b];
     }
     if (P.E <= 0) return;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -758,26 +762,23 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     // grows with the slot b inside a thread and with the lane across the warp,
     // so among equal LB_w bits the lowest lane, then the lowest b, has the
     // smallest t (the same keys as a 64-bit (LB_w bits << 32 | t) minimum).
+    // Per round: the thread minimum (no index tracking), the warp minimum, the
+    // lowest lane holding it, and that lane's lowest slot holding it.
     uint32_t kb[W];
 #pragma unroll
-    for (int b = 0; b < W; b++) {
-        const int64_t t = t0 + b;
-        kb[b] = (t >= tmin && t < tend) ? key_bits(v[b]) : 0xFFFFFFFFu;
-    }
+    for (int b = 0; b < W; b++) kb[b] = (vmask >> b & 1u) ? key_bits(v[b]) : 0xFFFFFFFFu;
     for (int e = 0; e < P.E; e++) {
         uint32_t best = kb[0];
-        int bs = 0;
 #pragma unroll
-        for (int b = 1; b < W; b++) {
-            if (kb[b] < best) {
-                best = kb[b];
-                bs = b;
-            }
-        }
+        for (int b = 1; b < W; b++) best = min(best, kb[b]);
         const uint32_t win = __reduce_min_sync(0xffffffffu, best);
         const int wl = __ffs(__ballot_sync(0xffffffffu, best == win)) - 1;
+        uint32_t hit = 0;
+#pragma unroll
+        for (int b = 0; b < W; b++) hit |= (uint32_t)(kb[b] == win) << b;
+        const int bs = __ffs(hit) - 1;  // valid on lane wl
         const int tw = __shfl_sync(0xffffffffu, (int)(t0 + bs), wl);
-        if (lane == wl) {
+        if (lane == wl && e + 1 < P.E) {
 #pragma unroll
             for (int b = 0; b < W; b++)
                 if (b == bs) kb[b] = 0xFFFFFFFFu;
