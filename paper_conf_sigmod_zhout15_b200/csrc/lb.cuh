@@ -29,6 +29,9 @@
 #ifndef SMILER_DIAG_UNROLL2
 #define SMILER_DIAG_UNROLL2 0
 #endif
+#ifndef SMILER_TMA_SYNC2
+#define SMILER_TMA_SYNC2 1  // TMA ring scan: one CTA barrier per two CSG rows
+#endif
 #ifndef SMILER_TMA_EMPTYBAR
 #define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower)
 #endif
@@ -1130,7 +1133,15 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
 // 2- or 4-byte loads, no per-element address arithmetic, whole 512-byte rows
 // per request.  Sums, emission and the tau set are group_scan_reg's.
 // ---------------------------------------------------------------------------
-constexpr int kTmaStages = 4;
+#ifndef SMILER_TMA_STAGES_W16
+#define SMILER_TMA_STAGES_W16 4
+#endif
+#ifndef SMILER_TMA_MINB_W16
+#define SMILER_TMA_MINB_W16 2
+#endif
+// TMA ring depth (a power of two) and CTAs per SM the register budget must fit
+template <int W> constexpr int tma_stages() { return W >= 16 ? SMILER_TMA_STAGES_W16 : 4; }
+template <int W> constexpr int tma_minb() { return W >= 16 ? SMILER_TMA_MINB_W16 : SMILER_GS_MINB(W); }
 template <typename PV> constexpr int tma_align_elems() { return 16 / (int)sizeof(PV); }
 // one stage: per plane a [W][256] main box and a [W][A] tail box, every box at
 // a 128-byte aligned shared-memory offset
@@ -1141,7 +1152,7 @@ template <int W, typename PV> constexpr size_t tma_stage_elems() {
     return (size_t)2 * W * kScanThreads + 2 * tma_tail_pitch<W, PV>();
 }
 template <int W, typename PV> constexpr size_t tma_scan_smem() {
-    return (size_t)kTmaStages * tma_stage_elems<W, PV>() * sizeof(PV);
+    return (size_t)tma_stages<W>() * tma_stage_elems<W, PV>() * sizeof(PV);
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -1196,10 +1207,11 @@ __device__ __forceinline__ void tma_row_add(const PV *pe, int nrow, V (&se)[W], 
 }
 
 template <typename S, int W, typename PV>
-__global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tma_kernel(
+__global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_kernel(
     const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_tail, const MQMeta *meta,
     const QParams P, typename Tr<S>::V *lb, int32_t *tauc, int nb, int n_mq, int row0, int prows) {
     using V = typename Tr<S>::V;
+    constexpr int kTmaStages = tma_stages<W>();
     constexpr int NT = kScanThreads;
     constexpr int A = tma_align_elems<PV>();      // TMA start-column granule (16 bytes)
     constexpr int STAGE = (int)tma_stage_elems<W, PV>();
@@ -1222,9 +1234,9 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
     // tile's rows stream in while this one emits.
     const int ntiles = n_mq * nb;
     const int my_tiles = (int)blockIdx.x < ntiles ? (ntiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
-    const int64_t g_end = (int64_t)my_tiles * mmax;
-    auto issue = [&](int64_t g) {  // global row g -> stage g % kTmaStages
-        const int k = (int)(g / mmax), j = (int)(g - (int64_t)k * mmax);
+    const int g_end = my_tiles * mmax;  // rows of this CTA (32-bit: a few thousand)
+    auto issue = [&](int g) {  // global row g -> stage g % kTmaStages
+        const int k = g / mmax, j = g - k * mmax;
         const int tile = (int)blockIdx.x + k * (int)gridDim.x;
         const int mq = tile / nb, bx = tile - mq * nb;
         // tensor row of this stream's P_EQ row 0: the streams' rings are
@@ -1233,10 +1245,10 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
         int pr = j * W + P.ring_cursor;
         pr -= pr >= n_sw ? n_sw : 0;
         pr -= pr >= n_sw ? n_sw : 0;
-        const int st = (int)(g % kTmaStages);
+        const int st = g & (kTmaStages - 1);
         mbar_expect_tx(&s_full[st], STAGE_BYTES);
         const int col = bx * NT - 1 - j;
-        const int ca = col - (((col % A) + A) % A);  // floor to the 16-byte granule
+        const int ca = col & ~(A - 1);  // floor to the 16-byte granule (A is a power of two)
         PV *sb = s_ring + (size_t)st * STAGE;
         tma_load_2d(sb, &tmap, ca, row_base + pr, &s_full[st]);
         tma_load_2d(sb + W * NT, &tmap, ca, row_base + prows + pr, &s_full[st]);
@@ -1252,14 +1264,14 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
     }
     __syncthreads();
     if (x == 0)
-        for (int64_t g = 0; g < kTmaStages && g < g_end; g++) issue(g);
+        for (int g = 0; g < kTmaStages && g < g_end; g++) issue(g);
     uint64_t emit_rows = 0, save_rows = 0;
     for (int i = 0; i < nl; i++) {
         const int qi = P.len[i] / W;
         if (qi >= 1) emit_rows |= 1ull << (qi - 1);
         if (qi >= 2) save_rows |= 1ull << (qi - 2);
     }
-    int64_t g = 0;
+    int g = 0;
     for (int k = 0; k < my_tiles; k++) {
         const int tile = (int)blockIdx.x + k * (int)gridDim.x;
         const int mq = tile / nb, bx = tile - mq * nb;
@@ -1272,11 +1284,11 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
 #pragma unroll
         for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
         for (int j = 0; j < mmax; j++, g++) {
-            const int st = (int)(g % kTmaStages);
+            const int st = g & (kTmaStages - 1);
             mbar_wait(&s_full[st], (uint32_t)(g / kTmaStages) & 1u);
             const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
             const int col = (int)(Rb - j);
-            const int xo = x + (((col % A) + A) % A);  // this thread's column within the aligned boxes
+            const int xo = x + (col & (A - 1));  // this thread's column within the aligned boxes
             const PV *sb = s_ring + (size_t)st * STAGE;
             // main-box columns (all but at most A-1 threads of the last warp) use
             // compile-time row pitches, so the 2W loads take immediate offsets
@@ -1297,10 +1309,23 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_tm
                 issue(g + kTmaStages);
             }
 #else
+            if (SMILER_TMA_SYNC2 && kTmaStages >= 4) {
+            // one CTA barrier per two rows: after odd rows (and the CTA's last row)
+            // the stages of rows g-1 and g are free and are refilled together
+            if ((g & 1) || g + 1 == g_end) {
+                __syncthreads();  // every thread has read the stages of rows g-1, g
+                if (x == 0) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    if ((g & 1) && g - 1 + kTmaStages < g_end) issue(g - 1 + kTmaStages);
+                    if (g + kTmaStages < g_end) issue(g + kTmaStages);
+                }
+            }
+            } else {
             __syncthreads();  // every thread has read stage st
             if (x == 0 && g + kTmaStages < g_end) {
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 issue(g + kTmaStages);
+            }
             }
 #endif
             const bool live = bx < m.nblk;  // grids are sized for the longest sensor of the chunk

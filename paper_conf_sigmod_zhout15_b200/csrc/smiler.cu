@@ -200,9 +200,12 @@ static int meta_stage(smiler_index *idx, int n, MQMeta **out, int *slot) {
 }
 
 // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per kernel and size.
+// Opt a kernel in to `bytes` of dynamic shared memory.  Always set (not only
+// above 48 KB): the default cap is 48 KB minus the kernel's STATIC shared
+// memory, so e.g. 34 KB dynamic + 16 KB static fails to launch without it.
 static void set_smem(const void *kern, size_t bytes) {
     static std::map<const void *, size_t> done;
-    if (bytes <= 48 * 1024) return;
+    if (bytes == 0) return;
     auto it = done.find(kern);
     if (it != done.end() && it->second >= bytes) return;
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
