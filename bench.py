@@ -611,7 +611,10 @@ def main():
     # toward zero (smiler_knn_opts.exact_postings = 0), otherwise 2 x 4 bytes
     pair_bytes = 4 if (R.streaming and args.dtype == "f32" and wl.window in (4, 8, 16, 32)) else 8
     post_bytes_step = pair_bytes * n_sw * sum(p // wl.window for p in pts)
-    lb_bytes_step = 4 * n_len * sum(pts)
+    # LB_w array entry: fp16 rounded down on the product path (one direction of the
+    # library's lb_bytes stat, which counts the a4 write and the a6 read), else 4 B
+    lb_entry = (acc["lb_bytes"] / (2.0 * n_len * sum(pts) * steps)) if acc["lb_bytes"] else 4.0
+    lb_bytes_step = lb_entry * n_len * sum(pts)
 
     # continuous streams recompute only SW_0 (EQ + EC) and SW_1..SW_rho_max (EQ):
     # (rho_max + 2) / 2 term-pair equivalents per (DW, j) instead of n_sw

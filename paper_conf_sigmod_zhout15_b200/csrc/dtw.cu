@@ -33,10 +33,15 @@ namespace smiler {
 #endif
 constexpr int kDtwThreads = SMILER_DTW_THREADS;
 constexpr int kDtwWarps = kDtwThreads / 32;
-constexpr int kRows = 4;                       // rows per register block
+#ifndef SMILER_DTW_KROWS_WIDE
+#define SMILER_DTW_KROWS_WIDE 4
+#endif
+constexpr int kRowsMax = 8;
+// rows per register block (interleaved by the scheduler): 4, or the wide-band setting
+template <int RHO> constexpr int dtw_krows() { return RHO > 12 ? SMILER_DTW_KROWS_WIDE : 4; }
 
-// Per-warp query staging length (values): d + W + kRows, rounded up to 4.
-__host__ __device__ inline int dtw_qstage(int d, int rho) { return (d + 2 * rho + 1 + kRows + 3) & ~3; }
+// Per-warp query staging length (values): d + W + kRowsMax, rounded up to 4.
+__host__ __device__ inline int dtw_qstage(int d, int rho) { return (d + 2 * rho + 1 + kRowsMax + 3) & ~3; }
 
 template <typename V> __device__ __forceinline__ V vmin3(V a, V b, V c);
 template <> __device__ __forceinline__ float vmin3(float a, float b, float c) {
@@ -84,6 +89,7 @@ template <typename S, int RHO>
 __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE : 1)) dtw_kernel(const DtwParams<S> p) {
     using V = typename Tr<S>::V;
     constexpr int W = 2 * RHO + 1;
+    constexpr int kRows = dtw_krows<RHO>();
     constexpr bool IS_F = std::is_same<S, float>::value;
     const V INF = Tr<S>::inf();
     extern __shared__ __align__(16) unsigned char dtw_smem[];

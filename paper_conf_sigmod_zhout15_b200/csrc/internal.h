@@ -58,6 +58,7 @@ struct QParams {
     int ring_cursor;  // continuous streams: physical posting row of SW_b is (b + ring_cursor) mod n_sw
     int lbsel;        // which sums make the bound: 0 = max(EQ, EC) (Eq. 5 / Thm 4.1), 1 = EQ, 2 = EC
     int fuse;         // 1: the LB kernel filters (LB <= thr) and appends survivors itself (a4+a6)
+    int lb_half;      // 1: the LB_w array holds fp16 rounded down (<= the bound: still a lower bound)
     const uint32_t *thr;  // fuse: per-segment admission bound (tau_select_kernel)
     int32_t *surv;        // fuse: survivor t lists (segment layout)
     int32_t *scount;      // fuse: survivors per segment

@@ -342,7 +342,14 @@ __global__ void tau_share_kernel(uint64_t *tau_key, uint32_t *thr, unsigned long
 constexpr int kFiltThreads = 256;
 constexpr int kFiltItems = 32;
 
-template <typename S>
+// LH: the LB_w array holds fp16 rounded down (P.lb_half); the comparison is
+// then made in float against the threshold rounded up, which keeps a superset
+// of the candidates with LB_w <= tau (every survivor is verified exactly).
+// fp16 rows are read with 16-byte loads from the aligned address at or below the
+// block's first t (a block covers kFiltSpanH candidates, so 1024 vectors of 8
+// cover it for any alignment); halves outside the block's range are masked.
+constexpr int kFiltSpanH = kFiltThreads * kFiltItems - 8;
+template <typename S, bool LH>
 __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<S>::V *lb,
                                                              const MQMeta *meta, const QParams P,
                                                              const uint32_t *thr, int32_t *surv,
@@ -356,21 +363,58 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
     const int d = P.len[i];
     const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
     const int64_t te = min(m.t_hi, m.n - m.hz - d + 1);
-    const int64_t t0 = tb + (int64_t)blockIdx.x * kFiltThreads * kFiltItems;
+    const int span = LH ? kFiltSpanH : kFiltThreads * kFiltItems;
+    const int64_t t0 = tb + (int64_t)blockIdx.x * span;
     if (t0 >= te) return;
+    const int64_t t1 = min(te, t0 + span);
     const uint32_t th = thr[seg];
-    const V *src = lb + m.seg_off + (int64_t)i * m.n;
     uint32_t flags = 0;
+    int64_t ta = 0;  // LH: t of the first half of the block's aligned window
+    if constexpr (LH) {
+        float thf;
+        if constexpr (std::is_same<V, float>::value)
+            thf = __uint_as_float(th);
+        else
+            thf = __int2float_ru((int32_t)th);
+        // h <= thf (float)  <=>  h <= thf rounded up to fp16 (h is an fp16 value);
+        // the +inf threshold of "no pruning" stays +inf
+        const __half2 th2 = __half2half2(__float2half_ru(thf));
+        const __half *row = reinterpret_cast<const __half *>(lb) + m.seg_off + (int64_t)i * m.n;
+        const uintptr_t a0 = reinterpret_cast<uintptr_t>(row + t0);
+        const int4 *vb = reinterpret_cast<const int4 *>(a0 & ~(uintptr_t)15);
+        ta = t0 - (int64_t)((a0 & 15) >> 1);
+        const int r0 = (int)(t0 - ta), r1 = (int)(t1 - ta);  // block range relative to ta (< 2^31)
 #pragma unroll
-    for (int it = 0; it < kFiltItems; it++) {
-        const int64_t t = t0 + (int64_t)it * kFiltThreads + threadIdx.x;
-        if (t < te) {
-            bool keep;
-            if constexpr (std::is_same<V, float>::value)
-                keep = src[t] <= __uint_as_float(th);
-            else
-                keep = src[t] <= (int32_t)th;
-            flags |= (uint32_t)keep << it;
+        for (int it = 0; it < kFiltItems / 8; it++) {
+            const int vi = it * kFiltThreads + threadIdx.x;
+            const int rv = vi * 8;
+            if (rv < r1 && rv + 8 > r0) {
+                const int lo = max(0, r0 - rv), hi = min(8, r1 - rv);
+                const uint32_t vm = ((1u << hi) - 1u) & ~((1u << lo) - 1u);
+                const int4 raw = vb[vi];
+                const __half2 *h2 = reinterpret_cast<const __half2 *>(&raw);
+                uint32_t kb = 0;
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                    const uint32_t r = __hle2_mask(h2[q], th2);  // 0xFFFF per lane that holds
+                    kb |= ((r & 1u) | ((r >> 15) & 2u)) << (2 * q);
+                }
+                flags |= (kb & vm) << (it * 8);
+            }
+        }
+    } else {
+        const V *src = lb + m.seg_off + (int64_t)i * m.n;
+#pragma unroll
+        for (int it = 0; it < kFiltItems; it++) {
+            const int64_t t = t0 + (int64_t)it * kFiltThreads + threadIdx.x;
+            if (t < t1) {
+                bool keep;
+                if constexpr (std::is_same<V, float>::value)
+                    keep = src[t] <= __uint_as_float(th);
+                else
+                    keep = src[t] <= (int32_t)th;
+                flags |= (uint32_t)keep << it;
+            }
         }
     }
     int total;
@@ -380,8 +424,13 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
     int o = s_base + pos;
     int32_t *dst = surv + m.seg_off + (int64_t)i * m.n;
 #pragma unroll
-    for (int it = 0; it < kFiltItems; it++)
-        if (flags >> it & 1) dst[o++] = (int32_t)(t0 + (int64_t)it * kFiltThreads + threadIdx.x);
+    for (int it = 0; it < kFiltItems; it++) {
+        if (flags >> it & 1) {
+            const int64_t t = LH ? ta + (int64_t)((it / 8) * kFiltThreads + threadIdx.x) * 8 + (it % 8)
+                                 : t0 + (int64_t)it * kFiltThreads + threadIdx.x;
+            dst[o++] = (int32_t)t;
+        }
+    }
 }
 
 // no-prune mode: every owned candidate of every segment is a survivor.

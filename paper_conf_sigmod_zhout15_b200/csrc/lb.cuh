@@ -694,6 +694,10 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 
 // Write the W final LB_w values of IQ i held by this thread (slots e = s0 + b,
 // t = e - d_i contiguous) and emit its warp's tau candidates.
+// LB_w -> fp16 rounded toward -inf: never above the bound (saturates at 65504)
+__device__ __forceinline__ __half lb_to_half(float v) { return __float2half_rd(v); }
+__device__ __forceinline__ __half lb_to_half(int32_t v) { return __int2half_rd(v); }
+
 template <typename V, int W>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
                                           V *lb, int32_t *tauc, int mq, int bx = -1) {
@@ -742,7 +746,22 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
             if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
         return;
     }
-    if (vmask == kAll && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
+    if (P.lb_half) {  // LB_w array as fp16 rounded down (a valid, slightly looser bound)
+        __half *oh = reinterpret_cast<__half *>(lb) + m.seg_off + (int64_t)i * m.n + t0;
+        if (vmask == kAll && W % 8 == 0 && ((reinterpret_cast<uintptr_t>(oh) & 15) == 0)) {
+#pragma unroll
+            for (int b = 0; b < W; b += 8) {
+                __align__(16) __half hv[8];
+#pragma unroll
+                for (int q = 0; q < 8; q++) hv[q] = lb_to_half(v[b + q]);
+                *reinterpret_cast<int4 *>(oh + b) = *reinterpret_cast<const int4 *>(hv);
+            }
+        } else {
+#pragma unroll
+            for (int b = 0; b < W; b++)
+                if (vmask >> b & 1u) oh[b] = lb_to_half(v[b]);
+        }
+    } else if (vmask == kAll && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
 #pragma unroll
         for (int b = 0; b < W; b += 4) {
             typename Tr<int16_t>::V4 pk;  // 4 x 32-bit lanes (int or float bits)

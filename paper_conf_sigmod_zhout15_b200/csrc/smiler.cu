@@ -946,8 +946,12 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // seeded only by the previous neighbours, E = 0), the LB kernel compares
         // each LB_w with tau_i as it is produced and appends the survivors; the
         // LB_w array is never written or re-read (P:1437-1448 in one pass).
-        const bool fuse = use_prev && E == 0 && !lb_only && !o.no_prune &&
-                          (pl.direct || (pl.fused && pl.fused_kind == 0) || (!pl.fused && pl.scan_reg));
+        const bool diag_emitters = pl.direct || (pl.fused && pl.fused_kind == 0) || (!pl.fused && pl.scan_reg);
+        const bool fuse = use_prev && E == 0 && !lb_only && !o.no_prune && diag_emitters;
+        // LB_w array as fp16 rounded down for the filter (its only reader besides the
+        // tau trim, which takes the bounds from P.taulb): half the bytes written by
+        // a4 and read by a6.  lb_only (smiler_lower_bounds) and exact_postings keep V.
+        P.lb_half = !lb_only && !o.no_prune && diag_emitters && !o.exact_postings;
         TRY(tm.mark(0));
         // ---- a2 ----------------------------------------------------------
         query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env,
@@ -1153,7 +1157,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             CHECK_LAUNCH();
             launches++;
         }
-        lb_bytes += 2 * seg_tot * 4;
+        if (!P.fuse) lb_bytes += 2 * seg_tot * (P.lb_half ? 2 : (int64_t)sizeof(V));  // a4 write + a6 read
         TRY(tm.mark(3));
         if (lb_only) {
             // copy LB_w [n_mq][n_len][N] and postings out
@@ -1178,10 +1182,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             if (fuse) {
                 // survivors were appended by the LB kernel
             } else if (!o.no_prune) {
-                dim3 grid((unsigned)((nmax + kFiltThreads * kFiltItems - 1) / (kFiltThreads * kFiltItems)),
-                          (unsigned)nseg);
-                filter_kernel<S><<<grid, kFiltThreads, 0, idx->stream>>>(idx->lb.as<V>(), d_meta, P, thr,
-                                                                         idx->surv.as<int32_t>(), scount);
+                const int span = P.lb_half ? kFiltSpanH : kFiltThreads * kFiltItems;
+                dim3 grid((unsigned)((nmax + span - 1) / span), (unsigned)nseg);
+                if (P.lb_half)
+                    filter_kernel<S, true><<<grid, kFiltThreads, 0, idx->stream>>>(idx->lb.as<V>(), d_meta, P, thr,
+                                                                               idx->surv.as<int32_t>(), scount);
+                else
+                    filter_kernel<S, false><<<grid, kFiltThreads, 0, idx->stream>>>(idx->lb.as<V>(), d_meta, P,
+                                                                                thr, idx->surv.as<int32_t>(),
+                                                                                scount);
             } else {
                 dim3 grid((unsigned)std::min<int64_t>((nmax + 255) / 256, 1024), (unsigned)nseg);
                 all_candidates_kernel<<<grid, 256, 0, idx->stream>>>(d_meta, P, idx->surv.as<int32_t>(), scount);
