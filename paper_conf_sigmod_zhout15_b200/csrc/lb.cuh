@@ -67,6 +67,15 @@ template <> __device__ __forceinline__ void post_st<__half, float>(__half *p, fl
 }
 template <typename V, typename PV> __device__ __forceinline__ V post_cv(PV x) { return x; }
 template <> __device__ __forceinline__ float post_cv<float, __half>(__half x) { return __half2float(x); }
+// acc += posting entry.  fp16 entries into f32 sums use sm_100's mixed-precision
+// add (PTX add.rn.f32.f16, one FHADD): the fp16 -> f32 conversion is exact, so
+// the result is bit-identical to converting first and adding in f32.
+template <typename V, typename PV> __device__ __forceinline__ void post_acc(V &acc, PV x) { acc += post_cv<V>(x); }
+template <> __device__ __forceinline__ void post_acc<float, __half>(float &acc, __half x) {
+    float r;
+    asm("add.rn.f32.f16 %0, %1, %2;" : "=f"(r) : "h"(__half_as_ushort(x)), "f"(acc));
+    acc = r;
+}
 
 // emission table: em[j*w + b] = lo | hi << 8, the IQ range [lo, hi) with
 // m_i(b) == j + 1 (contiguous in i because d_i increases).
@@ -1110,8 +1119,8 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
         if (LA && j + 1 < mmax) load(j + 1, rr);
 #pragma unroll
         for (int b = 0; b < W; b++) {
-            se[b] += post_cv<V>(pe[b]);
-            sc[b] += post_cv<V>(pc[b]);
+            post_acc<V>(se[b], pe[b]);
+            post_acc<V>(sc[b], pc[b]);
         }
         if (!LA && j + 1 < mmax) load(j + 1, rr);
         if (emit_rows >> j & 1ull) {
@@ -1219,9 +1228,10 @@ __device__ __forceinline__ void tma_row_add(const PV *pe, int nrow, V (&se)[W], 
     }
 #pragma unroll
     for (int b = 0; b < W; b++) {
-        const V e = post_cv<V>(ve[b]), c = post_cv<V>(vc[b]);
-        se[b] += (FULL || b < nrow) ? e : (V)0;
-        sc[b] += (FULL || b < nrow) ? c : (V)0;
+        if (FULL || b < nrow) {
+            post_acc<V>(se[b], ve[b]);
+            post_acc<V>(sc[b], vc[b]);
+        }
     }
 }
 
