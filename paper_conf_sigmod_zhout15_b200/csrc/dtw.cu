@@ -82,6 +82,18 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
     }
 }
 
+#ifndef SMILER_DTW_CPASYNC
+#define SMILER_DTW_CPASYNC 1  // f32: candidate rows staged with cp.async, double-buffered
+#endif
+// shared-memory row buffers per warp for the candidate staging
+template <typename S> constexpr int dtw_cbufs() { return (std::is_same<S, float>::value && SMILER_DTW_CPASYNC) ? 2 : 1; }
+
+__device__ __forceinline__ void cp_async4(void *dst, const void *src, bool ok) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+                 "l"(src), "r"(ok ? 4 : 0)
+                 : "memory");
+}
+
 #ifndef SMILER_DTW_MINB_WIDE
 #define SMILER_DTW_MINB_WIDE 1  // CTAs per SM the compiler must fit for rho > 12 (register cap)
 #endif
@@ -96,8 +108,10 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
     const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5;
     const int qs = dtw_qstage(p.d, RHO);
-    V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (qs + 32 * 33);
-    V (*s_c)[33] = reinterpret_cast<V (*)[33]>(sq + qs);
+    constexpr int NB = dtw_cbufs<S>();
+    constexpr bool ASYNC = NB == 2;
+    V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (qs + NB * 32 * 33);
+    V (*s_cb)[33] = reinterpret_cast<V (*)[33]>(sq + qs);  // NB buffers of [32][33]
     const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int nw = (gridDim.x * blockDim.x) >> 5;
     const int total = p.task_off[p.n_mq];
@@ -145,17 +159,42 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
         for (int u = 0; u < W; u++) band[u] = (u == RHO) ? (V)0 : INF;
 
         const S *cs = p.series + m.series_off;
-        for (int j0 = 0; j0 < d; j0 += 32) {
-            __syncwarp();
+        // rows j0 .. j0+31 of the warp's 32 candidates -> buf[row][candidate]
+        // (f32: asynchronous 4-byte copies, zero-filled outside; one commit group)
+        auto stage_async = [&](V (*buf)[33], int j0) {
             const bool in_row = (j0 + lane) < d;
 #pragma unroll 4
             for (int l = 0; l < 32; l++) {
-                int tl = __shfl_sync(0xffffffffu, t, l);
-                V v = (V)0;
-                if (tl >= 0 && in_row) v = (V)cs[tl + j0 + lane];
-                s_c[lane][l] = v;
+                const int tl = __shfl_sync(0xffffffffu, t, l);
+                const bool ok = tl >= 0 && in_row;
+                cp_async4(&buf[lane][l], ok ? (const void *)(cs + tl + j0 + lane) : (const void *)cs, ok);
             }
-            __syncwarp();
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        };
+        if constexpr (ASYNC) stage_async(s_cb, 0);
+        for (int j0 = 0, blk = 0; j0 < d; j0 += 32, blk++) {
+            V (*s_c)[33] = s_cb + (ASYNC ? (blk & 1) * 32 : 0);
+            if constexpr (ASYNC) {
+                // the next block streams in while this one is computed
+                if (j0 + 32 < d) {
+                    stage_async(s_cb + ((blk + 1) & 1) * 32, j0 + 32);
+                    asm volatile("cp.async.wait_group 1;" ::: "memory");
+                } else {
+                    asm volatile("cp.async.wait_group 0;" ::: "memory");
+                }
+                __syncwarp();
+            } else {
+                __syncwarp();
+                const bool in_row = (j0 + lane) < d;
+#pragma unroll 4
+                for (int l = 0; l < 32; l++) {
+                    int tl = __shfl_sync(0xffffffffu, t, l);
+                    V v = (V)0;
+                    if (tl >= 0 && in_row) v = (V)cs[tl + j0 + lane];
+                    s_c[lane][l] = v;
+                }
+                __syncwarp();
+            }
             const int jn = min(32, d - j0);
             int r = 0;
             for (; r + kRows <= jn; r += kRows) {
@@ -181,6 +220,7 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
                 for (int x = 0; x < W; x++) qr[x] = sq[j - 1 + x];
                 dp_row<V, RHO, !IS_F>(band, qr, s_c[r][lane], j, d, INF);
             }
+            if constexpr (ASYNC) __syncwarp();  // buffer blk & 1 is refilled two blocks later
         }
         const V dist = band[RHO];
         const uint64_t key = t >= 0 ? (((uint64_t)vbits<V>(dist) << 32) | (uint32_t)t) : kKeyMax;
@@ -202,11 +242,12 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
 template <typename S, int RHO>
 static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
     using V = typename Tr<S>::V;
-    size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + 32 * 33) * sizeof(V);
+    constexpr int NB = dtw_cbufs<S>();
+    size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + NB * 32 * 33) * sizeof(V);
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(dtw_kernel<S, RHO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + 32 * 33) * sizeof(V)));
+                             (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + NB * 32 * 33) * sizeof(V)));
         attr = true;
     }
     static int occ = 0, sms = 0;
@@ -216,7 +257,7 @@ static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(
             &occ, dtw_kernel<S, RHO>, kDtwThreads,
-            (size_t)kDtwWarps * (dtw_qstage(256, RHO) + 32 * 33) * sizeof(V));
+            (size_t)kDtwWarps * (dtw_qstage(256, RHO) + NB * 32 * 33) * sizeof(V));
         if (occ < 1) occ = 1;
     }
     if (grid <= 0) grid = sms * occ;
