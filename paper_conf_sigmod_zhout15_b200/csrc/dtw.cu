@@ -83,7 +83,7 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
 }
 
 #ifndef SMILER_DTW_CPASYNC
-#define SMILER_DTW_CPASYNC 1  // f32: candidate rows staged with cp.async, double-buffered
+#define SMILER_DTW_CPASYNC 0  // 1: f32 candidate rows staged with cp.async, double-buffered (measured slower: occupancy)
 #endif
 // shared-memory row buffers per warp for the candidate staging
 template <typename S> constexpr int dtw_cbufs() { return (std::is_same<S, float>::value && SMILER_DTW_CPASYNC) ? 2 : 1; }

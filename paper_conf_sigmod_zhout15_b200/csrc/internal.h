@@ -14,7 +14,7 @@ constexpr int kMaxK = 1024;      // max k
 constexpr int kMaxWindow = 64;   // max omega
 constexpr int kMaxRhoFast = 32;  // rho handled by the register-band DTW kernels
 constexpr int kSortCap = 4096;   // keys sorted in shared memory by one CTA
-constexpr int kTrimBigCap = 55296;  // tau-set trim: 32-bit keys in shared memory (216 KB)
+constexpr int kTrimBigCap = 27648;  // tau-set trim: 32-bit keys + t in shared memory (216 KB)
 constexpr int kMaxPredK = 128;   // neighbours per GP predictor (k x k fp64 factor in shared memory)
 constexpr uint64_t kKeyMax = ~0ull;
 

@@ -652,18 +652,19 @@ __global__ void __launch_bounds__(256) tau_trim_chunk_kernel(const int32_t *tauc
 
 // tau_trim_kernel for tile lists too long for a 64-bit key sort (window-range
 // scale, C4: ~49k per item query): only the 32-bit LB_w bits are kept in shared
-// memory (<= kTrimBigCap entries), the keep-th smallest is radix-selected (four
+// memory with their t (<= kTrimBigCap entries), the keep-th smallest is radix-selected (four
 // 8-bit MSB passes over shared memory), and the candidates below it, then those
 // equal to it up to `keep`, are compacted to the front in any order (any subset
 // of verified candidates gives a valid tau).
 template <typename S>
-__global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
+__global__ void __launch_bounds__(256) tau_trim_big_kernel(int32_t *tauc, int LT, int LTt, int keep, int kprev,
                                                           const typename Tr<S>::V *lb, const MQMeta *meta,
                                                           int n_len, const uint32_t *tlb) {
-    extern __shared__ __align__(16) uint32_t s_lbk[];
+    extern __shared__ __align__(16) uint32_t s_lbk[];  // [LTt] LB bits, then [LTt] t
     __shared__ int s_hist[256];
     __shared__ uint32_t s_sel[2];
     __shared__ int s_cnt;
+    int32_t *s_t = reinterpret_cast<int32_t *>(s_lbk + LTt);
     const int seg = blockIdx.x;
     const int mq = seg / n_len, i = seg % n_len;
     const MQMeta m = meta[mq];
@@ -672,6 +673,7 @@ __global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT
     const uint32_t *lrow = tlb ? tlb + (int64_t)seg * LT : nullptr;
     for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
         const int t = row[x];
+        s_t[x] = t;
         s_lbk[x] = t >= 0 ? (lrow ? lrow[x] : key_bits(lbi[t])) : 0xFFFFFFFFu;
     }
     // keep-th smallest valid value (MSB radix select over shared memory)
@@ -716,39 +718,28 @@ __global__ void __launch_bounds__(512) tau_trim_big_kernel(int32_t *tauc, int LT
     }
     const uint32_t thr = few ? 0xFFFFFFFEu : prefix;
     // previous neighbours [LTt, LTt + kprev) -> [keep, keep + kprev): read them first
-    int32_t pv[2];  // kprev <= 2 * 512 = kMaxK
+    int32_t pv[4];  // kprev <= 4 * 256 = kMaxK
 #pragma unroll
-    for (int r = 0; r < 2; r++) {
-        const int j = threadIdx.x + r * 512;
+    for (int r = 0; r < 4; r++) {
+        const int j = threadIdx.x + r * 256;
         pv[r] = j < kprev ? row[LTt + j] : -1;
-    }
-    int32_t tl[kTrimBigCap / 512];  // this thread's tile t values (row is rewritten below)
-#pragma unroll
-    for (int r = 0; r < kTrimBigCap / 512; r++) {
-        const int x = threadIdx.x + r * 512;
-        tl[r] = x < LTt ? row[x] : -1;
     }
     if (threadIdx.x == 0) s_cnt = 0;
     __syncthreads();
-#pragma unroll
-    for (int r = 0; r < kTrimBigCap / 512; r++) {
-        const int x = threadIdx.x + r * 512;
-        if (x < LTt && s_lbk[x] < thr) row[atomicAdd(&s_cnt, 1)] = tl[r];
-    }
+    for (int x = threadIdx.x; x < LTt; x += blockDim.x)
+        if (s_lbk[x] < thr) row[atomicAdd(&s_cnt, 1)] = s_t[x];
     __syncthreads();
-#pragma unroll
-    for (int r = 0; r < kTrimBigCap / 512; r++) {
-        const int x = threadIdx.x + r * 512;
-        if (x < LTt && s_lbk[x] == thr && s_lbk[x] != 0xFFFFFFFFu) {
+    for (int x = threadIdx.x; x < LTt; x += blockDim.x) {
+        if (s_lbk[x] == thr && s_lbk[x] != 0xFFFFFFFFu) {
             const int o = atomicAdd(&s_cnt, 1);
-            if (o < keep) row[o] = tl[r];
+            if (o < keep) row[o] = s_t[x];
         }
     }
     __syncthreads();
     for (int x = min(s_cnt, keep) + threadIdx.x; x < keep; x += blockDim.x) row[x] = -1;
 #pragma unroll
-    for (int r = 0; r < 2; r++) {
-        const int j = threadIdx.x + r * 512;
+    for (int r = 0; r < 4; r++) {
+        const int j = threadIdx.x + r * 256;
         if (j < kprev) row[keep + j] = pv[r];
     }
 }

@@ -907,9 +907,9 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                         launches++;
                         trim1(idx->surv.as<int32_t>(), ostride, ostride, reinterpret_cast<const uint32_t *>(idx->fin.p));
                     } else {  // 32-bit LB keys, radix select in shared memory
-                        const size_t sm = (size_t)4 * LTt;
+                        const size_t sm = (size_t)8 * LTt;
                         set_smem((const void *)tau_trim_big_kernel<S>, sm);
-                        tau_trim_big_kernel<S><<<nseg, 512, sm, idx->stream>>>(
+                        tau_trim_big_kernel<S><<<nseg, 256, sm, idx->stream>>>(
                             idx->tauc.as<int32_t>(), LT, LTt, keep, kpv, idx->lb.as<V>(), d_meta, nl, tlb);
                     }
                     CHECK_LAUNCH();
