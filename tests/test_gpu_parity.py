@@ -603,3 +603,68 @@ def test_stream_fp16_postings_saturate(pkg, orc):
     oid, od = orc.knn(wl, mode="f32", threads=THREADS)
     np.testing.assert_array_equal(ids, oid)
     np.testing.assert_array_equal(dists, od)
+
+
+# ---------------------------------------------------------------------------
+# full size, in the launch configuration bench.py times (BASELINE configs[2..4])
+# ---------------------------------------------------------------------------
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg,dtype", [("C3", "i16"), ("C3", "f32"), ("C5", "f32")])
+def test_streams_full_size_sampled(pkg, orc, cfg, dtype):
+    """C3 / C5 at full size through the stream calls the bench times: every
+    master query of every sensor in one batch, ticks through the reused ring;
+    sampled streams equal the oracle's brute-force kNN bit for bit."""
+    wl = synth.make_workload(cfg, dtype, step=0, consecutive=True)
+    D = wl.D
+    rng = np.random.default_rng(11)
+    sample = np.sort(rng.choice(wl.n_mq, size=6, replace=False)).tolist()
+    mode = None if dtype == "i16" else "f32"
+
+    def check(ws, ids, dists):
+        oid, od = orc.knn(ws, mode=mode, mq_subset=sample, threads=THREADS)
+        np.testing.assert_array_equal(ids[sample], oid)
+        if dtype == "i16":
+            np.testing.assert_array_equal(dists[sample].astype(np.int64), od)
+        else:
+            np.testing.assert_array_equal(dists[sample], od)
+
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        with pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor) as st:
+            ids, dists = st.first
+            check(wl, ids, dists)
+            ws = wl
+            for s in (1, 2):
+                ws = synth.make_workload(cfg, dtype, step=s, consecutive=True)
+                ids, dists, stt = st.step(np.ascontiguousarray(ws.queries[:, D - 1]), stats=True)
+                assert stt["survivors"] < stt["candidates"]
+            check(ws, ids, dists)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_c4_full_size_sampled(pkg, orc, dtype):
+    """C4 at full size (1e8 points, 16 master queries, one call as the bench
+    times it): pruning equals the GPU's exhaustive search, every returned
+    distance is the oracle's DTW of that segment, and no sampled candidate
+    beats the k-th result."""
+    wl = synth.make_workload("C4", dtype)
+    rhos = wl.rhos()
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        ids, dists, st = idx.knn(wl.queries, wl.lengths, wl.k, stats=True)
+        bi, bd = idx.knn(wl.queries[:2], wl.lengths, wl.k, no_prune=True)
+        np.testing.assert_array_equal(ids[:2], bi)
+        np.testing.assert_array_equal(dists[:2], bd)
+        rng = np.random.default_rng(7)
+        for j in range(0, wl.n_mq, 3):
+            for i, d in enumerate(wl.lengths):
+                q = wl.queries[j, wl.D - d:]
+                ex = orc.dtw_list(wl.series, q, rhos[i], ids[j, i])
+                if dtype == "f32":
+                    ex = ex[0]
+                np.testing.assert_array_equal(dists[j, i].astype(ex.dtype), ex)
+                ts = rng.integers(0, len(wl.series) - d + 1, size=256)
+                g = idx.dtw(0, q, rhos[i], ts)
+                kth = (dists[j, i, -1], ids[j, i, -1])
+                for t, v in zip(ts.tolist(), g.tolist()):
+                    assert (v, t) >= kth or t in ids[j, i]
+    assert st["survivors"] < st["candidates"]
