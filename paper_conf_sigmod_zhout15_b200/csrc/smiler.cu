@@ -1026,7 +1026,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 launches++;
             } else if (ndw_max > 0 && sctx && sctx->mode == 1) {
                 // continuous step, static w: SW_0 (EQ + EC) and SW_1..SW_rho (EQ only)
-                dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
+                dim3 grid((unsigned)((ndw_max + 128 * SMILER_INC_TILES - 1) / (128 * SMILER_INC_TILES)), (unsigned)B);
                 size_t smem = 3 * sizeof(V) * D;
                 auto go = [&](auto kern, auto *pb) {
                     set_smem((const void *)kern, smem);
