@@ -29,6 +29,9 @@
 #ifndef SMILER_DIAG_UNROLL2
 #define SMILER_DIAG_UNROLL2 0
 #endif
+#ifndef SMILER_DIAG_SPLIT2
+#define SMILER_DIAG_SPLIT2 1  // lb_diag w = 16: local chunk sums + one uniform branch instead of slot rotation
+#endif
 #ifndef SMILER_INC_TILES
 #define SMILER_INC_TILES 4  // 128-DW tiles per CTA of the incremental a3 kernel (1: 7.79 ms, 4: 7.00 ms on C5)
 #endif
@@ -949,13 +952,26 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
         // chunk always accumulates into slots 0..BC-1 and the slot arrays are
         // rotated by BC afterwards (identity again after W / BC chunks).
         constexpr int NCH = W / BC;
+        // two chunks (w = 16): the chunk accumulates into local sums that one
+        // uniform branch adds to slots 0..7 or 8..15 (no slot rotation)
+        constexpr bool SPLIT2 = SMILER_DIAG_SPLIT2 && NCH == 2;
 #pragma unroll 1
         for (int h = 0; h < NCH; h++) {
             const int b0 = h * BC;
             const int nv = nrow - b0;
+            V te2[BC], tc2[BC];
+            if constexpr (SPLIT2) {
+#pragma unroll
+                for (int b = 0; b < BC; b++) te2[b] = tc2[b] = (V)0;
+            }
             auto acc = [&](int bb, V eq, V ec) {
-                se[bb] += eq;
-                sc[bb] += ec;
+                if constexpr (SPLIT2) {
+                    te2[bb] += eq;
+                    tc2[bb] += ec;
+                } else {
+                    se[bb] += eq;
+                    sc[bb] += ec;
+                }
             };
             const int pb = D - W - j * W - b0 - (BC - 1);
             if (nv >= BC) {  // full chunk: aligned 16-byte window loads
@@ -970,15 +986,24 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                     wu[k] = u.x, wu[k + 1] = u.y, wu[k + 2] = u.z, wu[k + 3] = u.w;
                     wl[k] = l.x, wl[k + 1] = l.y, wl[k + 2] = l.z, wl[k + 3] = l.w;
                 }
-#if SMILER_LB_FOLD
-                posting_chunk_w_fold<V, W, BC, WL, W>(c, U, L, wq, wu, wl, se, sc);
-#else
-                posting_chunk_w<V, W, BC, false, WL>(c, U, L, wq, wu, wl, BC, acc);
-#endif
+                if constexpr (SPLIT2)
+                    posting_chunk_w_fold<V, W, BC, WL, BC>(c, U, L, wq, wu, wl, te2, tc2);
+                else if constexpr (SMILER_LB_FOLD)
+                    posting_chunk_w_fold<V, W, BC, WL, W>(c, U, L, wq, wu, wl, se, sc);
+                else
+                    posting_chunk_w<V, W, BC, false, WL>(c, U, L, wq, wu, wl, BC, acc);
             } else if (nv > 0) {
                 posting_chunk<V, W, BC, true>(c, U, L, sqq + qshift, squ + qshift, sql + qshift, pb, nv, acc);
             }
-            if (NCH > 1) {  // rotate the slots left by BC
+            if constexpr (SPLIT2) {
+                if (h == 0) {
+#pragma unroll
+                    for (int b = 0; b < BC; b++) se[b] += te2[b], sc[b] += tc2[b];
+                } else {
+#pragma unroll
+                    for (int b = 0; b < BC; b++) se[BC + b] += te2[b], sc[BC + b] += tc2[b];
+                }
+            } else if (NCH > 1) {  // rotate the slots left by BC
                 V te[BC], tc[BC];
 #pragma unroll
                 for (int b = 0; b < BC; b++) te[b] = se[b], tc[b] = sc[b];
