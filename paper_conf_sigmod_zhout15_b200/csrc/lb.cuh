@@ -308,6 +308,39 @@ __device__ __forceinline__ void posting_chunk(const V (&c)[W], const V (&U)[W], 
 // SWs overlap in w-1 positions, so one chunk needs w+BC-1 MQ positions
 // {q, U(Q), L(Q)} loaded once into registers (no shared-memory load per term).
 // 8 ALU ops per (b, r, j) term pair.  Output post[mq][b][r] = {P_EQ, P_EC}.
+// One disjoint window (w consecutive points of the series or an envelope) into
+// registers: 16-byte vector loads when the window is 16-byte aligned (sensors
+// start on 64-element boundaries, so every DW of w >= 4 f32 / w >= 8 i16 is).
+template <typename S, typename V, int W>
+__device__ __forceinline__ void load_dw(const S *p, V (&o)[W]) {
+    if constexpr (std::is_same<S, float>::value && W % 4 == 0) {
+        if ((reinterpret_cast<uintptr_t>(p) & 15) == 0) {
+#pragma unroll
+            for (int q = 0; q < W / 4; q++) {
+                const float4 v = __ldg(reinterpret_cast<const float4 *>(p) + q);
+                o[4 * q] = v.x, o[4 * q + 1] = v.y, o[4 * q + 2] = v.z, o[4 * q + 3] = v.w;
+            }
+            return;
+        }
+    } else if constexpr (std::is_same<S, int16_t>::value && W % 8 == 0) {
+        if ((reinterpret_cast<uintptr_t>(p) & 15) == 0) {
+#pragma unroll
+            for (int q = 0; q < W / 8; q++) {
+                const int4 v = __ldg(reinterpret_cast<const int4 *>(p) + q);
+                const int32_t wv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                for (int h = 0; h < 4; h++) {
+                    o[8 * q + 2 * h] = (V)(int16_t)(wv[h] & 0xFFFF);
+                    o[8 * q + 2 * h + 1] = (V)(int16_t)(wv[h] >> 16);
+                }
+            }
+            return;
+        }
+    }
+#pragma unroll
+    for (int j = 0; j < W; j++) o[j] = (V)p[j];
+}
+
 // ---------------------------------------------------------------------------
 template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
@@ -341,12 +374,9 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
         const int nmir = m.prows - n_sw;  // mirrored leading rows (TMA ring)
         const int64_t base = m.series_off + r * W;
         V c[W], U[W], L[W];
-#pragma unroll
-        for (int j = 0; j < W; j++) {
-            c[j] = (V)series[base + j];
-            U[j] = (V)UC[base + j];
-            L[j] = (V)LC[base + j];
-        }
+        load_dw<S, V, W>(series + base, c);
+        load_dw<S, V, W>(UC + base, U);
+        load_dw<S, V, W>(LC + base, L);
         int b0 = 0;
         auto put = [&](int b, V eq, V ec) {  // ring cursor 0 at a full build: row b
             PV *o = oe + (int64_t)b * pst;
@@ -422,12 +452,9 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
     PV *oe = post + m.post_off + r;
     const int64_t base = m.series_off + r * W;
     V c[W], U[W], L[W];
-#pragma unroll
-    for (int j = 0; j < W; j++) {
-        c[j] = (V)series[base + j];
-        U[j] = (V)UC[base + j];
-        L[j] = (V)LC[base + j];
-    }
+    load_dw<S, V, W>(series + base, c);
+    load_dw<S, V, W>(UC + base, U);
+    load_dw<S, V, W>(LC + base, L);
     const int64_t pst = m.pstride;
     const int64_t plane = (int64_t)m.prows * pst;
     const int nmir = m.prows - n_ring;  // mirrored leading physical rows (TMA ring)
