@@ -926,21 +926,37 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
     }
     const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
     const int64_t R0 = Rb - HALO;  // DW of tile column 0
-    // 8 iterations' loads in flight before their shared-memory stores
-#pragma unroll 8
-    for (int idx = threadIdx.x; idx < NC * W; idx += NT) {
-        const int col = idx / W, jj = idx % W;
+    // 4 consecutive points per item (16-byte f32 / 8-byte i16 vector loads:
+    // sensors start on 64-element boundaries), 16-byte shared-memory stores
+    // (DS is a multiple of 4); 4 iterations' loads in flight
+    constexpr int W4 = W / 4;
+#pragma unroll 4
+    for (int idx = threadIdx.x; idx < NC * W4; idx += NT) {
+        const int col = idx / W4, q = idx % W4;
         const int64_t rp = R0 + col;
-        V c = (V)0, u = (V)0, l = (V)0;
+        V4 c = {}, u = {}, l = {};
         if (rp >= 0 && rp < m.n_dw) {
-            const int64_t g = m.series_off + rp * W + jj;
-            c = (V)series[g];
-            u = (V)UC[g];
-            l = (V)LC[g];
+            const int64_t g = m.series_off + rp * W + 4 * q;
+            if constexpr (std::is_same<S, float>::value) {
+                const float4 a = __ldg(reinterpret_cast<const float4 *>(series + g));
+                const float4 b = __ldg(reinterpret_cast<const float4 *>(UC + g));
+                const float4 e = __ldg(reinterpret_cast<const float4 *>(LC + g));
+                c = make_float4(a.x, a.y, a.z, a.w);
+                u = make_float4(b.x, b.y, b.z, b.w);
+                l = make_float4(e.x, e.y, e.z, e.w);
+            } else {
+                auto unpack = [](uint2 v) {
+                    return make_int4((int16_t)(v.x & 0xFFFF), (int16_t)((int32_t)v.x >> 16),
+                                     (int16_t)(v.y & 0xFFFF), (int16_t)((int32_t)v.y >> 16));
+                };
+                c = unpack(__ldg(reinterpret_cast<const uint2 *>(series + g)));
+                u = unpack(__ldg(reinterpret_cast<const uint2 *>(UC + g)));
+                l = unpack(__ldg(reinterpret_cast<const uint2 *>(LC + g)));
+            }
         }
-        cs[col * DS + jj] = c;
-        us[col * DS + jj] = u;
-        ls[col * DS + jj] = l;
+        *reinterpret_cast<V4 *>(cs + col * DS + 4 * q) = c;
+        *reinterpret_cast<V4 *>(us + col * DS + 4 * q) = u;
+        *reinterpret_cast<V4 *>(ls + col * DS + 4 * q) = l;
     }
     __syncthreads();
     const int x = threadIdx.x;
