@@ -82,6 +82,10 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
     }
 }
 
+#ifndef SMILER_DTW_STAGE_UNROLL
+#define SMILER_DTW_STAGE_UNROLL 4  // candidate-row loads in flight per lane before their stores
+#endif
+constexpr int kStageUnroll = SMILER_DTW_STAGE_UNROLL;
 #ifndef SMILER_DTW_CPASYNC
 #define SMILER_DTW_CPASYNC 0  // 1: f32 candidate rows staged with cp.async, double-buffered (measured slower: occupancy)
 #endif
@@ -186,7 +190,7 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
             } else {
                 __syncwarp();
                 const bool in_row = (j0 + lane) < d;
-#pragma unroll 4
+#pragma unroll kStageUnroll
                 for (int l = 0; l < 32; l++) {
                     int tl = __shfl_sync(0xffffffffu, t, l);
                     V v = (V)0;
