@@ -384,14 +384,23 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
         const int4 *vb = reinterpret_cast<const int4 *>(a0 & ~(uintptr_t)15);
         ta = t0 - (int64_t)((a0 & 15) >> 1);
         const int r0 = (int)(t0 - ta), r1 = (int)(t1 - ta);  // block range relative to ta (< 2^31)
+        // all vector loads of the thread first (4 x 16 B in flight), then the compares
+        constexpr int NV = kFiltItems / 8;
+        int4 rawv[NV];
 #pragma unroll
-        for (int it = 0; it < kFiltItems / 8; it++) {
+        for (int it = 0; it < NV; it++) {
+            const int vi = it * kFiltThreads + threadIdx.x;
+            const int rv = vi * 8;
+            rawv[it] = (rv < r1 && rv + 8 > r0) ? __ldg(vb + vi) : make_int4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int it = 0; it < NV; it++) {
             const int vi = it * kFiltThreads + threadIdx.x;
             const int rv = vi * 8;
             if (rv < r1 && rv + 8 > r0) {
                 const int lo = max(0, r0 - rv), hi = min(8, r1 - rv);
                 const uint32_t vm = ((1u << hi) - 1u) & ~((1u << lo) - 1u);
-                const int4 raw = vb[vi];
+                const int4 raw = rawv[it];
                 const __half2 *h2 = reinterpret_cast<const __half2 *>(&raw);
                 uint32_t kb = 0;
 #pragma unroll
