@@ -83,7 +83,7 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
 }
 
 #ifndef SMILER_DTW_STAGE_UNROLL
-#define SMILER_DTW_STAGE_UNROLL 4  // candidate-row loads in flight per lane before their stores
+#define SMILER_DTW_STAGE_UNROLL 16  // candidate-row loads in flight per lane before their stores
 #endif
 constexpr int kStageUnroll = SMILER_DTW_STAGE_UNROLL;
 #ifndef SMILER_DTW_CPASYNC
@@ -190,12 +190,18 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
             } else {
                 __syncwarp();
                 const bool in_row = (j0 + lane) < d;
-#pragma unroll kStageUnroll
-                for (int l = 0; l < 32; l++) {
-                    int tl = __shfl_sync(0xffffffffu, t, l);
-                    V v = (V)0;
-                    if (tl >= 0 && in_row) v = (V)cs[tl + j0 + lane];
-                    s_c[lane][l] = v;
+                // kStageUnroll loads in flight before their stores (explicitly
+                // batched: the compiler otherwise alternates load / store)
+#pragma unroll 1
+                for (int l0 = 0; l0 < 32; l0 += kStageUnroll) {
+                    S vals[kStageUnroll];
+#pragma unroll
+                    for (int q = 0; q < kStageUnroll; q++) {
+                        const int tl = __shfl_sync(0xffffffffu, t, l0 + q);
+                        vals[q] = (tl >= 0 && in_row) ? __ldg(cs + tl + j0 + lane) : (S)0;
+                    }
+#pragma unroll
+                    for (int q = 0; q < kStageUnroll; q++) s_c[lane][l0 + q] = (V)vals[q];
                 }
                 __syncwarp();
             }
