@@ -1,6 +1,8 @@
 # Round-1 evidence for HEAD: bench lines (all configs), the default command's ncu launch list,
 # ncu --set full summaries of the top kernels (reports reduced on the box: gpurun_out cap 64 MiB)
-O=gpurun_out/r01e; mkdir -p $O
+O=${1:-gpurun_out/r01e}; mkdir -p $O
+timeout 1500 python -m pytest tests -m gpu -q -x -p no:cacheprovider > $O/pytest_gpu.txt 2>&1; tail -2 $O/pytest_gpu.txt
+timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print(\"smoke ok\")" > $O/smoke.txt 2>&1
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,clocks.mem --format=csv > $O/gpu.txt
 timeout 900 python bench.py > $O/bench_C2_f32.json 2> $O/bench_C2_f32.err
 timeout 900 python bench.py --dtype i16 > $O/bench_C2_i16.json 2> $O/bench_C2_i16.err
