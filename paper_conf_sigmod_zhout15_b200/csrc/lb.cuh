@@ -976,14 +976,17 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
 #if SMILER_DIAG_UNROLL2
 #pragma unroll 2
 #endif
-    for (int j = 0; j < mmax; j++) {
-        const int col = x + HALO - j;  // DW r - j
+    // DW r - j of row j: one loop-carried pointer (us / ls at fixed offsets),
+    // so the row prologue does not re-derive tid and the tile base each row
+    const V *cp = cs + (x + HALO) * DS;
+    if (P.k < 0) emit_rows = save_rows = 0;  // timing experiment: main loop only
+    for (int j = 0; j < mmax; j++, cp -= DS) {
         V c[W], U[W], L[W];
 #pragma unroll
         for (int jj = 0; jj < W; jj += 4) {
-            const V4 a = *reinterpret_cast<const V4 *>(cs + col * DS + jj);
-            const V4 u = *reinterpret_cast<const V4 *>(us + col * DS + jj);
-            const V4 l = *reinterpret_cast<const V4 *>(ls + col * DS + jj);
+            const V4 a = *reinterpret_cast<const V4 *>(cp + jj);
+            const V4 u = *reinterpret_cast<const V4 *>(cp + kDiagCols * DS + jj);
+            const V4 l = *reinterpret_cast<const V4 *>(cp + 2 * kDiagCols * DS + jj);
             c[jj] = a.x, c[jj + 1] = a.y, c[jj + 2] = a.z, c[jj + 3] = a.w;
             U[jj] = u.x, U[jj + 1] = u.y, U[jj + 2] = u.z, U[jj + 3] = u.w;
             L[jj] = l.x, L[jj + 1] = l.y, L[jj + 2] = l.z, L[jj + 3] = l.w;
@@ -1056,7 +1059,6 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                 for (int b = 0; b < BC; b++) se[W - BC + b] = te[b], sc[W - BC + b] = tc[b];
             }
         }
-        if (P.k < 0) continue;  // timing experiment: main loop only
         // rows q_i - 1: compose IQ i from the values saved after row q_i - 2
         // (slots b > r_i) and the current sums (b <= r_i), then write it
         if (emit_rows >> j & 1ull) {
