@@ -1065,9 +1065,11 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
             for (int i = 0; i < nl; i++) {
                 const int qi = P.len[i] / W, ri = P.len[i] % W;
                 if (j == qi - 1) {
+                    // saved[] is still all zero at row 0 (the first save follows
+                    // row 0's emissions), so q_i = 1 needs no separate case
                     V v[W];
 #pragma unroll
-                    for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? saved[b] : (V)0) : lbpick(P, se[b], sc[b]);
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? saved[b] : lbpick(P, se[b], sc[b]);
                     diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }
