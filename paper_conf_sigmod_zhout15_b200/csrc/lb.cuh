@@ -745,7 +745,7 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 __device__ __forceinline__ __half lb_to_half(float v) { return __float2half_rd(v); }
 __device__ __forceinline__ __half lb_to_half(int32_t v) { return __int2half_rd(v); }
 
-template <typename V, int W>
+template <typename V, int W, bool FASTMASK = true>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
                                           V *lb, int32_t *tauc, int mq, int bx = -1) {
     static_assert(W <= 32, "slot mask is 32-bit");
@@ -756,10 +756,14 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     const int64_t t0 = s0 - d;
     // valid slots b: tmin <= t0 + b < tend, as one bit mask (two 64-bit
     // compares per emission instead of two per slot)
-    const int blo = (int)max((int64_t)0, min((int64_t)W, tmin - t0));
-    const int bhi = (int)max((int64_t)0, min((int64_t)W, tend - t0));
-    const uint32_t vmask = (uint32_t)(((1ull << bhi) - 1ull) & ~((1ull << blo) - 1ull));
     constexpr uint32_t kAll = (uint32_t)((1ull << W) - 1ull);
+    uint32_t vmask = kAll;  // interior slots (all but the tiles at a range end)
+    // (FASTMASK = false: always the general form; lb_diag w = 16 measured faster so)
+    if (!FASTMASK || t0 < tmin || t0 + W > tend) {
+        const int blo = (int)max((int64_t)0, min((int64_t)W, tmin - t0));
+        const int bhi = (int)max((int64_t)0, min((int64_t)W, tend - t0));
+        vmask = (uint32_t)(((1ull << bhi) - 1ull) & ~((1ull << blo) - 1ull));
+    }
     if (P.fuse) {  // a6 here: keep LB <= thr (ties survive), warp-aggregated append
         const int seg = mq * P.n_len + i;
         const uint32_t th = P.thr[seg];
@@ -1070,7 +1074,7 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
                     V v[W];
 #pragma unroll
                     for (int b = 0; b < W; b++) v[b] = b > ri ? saved[b] : lbpick(P, se[b], sc[b]);
-                    diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
+                    diag_emit<V, W, (W <= 8)>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }
         }
