@@ -38,6 +38,9 @@
 #ifndef SMILER_TMA_SYNC2
 #define SMILER_TMA_SYNC2 1  // TMA ring scan: one CTA barrier per two CSG rows
 #endif
+#ifndef SMILER_TAU_PACKED
+#define SMILER_TAU_PACKED 1  // tau-set keys: LB_w bits with the slot in the low bits
+#endif
 #ifndef SMILER_TMA_EMPTYBAR
 #define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower)
 #endif
@@ -831,6 +834,41 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const int unit = (bx >= 0 ? bx : (int)blockIdx.x) * nw + warp;  // tau units are warps of tile bx
     int32_t *dst = tauc + (int64_t)(mq * P.n_len + i) * P.LT + (int64_t)unit * P.E;
+#if SMILER_TAU_PACKED
+    // The E (near-)smallest LB_w of the warp, one 32-bit key per slot: the
+    // LB_w bits (non-negative float or int: unsigned order = value order) with
+    // their lowest SB bits replaced by the slot b.  The minimum key names its
+    // slot directly (no per-slot hit search), and the stored bound
+    // (bits & ~mask) is never above the slot's LB_w.  The tau set only has to
+    // hold >= k verified candidates for tau to bound the k-th NN key (R8), so
+    // choosing among LB_w equal up to the low SB bits is still valid.
+    constexpr int SB = W <= 4 ? 2 : (W <= 8 ? 3 : (W <= 16 ? 4 : 5));
+    constexpr uint32_t SM = (1u << SB) - 1u;
+    uint32_t kb[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) kb[b] = (vmask >> b & 1u) ? ((key_bits(v[b]) & ~SM) | (uint32_t)b) : 0xFFFFFFFFu;
+    uint32_t best = kb[0];
+#pragma unroll
+    for (int b = 1; b < W; b++) best = min(best, kb[b]);
+    for (int e = 0; e < P.E; e++) {
+        const uint32_t win = __reduce_min_sync(0xffffffffu, best);
+        const int wl = __ffs(__ballot_sync(0xffffffffu, best == win)) - 1;
+        const int tw = __shfl_sync(0xffffffffu, (int)t0, wl) + (int)(win & SM);
+        if (lane == wl && e + 1 < P.E) {
+            best = 0xFFFFFFFFu;
+#pragma unroll
+            for (int b = 0; b < W; b++) {
+                kb[b] = kb[b] == win ? 0xFFFFFFFFu : kb[b];
+                best = min(best, kb[b]);
+            }
+        }
+        if (lane == 0) {
+            dst[e] = win != 0xFFFFFFFFu ? tw : -1;
+            if (P.taulb) P.taulb[dst - tauc + e] = win != 0xFFFFFFFFu ? (win & ~SM) : win;
+        }
+    }
+}
+#else
     // The E smallest (LB_w, t) keys of the warp with 32-bit compares only: t
     // grows with the slot b inside a thread and with the lane across the warp,
     // so among equal LB_w bits the lowest lane, then the lowest b, has the
@@ -862,6 +900,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
         }
     }
 }
+#endif
 
 // ---------------------------------------------------------------------------
 // a3+a4 fused, diagonal form (one-shot batches, default).  Thread x owns the
