@@ -38,6 +38,9 @@
 #ifndef SMILER_TMA_SYNC2
 #define SMILER_TMA_SYNC2 1  // TMA ring scan: one CTA barrier per two CSG rows
 #endif
+#ifndef SMILER_DIAG_MINB8
+#define SMILER_DIAG_MINB8 6  // lb_diag CTAs per SM for w <= 8 (80 registers, no spills; 5: -0.4%, 4: -3%, 7: -5%)
+#endif
 #ifndef SMILER_TAU_PACKED
 #define SMILER_TAU_PACKED 1  // tau-set keys: LB_w bits with the slot in the low bits
 #endif
@@ -922,7 +925,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
 template <int W> struct DiagStride { static constexpr int v = (W == 4) ? 12 : W + 4; };
 
 template <typename S, int W>
-__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? 5 : 3))
+__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_MINB8 : 3))
     lb_diag_kernel(const S *series, const S *UC, const S *LC, const MQMeta *meta,
                    const typename Tr<S>::V4 *qtab, const QParams P, typename Tr<S>::V *lb,
                    int32_t *tauc) {
