@@ -78,6 +78,8 @@ class Workload:
     k: int                         # max(EKV)
     window: int                    # omega
     band: float                    # >= 1: absolute rho; in (0,1): rho_i = floor(band * d_i)
+    tails: Optional[List[np.ndarray]] = None  # held-out tail of each sensor (the MQs' source)
+    qoff: Optional[np.ndarray] = None         # int64 [n_mq]: tail offset of each MQ's first point
 
     @property
     def n_sensors(self) -> int:
@@ -96,6 +98,20 @@ class Workload:
 
     def rhos(self) -> List[int]:
         return band_to_rhos(self.band, self.lengths)
+
+    def queries_at(self, step: int) -> np.ndarray:
+        """The master queries after `step` more points of a continuous stream
+        (each MQ slides one point per step over its sensor's tail)."""
+        D = self.D
+        out = np.empty_like(self.queries)
+        for j in range(self.n_mq):
+            o = int(self.qoff[j]) + step
+            out[j] = self.tails[int(self.query_sensor[j])][o:o + D]
+        return out
+
+    def new_points(self, step: int) -> np.ndarray:
+        """The point each stream appends at continuous step `step` (>= 1)."""
+        return np.ascontiguousarray(self.queries_at(step)[:, self.D - 1])
 
 
 def band_to_rhos(band: float, lengths: Sequence[int]) -> List[int]:
@@ -147,7 +163,7 @@ def make_workload(name: str, dtype: str = "i16", *, n: Optional[int] = None,
     if not 0 <= step < STEP_MAX:
         raise ValueError("step must be in [0, %d)" % STEP_MAX)
     H = D + spread * mqs + STEP_MAX + 1
-    parts, queries, qs = [], [], []
+    parts, queries, qs, tails, qoff = [], [], [], [], []
     offsets = [0]
     for s in range(ns):
         z = sensor_series(cid, s, N, H, periods[s % len(periods)])
@@ -155,16 +171,19 @@ def make_workload(name: str, dtype: str = "i16", *, n: Optional[int] = None,
         parts.append(x[:N])
         offsets.append(offsets[-1] + N)
         tail = x[N:]
+        tails.append(tail)
         for j in range(mqs):
             off = spread * j + step
             queries.append(tail[off:off + D])
             qs.append(s)
+            qoff.append(off)
     series = np.concatenate(parts)
     return Workload(name=name, dtype=dtype, series=series,
                     offsets=np.asarray(offsets, dtype=np.int64),
                     queries=np.ascontiguousarray(np.stack(queries)),
                     query_sensor=np.asarray(qs, dtype=np.int32),
-                    lengths=lens, k=kk, window=w, band=bd)
+                    lengths=lens, k=kk, window=w, band=bd, tails=tails,
+                    qoff=np.asarray(qoff, dtype=np.int64))
 
 
 def random_walk_small(seed: int, n: int, dtype: str, lo: int = -40, hi: int = 40) -> np.ndarray:

@@ -358,3 +358,96 @@ def test_generator_is_seeded_and_shaped():
     assert c5.rhos() == [3, 6, 12, 25] and c5.n_mq == 6
     z = synth.sensor_series(2, 0, 10000, 100, 144)
     assert abs(z[:10000].mean()) < 1e-9 and abs(z[:10000].std() - 1) < 1e-9
+
+
+# --------------------------------------------------------------------------
+# P13 pins of the oracle's FLOAT paths: inputs x/8 (x small integers) make every
+# f32 / f64 operation of the oracle exact, so each float function must equal
+# its integer twin divided by 64 exactly -- and the integer twins are pinned
+# above (golden example, Eq. 5 shift sums, path enumeration).  A dropped term,
+# a wrong sign or index, a transposed operand or a wrong suffix offset in a
+# float function breaks the equality.
+# --------------------------------------------------------------------------
+def _dyadic_cases():
+    g = json.load(open(GOLD))
+    yield np.array(g["C"], np.int64), np.array(g["MQ"], np.int64), g["w"], g["rho"], [iq["d"] for iq in g["IQ"]]
+    rng = np.random.default_rng(1313)
+    for seed in range(4):
+        w = int(rng.integers(2, 9))
+        lengths = sorted(set(int(x) for x in rng.integers(w, 5 * w, size=3)))
+        D = lengths[-1]
+        n = int(rng.integers(D + 20, 260))
+        x = synth.random_walk_small(100 + seed, n + D, "i16", -40, 40).astype(np.int64)
+        yield x[:n], x[n:], w, int(rng.integers(0, 6)), lengths
+
+
+def test_postings_f64_equals_i64_over_64_dyadic(orc):
+    """orc_postings_f64 on x/8 inputs == orc_postings_i64 / 64."""
+    for c, mq, w, rho, _ in _dyadic_cases():
+        UC, LC = orc.envelope(c, rho)
+        UQ, LQ = orc.envelope(mq, rho)
+        PE, PC = orc.postings(c, UC, LC, mq, UQ, LQ, w)
+        f = lambda a: np.asarray(a, np.float64) / 8.0
+        FE, FC = orc.postings(f(c), f(UC), f(LC), f(mq), f(UQ), f(LQ), w)
+        assert FE.dtype == np.float64
+        np.testing.assert_array_equal(FE * 64.0, PE.astype(np.float64))
+        np.testing.assert_array_equal(FC * 64.0, PC.astype(np.float64))
+        assert PE.any() and PC.any()          # not a vacuous all-zero case
+
+
+def test_lb_f64_equals_i64_over_64_dyadic(orc):
+    """orc_lb_f64 (LB_EQ, LB_EC, LB_en of Thm 4.1; LB_w and its two sums of
+    Thm 4.3 / Eq. 5) on x/8 inputs == orc_lb_i64 / 64, for every t and d."""
+    for c, mq, w, rho, lengths in _dyadic_cases():
+        UC, LC = orc.envelope(c, rho)
+        UQ, LQ = orc.envelope(mq, rho)
+        f = lambda a: np.asarray(a, np.float64) / 8.0
+        for d in lengths:
+            li = orc.lower_bounds(c, UC, LC, mq, UQ, LQ, d, w)
+            lf = orc.lower_bounds(f(c), f(UC), f(LC), f(mq), f(UQ), f(LQ), d, w)
+            for key in ("eq", "ec", "en", "w", "weq", "wec"):
+                np.testing.assert_array_equal(lf[key] * 64.0, li[key].astype(np.float64), err_msg=key)
+            assert li["w"].any()
+            if rho > 0:   # rho = 0: U = L = the series, so both sums are sum (q - c)^2
+                assert (li["weq"] != li["wec"]).any()
+
+
+@pytest.mark.parametrize("mode", ["f32", "f64"])
+def test_knn_float_suffix_offsets_dyadic(orc, mode):
+    """orc_knn_f32 / orc_knn_f64 with item queries SHORTER than the MQ
+    (lengths [3, 5, 6], D = 6: IQ_i = the last d_i points) on x/8
+    inputs == orc_knn_i16 / 64 == the kNN of path-enumeration DTWs / 64."""
+    for trial in range(4):
+        rng = np.random.default_rng(600 + trial)
+        n = 40
+        xi = rng.integers(-30, 31, size=n + 6)
+        series_i, mq_i = xi[:n].astype(np.int16), xi[n:].astype(np.int16)
+        series_f, mq_f = (series_i / 8.0).astype(np.float32), (mq_i / 8.0).astype(np.float32)
+        lengths, rhos, k = [3, 5, 6], [1, 2, 1], 9
+        ids_i, d_i = orc.knn_one(series_i, mq_i, lengths, rhos, k)
+        ids_f, d_f = orc.knn_one(series_f, mq_f, lengths, rhos, k, mode=mode)
+        np.testing.assert_array_equal(ids_f, ids_i)
+        np.testing.assert_array_equal(d_f.astype(np.float64) * 64.0, d_i.astype(np.float64))
+        for li, (d, rho) in enumerate(zip(lengths, rhos)):
+            iq = [int(v) for v in mq_i[6 - d:]]
+            allk = sorted((dtw_by_paths(iq, [int(v) for v in series_i[t:t + d]], rho), t)
+                          for t in range(n - d + 1))[:k]
+            assert ids_f[li].tolist() == [t for _, t in allk]
+            assert (d_f[li].astype(np.float64) * 64.0).tolist() == [float(v) for v, _ in allk]
+
+
+@pytest.mark.parametrize("mode", ["f32", "f64"])
+def test_knn_float_owned_range_dyadic(orc, mode):
+    """The t_lo / t_hi candidate window of orc_knn_f32/f64 (window-range shards,
+    R24) equals brute force restricted to that window."""
+    xi = synth.random_walk_small(77, 300, "i16", -40, 40)
+    xf = synth.random_walk_small(77, 300, "f32", -40, 40)
+    lengths, rhos, k = [8, 13], [2, 3], 6
+    for t_lo, t_hi in ((0, 250), (17, 120), (100, 101)):
+        ids_i, d_i = orc.knn_one(xi[:250], xi[250:263], lengths, rhos, k, t_lo=t_lo, t_hi=t_hi)
+        ids_f, d_f = orc.knn_one(xf[:250], xf[250:263], lengths, rhos, k, mode=mode, t_lo=t_lo, t_hi=t_hi)
+        np.testing.assert_array_equal(ids_f, ids_i)
+        fin = ids_i >= 0
+        np.testing.assert_array_equal(d_f[fin].astype(np.float64) * 64.0, d_i[fin].astype(np.float64))
+        assert np.isinf(d_f[~fin]).all()
+        assert ((ids_i[fin] >= t_lo) & (ids_i[fin] < t_hi)).all()
