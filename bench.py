@@ -277,13 +277,13 @@ class Runner:
         self.op.tau_mult = args.tau_mult
         self.op_fast = pkg.KnnOpts(no_prune=0, timing=0, mq_chunk=0, two_level=int(args.two_level))
         self.op_fast.tau_mult = args.tau_mult
-        # A/B switches of the library (smiler_knn_opts.reserved[0], include/smiler.h); not a product knob
+        # A/B: kernel-path variant (smiler_knn_opts.variant, same results) and tau-set trim size
         ab = int(os.environ.get("SMILER_AB", "0"))
-        self.op.reserved[0] = ab
-        self.op_fast.reserved[0] = ab
-        keep = int(os.environ.get("SMILER_TAU_KEEP", "0"))   # reserved[2]: tau-set trim multiple (A/B)
-        self.op.reserved[2] = keep
-        self.op_fast.reserved[2] = keep
+        self.op.variant = ab
+        self.op_fast.variant = ab
+        keep = int(os.environ.get("SMILER_TAU_KEEP", "0"))
+        self.op.tau_keep = keep
+        self.op_fast.tau_keep = keep
         # C5 is a continuous prediction stream: every step is one tick of all
         # streams (each MQ advances one point); after the first tick the previous
         # tick's neighbours seed the thresholds (smiler_knn_step)

@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define SMILER_ABI_VERSION 2
+#define SMILER_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define SMILER_API __attribute__((visibility("default")))
@@ -97,10 +97,17 @@ typedef struct smiler_knn_opts {
                          > 0 = that many, < 0 = none.  With no tile set in a continuous
                          step the thresholds exist before the scan, and the LB kernel
                          filters as it goes (a4+a6 fused, no LB_w array) */
-    int32_t reserved[3];  /* 0; reserved[0] selects internal A/B variants in experiments (7: stream
-                             ring without TMA, 8: one tile per group-scan CTA, 9: radix-select tau-set trim); reserved[2]: tau-set trim
-                             (kept tile candidates per item query, in multiples of k; 0 = default
-                             8 one-shot / 1 continuous, < 0 = verify every tile candidate) */
+    int32_t variant;  /* kernel-path selector for tests and A/B timing; every variant computes
+                         the same (exact) result: 0 = automatic, 1 = row-form fused LB kernel,
+                         2 = scalar (not fp32x2-packed) diagonal LB kernel for F32,
+                         7 = stream ring scanned without TMA, 8 = one tile per ring-scan CTA,
+                         9 = radix-select tau-set trim, 10 = two-stage tau-set trim.  Any other
+                         value is EINVAL */
+    int32_t reserved; /* must be 0 (EINVAL otherwise) */
+    int32_t tau_keep; /* tau-set trim (reading R8): tile candidates kept per item query before
+                         the tau DTWs, in multiples of k; 0 = default (8 one-shot, 1 in a
+                         continuous step), < 0 = verify every tile candidate.  Any choice is a
+                         valid tau set; only the threshold's tightness changes */
     uint64_t *shared_tau; /* NULL, or a running threshold shared by calls that split ONE
                          search (window-range shards of the same series and master
                          queries): [n_mq][n_len] keys
@@ -155,7 +162,8 @@ enum {
  * device        CUDA device ordinal; cuda_stream a cudaStream_t (NULL = legacy
  *               default stream) used by every call on the handle.
  * out           receives the handle.
- * Errors: EINVAL (n_total < 1, bad offsets, window < 1, band < 0),
+ * Errors: EINVAL (n_total < 1, bad offsets, a sensor longer than 2^31 - 1
+ *         points (candidate starts are 32-bit), window < 1, band < 0),
  *         ERANGE (I16 value with |x| > 1023), ENOMEM, ECUDA.
  */
 SMILER_API int smiler_index_build(const void *series, smiler_dtype dtype, int64_t n_total,
@@ -186,10 +194,17 @@ SMILER_API int smiler_index_build_shard(const void *slice, smiler_dtype dtype, i
  * Eq. 21-24) and top-k selection (a8).
  *
  * queries       [n_mq][D] master queries, oldest -> newest, same
- *               dtype as the index; D = lengths[n_len-1].
+ *               dtype as the index; D = lengths[n_len-1].  I16 values must
+ *               satisfy |x| <= 1023 (R17): host queries are checked before any
+ *               work (ERANGE); device queries are checked by the query-prep
+ *               kernel, which clamps them for that call and raises a sticky
+ *               flag reported as ERANGE by this call when it synchronises
+ *               (host outputs or stats) or else by the next call on the handle.
  * query_sensor  [n_mq] sensor searched by each MQ; NULL -> 0.
  * lengths       ELV [n_len], strictly increasing, lengths[0] >= 1, each <= the
- *               sensor's length, lengths[n_len-1] = D <= 1024, n_len <= 16.
+ *               sensor's length, lengths[n_len-1] = D <= 1024 (F32) or <= 256
+ *               (I16: every DTW and bound then fits int32 exactly, R17),
+ *               n_len <= 16.
  *               Item query IQ_i = the last lengths[i] points of the MQ
  *               (P:859-860).
  * k             max(EKV), 1 <= k <= 1024; smaller k are prefixes.
@@ -202,7 +217,8 @@ SMILER_API int smiler_index_build_shard(const void *slice, smiler_dtype dtype, i
  * stats         may be NULL.
  * Results are exactly the brute-force kNN (filtering never dismisses a true
  * neighbour: Thm 4.1/4.3 with tau_i >= the k-th distance, R8, R16).
- * Errors: EINVAL, ENOMEM, ECUDA.
+ * Errors: EINVAL (bad argument, non-zero opts->reserved, unknown variant),
+ *         ERANGE (I16 query value outside [-1023, 1023]), ENOMEM, ECUDA.
  */
 SMILER_API int smiler_knn(smiler_index *idx, const void *queries, const int32_t *query_sensor,
                int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,

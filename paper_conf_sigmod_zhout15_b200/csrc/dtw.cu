@@ -21,6 +21,8 @@
 // i < 1 or i > d are inf (Eq. 22/23).  For f32 those cells get a query value
 // of +inf, which makes every such cell +inf without a mask; for int32 the
 // first and last rho rows run a masked variant.
+#include <map>
+#include <mutex>
 #include <type_traits>
 #include <utility>
 
@@ -249,28 +251,43 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
     }
 }
 
+// Per-device launch configuration of one dtw_kernel instantiation: the
+// shared-memory attribute is a per-device setting and the grid follows the
+// device's SM count, so both are kept per device (and guarded: handles on
+// different devices / threads are independent).
+struct DtwLaunchCfg {
+    int occ = 0, sms = 0;
+};
+template <typename S, int RHO>
+static DtwLaunchCfg dtw_cfg() {
+    using V = typename Tr<S>::V;
+    constexpr int NB = dtw_cbufs<S>();
+    static std::mutex mu;
+    static std::map<int, DtwLaunchCfg> per_dev;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = per_dev.find(dev);
+    if (it != per_dev.end()) return it->second;
+    DtwLaunchCfg c;
+    cudaFuncSetAttribute(dtw_kernel<S, RHO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + NB * 32 * 33) * sizeof(V)));
+    cudaDeviceGetAttribute(&c.sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c.occ, dtw_kernel<S, RHO>, kDtwThreads,
+                                                  (size_t)kDtwWarps * (dtw_qstage(256, RHO) + NB * 32 * 33) * sizeof(V));
+    if (c.occ < 1) c.occ = 1;
+    if (c.sms < 1) c.sms = 1;
+    per_dev[dev] = c;
+    return c;
+}
+
 template <typename S, int RHO>
 static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
     using V = typename Tr<S>::V;
     constexpr int NB = dtw_cbufs<S>();
     size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + NB * 32 * 33) * sizeof(V);
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(dtw_kernel<S, RHO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + NB * 32 * 33) * sizeof(V)));
-        attr = true;
-    }
-    static int occ = 0, sms = 0;
-    if (!occ) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &occ, dtw_kernel<S, RHO>, kDtwThreads,
-            (size_t)kDtwWarps * (dtw_qstage(256, RHO) + NB * 32 * 33) * sizeof(V));
-        if (occ < 1) occ = 1;
-    }
-    if (grid <= 0) grid = sms * occ;
+    const DtwLaunchCfg c = dtw_cfg<S, RHO>();
+    if (grid <= 0) grid = c.sms * c.occ;
     dtw_kernel<S, RHO><<<grid, kDtwThreads, smem, st>>>(p);
 }
 

@@ -2,6 +2,7 @@
 // libsmiler.so (not part of the C ABI; see include/smiler.h).
 #pragma once
 #include <cuda_runtime.h>
+#include <math.h>
 #include <stdint.h>
 
 #include "../../include/smiler.h"
@@ -58,7 +59,9 @@ struct QParams {
     int ring_cursor;  // continuous streams: physical posting row of SW_b is (b + ring_cursor) mod n_sw
     int lbsel;        // which sums make the bound: 0 = max(EQ, EC) (Eq. 5 / Thm 4.1), 1 = EQ, 2 = EC
     int fuse;         // 1: the LB kernel filters (LB <= thr) and appends survivors itself (a4+a6)
-    int lb_half;      // 1: the LB_w array holds fp16 rounded down (<= the bound: still a lower bound)
+    int lb_half;      // 1: the LB_w array holds fp16 of LB_w x lbs[mq] rounded down (R26)
+    const float *lbs; // lb_half: per-MQ power-of-two scale (query_prep_kernel: every bound x lbs fits fp16)
+    float post_unscale;  // fp16 stream ring: the entries hold P x 2^-e; sums are multiplied by 2^e
     const uint32_t *thr;  // fuse: per-segment admission bound (tau_select_kernel)
     int32_t *surv;        // fuse: survivor t lists (segment layout)
     int32_t *scount;      // fuse: survivors per segment
@@ -86,6 +89,19 @@ template <typename S> struct DtwParams {
 };
 
 template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st);
+
+// Largest power of two 2^e (|e| <= 60) with bound x 2^e <= 65504 (fp16 max):
+// the storage scale of bounds that never exceed `bound` (R26).  Scaling by a
+// power of two is exact, so rounding the scaled value down to fp16 keeps it a
+// lower bound, and no stored bound saturates.
+__host__ __device__ inline float fp16_fit_scale(double bound) {
+    if (!(bound > 0.0)) return 1.0f;
+    int e = 0;
+    double b = bound;
+    while (b * 2.0 <= 65504.0 && e < 60) { b *= 2.0; e++; }
+    while (b > 65504.0 && e > -60) { b *= 0.5; e--; }
+    return ldexpf(1.0f, e);
+}
 
 // DTW cells of one banded d x d matrix (|i-j| <= rho).
 inline int64_t dtw_cells(int d, int rho) {

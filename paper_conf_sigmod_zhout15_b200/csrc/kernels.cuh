@@ -196,22 +196,46 @@ __global__ void __launch_bounds__(256) envelope_kernel(const S *series, const in
 // ---------------------------------------------------------------------------
 // a2: query prep.  One CTA per MQ: MQ values in the arithmetic type (qv) and
 // the table {q, U(Q), L(Q), 0} with the MQ envelope of width rho_env clipped
-// to the MQ (R3, R4, R20).
+// to the MQ (R3, R4, R20).  Also:
+//  * I16: every value must satisfy |q| <= 1023 (R17); a violation sets *qflag
+//    (host-mapped) and the value is clamped so no later sum can overflow.
+//  * lbs[mq] = the fp16 storage scale of this MQ's bounds (R26): every LB is
+//    a sum of at most D terms, each at most (max|q| + max|x|)^2 (both values
+//    and both envelopes lie within [-max, max]).
 // ---------------------------------------------------------------------------
 template <typename S>
 __global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D, int rho,
                                                         typename Tr<S>::V *qv,
-                                                        typename Tr<S>::V4 *qtab) {
+                                                        typename Tr<S>::V4 *qtab, float smax,
+                                                        float *lbs, int *qflag) {
     using V = typename Tr<S>::V;
     using V4 = typename Tr<S>::V4;
     __shared__ V s[kMaxD];
+    __shared__ float s_max[8];
     const int mq = blockIdx.x;
+    float amax = 0.0f;
     for (int p = threadIdx.x; p < D; p += blockDim.x) {
         V v = (V)queries[(int64_t)mq * D + p];
+        if constexpr (std::is_same<S, int16_t>::value) {
+            if (v > 1023 || v < -1023) {
+                if (qflag) atomicOr(qflag, 1);
+                v = v > 1023 ? 1023 : -1023;
+            }
+        }
         s[p] = v;
         qv[(int64_t)mq * D + p] = v;
+        amax = fmaxf(amax, fabsf((float)v));
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
+    if ((threadIdx.x & 31) == 0) s_max[threadIdx.x >> 5] = amax;
     __syncthreads();
+    if (lbs && threadIdx.x == 0) {
+        float m = 0.0f;
+        for (int x = 0; x < (int)(blockDim.x >> 5); x++) m = fmaxf(m, s_max[x]);
+        const double a = (double)m + (double)smax;
+        lbs[mq] = fp16_fit_scale((double)D * a * a);
+    }
     for (int p = threadIdx.x; p < D; p += blockDim.x) {
         int lo = p - rho < 0 ? 0 : p - rho;
         int hi = p + rho > D - 1 ? D - 1 : p + rho;
@@ -376,9 +400,10 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
             thf = __uint_as_float(th);
         else
             thf = __int2float_ru((int32_t)th);
-        // h <= thf (float)  <=>  h <= thf rounded up to fp16 (h is an fp16 value);
-        // the +inf threshold of "no pruning" stays +inf
-        const __half2 th2 = __half2half2(__float2half_ru(thf));
+        // stored h = rd(LB x scale): h <= tau x scale (exact power-of-two product,
+        // rounded up if it underflows)  <=>  h <= that rounded up to fp16 (h is an
+        // fp16 value); the +inf threshold of "no pruning" stays +inf
+        const __half2 th2 = __half2half2(__float2half_ru(__fmul_ru(thf, P.lbs[mq])));
         const __half *row = reinterpret_cast<const __half *>(lb) + m.seg_off + (int64_t)i * m.n;
         const uintptr_t a0 = reinterpret_cast<uintptr_t>(row + t0);
         const int4 *vb = reinterpret_cast<const int4 *>(a0 & ~(uintptr_t)15);
@@ -778,6 +803,18 @@ __global__ void accum_counts_kernel(const int32_t *scount, const int32_t *fcount
         atomicAdd(&acc[0], (unsigned long long)fcount[s]);
         atomicAdd(&acc[1 + s % n_len], (unsigned long long)scount[s]);
     }
+}
+
+// max |x| over n values (the series bound of the fp16 storage scales, R26);
+// *out must start at 0 (non-negative floats order like their bits).
+template <typename S>
+__global__ void absmax_kernel(const S *x, int64_t n, unsigned *out) {
+    float m = 0.0f;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        m = fmaxf(m, fabsf((float)x[i]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(out, __float_as_uint(m));
 }
 
 // int16 range check for the I16 dtype (R17): counts |x| > 1023.

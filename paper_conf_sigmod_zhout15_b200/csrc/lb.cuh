@@ -44,6 +44,9 @@
 #ifndef SMILER_TAU_PACKED
 #define SMILER_TAU_PACKED 1  // tau-set keys: LB_w bits with the slot in the low bits
 #endif
+#ifndef SMILER_EXPERIMENTS
+#define SMILER_EXPERIMENTS 0  // 1: timing-only switches (smiler_knn_opts.reserved != 0, results invalid)
+#endif
 #ifndef SMILER_TMA_EMPTYBAR
 #define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower)
 #endif
@@ -73,9 +76,11 @@ __device__ __forceinline__ void tau_clear(const QParams &P, int mq, int units_pe
 // never above its value (saturating at 65504): a sum of such entries is still
 // a lower bound of LB_w, hence of DTW (Thm 4.3), so filtering stays exact while
 // the ring -- the bytes the group scan streams every step -- halves.
-template <typename PV, typename V> __device__ __forceinline__ void post_st(PV *p, V v) { *p = v; }
-template <> __device__ __forceinline__ void post_st<__half, float>(__half *p, float v) {
-    *p = __float2half_rz(v);
+template <typename PV, typename V> __device__ __forceinline__ void post_st(PV *p, V v, float) { *p = v; }
+// fp16 ring: the entry times the stream batch's power-of-two scale (exact),
+// rounded toward zero (never above; saturates at 65504, still a lower bound)
+template <> __device__ __forceinline__ void post_st<__half, float>(__half *p, float v, float sc) {
+    *p = __float2half_rz(v * sc);
 }
 template <typename V, typename PV> __device__ __forceinline__ V post_cv(PV x) { return x; }
 template <> __device__ __forceinline__ float post_cv<float, __half>(__half x) { return __half2float(x); }
@@ -352,7 +357,7 @@ template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S *UC, const S *LC,
                                                        const MQMeta *meta,
                                                        const typename Tr<S>::V4 *qtab, int D,
-                                                       int w_rt, PV *post) {
+                                                       int w_rt, PV *post, float pscale) {
     using V = typename Tr<S>::V;
     extern __shared__ __align__(16) unsigned char wl_smem[];
     V *sqq = reinterpret_cast<V *>(wl_smem);
@@ -386,11 +391,11 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
         int b0 = 0;
         auto put = [&](int b, V eq, V ec) {  // ring cursor 0 at a full build: row b
             PV *o = oe + (int64_t)b * pst;
-            post_st(o, eq);
-            post_st(o + plane, ec);
+            post_st(o, eq, pscale);
+            post_st(o + plane, ec, pscale);
             if (b < nmir) {
-                post_st(o + (int64_t)n_sw * pst, eq);
-                post_st(o + (int64_t)n_sw * pst + plane, ec);
+                post_st(o + (int64_t)n_sw * pst, eq, pscale);
+                post_st(o + (int64_t)n_sw * pst + plane, ec, pscale);
             }
         };
         for (; b0 + BC <= n_sw; b0 += BC)
@@ -411,8 +416,8 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
                 lb_term((V)series[base + j], squ[p0 + j], sql[p0 + j], eq);
                 lb_term(sqq[p0 + j], (V)UC[base + j], (V)LC[base + j], ec);
             }
-            post_st(oe + (int64_t)b * pst, eq);
-            post_st(oe + (int64_t)b * pst + plane, ec);
+            post_st(oe + (int64_t)b * pst, eq, pscale);
+            post_st(oe + (int64_t)b * pst + plane, ec, pscale);
         }
     }
 }
@@ -429,7 +434,7 @@ template <typename S, int W, typename PV = typename Tr<S>::V>
 __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, const S *UC, const S *LC,
                                                            const MQMeta *meta,
                                                            const typename Tr<S>::V4 *qtab, int D, int nrows,
-                                                           int cursor, PV *post) {
+                                                           int cursor, PV *post, float pscale) {
     using V = typename Tr<S>::V;
     constexpr int BC = W < 8 ? W : 8;
     extern __shared__ __align__(16) unsigned char wi_smem[];
@@ -469,8 +474,8 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
         int row = b + cursor;
         row -= row >= n_ring ? n_ring : 0;
         PV *o = oe + (int64_t)pl * plane + (int64_t)row * pst;
-        post_st(o, v);
-        if (row < nmir) post_st(o + (int64_t)n_ring * pst, v);
+        post_st(o, v, pscale);
+        if (row < nmir) post_st(o + (int64_t)n_ring * pst, v, pscale);
     };
     // SW_0: both lists
     posting_chunk<V, W, 1, false>(c, U, L, sqq, squ, sql, D - W, 1, [&](int, V eq, V ec) {
@@ -747,9 +752,11 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 
 // Write the W final LB_w values of IQ i held by this thread (slots e = s0 + b,
 // t = e - d_i contiguous) and emit its warp's tau candidates.
-// LB_w -> fp16 rounded toward -inf: never above the bound (saturates at 65504)
-__device__ __forceinline__ __half lb_to_half(float v) { return __float2half_rd(v); }
-__device__ __forceinline__ __half lb_to_half(int32_t v) { return __int2half_rd(v); }
+// LB_w x sc -> fp16 rounded toward -inf: never above the scaled bound.  sc is
+// the MQ's power-of-two storage scale (exact product; query_prep_kernel picks it
+// so that no bound of the MQ exceeds 65504 after scaling, R26).
+__device__ __forceinline__ __half lb_to_half(float v, float sc) { return __float2half_rd(v * sc); }
+__device__ __forceinline__ __half lb_to_half(int32_t v, float sc) { return __float2half_rd(__int2float_rd(v) * sc); }
 
 template <typename V, int W, bool FASTMASK = true>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
@@ -803,20 +810,21 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
             if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
         return;
     }
-    if (P.lb_half) {  // LB_w array as fp16 rounded down (a valid, slightly looser bound)
+    if (P.lb_half) {  // LB_w array as scaled fp16 rounded down (a valid, slightly looser bound)
         __half *oh = reinterpret_cast<__half *>(lb) + m.seg_off + (int64_t)i * m.n + t0;
+        const float sc = P.lbs[mq];
         if (vmask == kAll && W % 8 == 0 && ((reinterpret_cast<uintptr_t>(oh) & 15) == 0)) {
 #pragma unroll
             for (int b = 0; b < W; b += 8) {
                 __align__(16) __half hv[8];
 #pragma unroll
-                for (int q = 0; q < 8; q++) hv[q] = lb_to_half(v[b + q]);
+                for (int q = 0; q < 8; q++) hv[q] = lb_to_half(v[b + q], sc);
                 *reinterpret_cast<int4 *>(oh + b) = *reinterpret_cast<const int4 *>(hv);
             }
         } else {
 #pragma unroll
             for (int b = 0; b < W; b++)
-                if (vmask >> b & 1u) oh[b] = lb_to_half(v[b]);
+                if (vmask >> b & 1u) oh[b] = lb_to_half(v[b], sc);
         }
     } else if (vmask == kAll && W % 4 == 0 && ((reinterpret_cast<uintptr_t>(out + t0) & 15) == 0)) {
 #pragma unroll
@@ -1017,15 +1025,16 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_MINB8 : 3)
         if (qi >= 2) save_rows |= 1ull << (qi - 2);
     }
     // IQs shorter than W have no full DW anywhere (m = 0, R6): LB_w = 0
-    for (int i = 0; i < nl && P.len[i] < W; i++)
-        if (P.k >= 0) diag_emit<V, W>(saved, i, s0, m, P, lb, tauc, mq);
+    for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(saved, i, s0, m, P, lb, tauc, mq);
 #if SMILER_DIAG_UNROLL2
 #pragma unroll 2
 #endif
     // DW r - j of row j: one loop-carried pointer (us / ls at fixed offsets),
     // so the row prologue does not re-derive tid and the tile base each row
     const V *cp = cs + (x + HALO) * DS;
-    if (P.k < 0) emit_rows = save_rows = 0;  // timing experiment: main loop only
+#if SMILER_EXPERIMENTS
+    if (P.k < 0) emit_rows = save_rows = 0;  // timing experiment: main loop only (results invalid)
+#endif
     for (int j = 0; j < mmax; j++, cp -= DS) {
         V c[W], U[W], L[W];
 #pragma unroll
@@ -1127,11 +1136,204 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_MINB8 : 3)
             for (int b = 0; b < W; b++) saved[b] = lbpick(P, se[b], sc[b]);
         }
     }
+#if SMILER_EXPERIMENTS
     if (P.k < 0) {  // timing experiment: keep the sums alive
         V acc = (V)0;
 #pragma unroll
         for (int b = 0; b < W; b++) acc += se[b] + sc[b];
         if (acc == (V)12345) lb[0] = acc;
+    }
+#endif
+}
+
+// ---------------------------------------------------------------------------
+// lb_diag_kernel for f32 with sm_100's packed fp32x2 arithmetic (FADD2 /
+// FFMA2).  The EQ and EC terms of one (SW, DW, j) element share each packed
+// instruction:
+//   A = (c, L_C) + (-U_Q, -q)   = (c - U_Q, L_C - q)      EQ's v - U, EC's L - v
+//   B = (q, L_Q) + (-U_C, -c)   = (q - U_C, L_Q - c)      EC's v - U, EQ's L - v
+//   m = (max(A.x, B.y, 0), max(A.y, B.x, 0))             two FMNMX3
+// (the halves of B are crossed so that each FMNMX3 reads one even and one odd
+// register of the pairs: no register-bank conflict)
+//   (S_EQ, S_EC) = fma(m, m, (S_EQ, S_EC))               one FFMA2
+// 5 instructions per term pair instead of 8, with exactly the scalar form's
+// roundings (a + (-b) is a - b) and the same per-slot summation order, so
+// every LB_w is bit-identical to lb_diag_kernel<float, W>'s.  The DW tile
+// holds (c, L_C, -U_C, -c) and the MQ table (-U_Q, -q, q, L_Q) per point, so
+// one LDS.128 yields both operand pairs.  Tile, diagonal walk, emission and
+// tau set are lb_diag_kernel's.
+// smem: qx [x2_pad + D] float4 | tile [kDiagCols][W + 1] float4 (column stride
+// W + 1: the 8 lanes of one LDS.128 phase hit distinct bank quads).
+// ---------------------------------------------------------------------------
+#ifndef SMILER_DIAG_X2_MINB8
+#define SMILER_DIAG_X2_MINB8 6  // 78 registers, no spills: 5 CTAs 9.03 ms, 6: 8.44, 7: 8.49, 8: 8.88 (C2 LB)
+#endif
+__device__ __forceinline__ float2 lo2(const float4 &v) { return make_float2(v.x, v.y); }
+__device__ __forceinline__ float2 hi2(const float4 &v) { return make_float2(v.z, v.w); }
+
+// Term pairs of chunk slots bb < BC (valid: bb < nv) against the row's DW
+// points Pt[0..W) and the window Q[0..W+BC-1) (element (bb, j) uses
+// Q[BC-1-bb+j]).  Window-position-outer order: one Q entry live at a time,
+// and every slot still receives its terms in increasing j.
+template <int W, int BC, bool CHECK>
+__device__ __forceinline__ void x2_chunk(const float4 (&Pt)[W], const float4 *Q, int nv, float2 (&acc)[BC]) {
+#pragma unroll
+    for (int k = 0; k < W + BC - 1; k++) {
+        const float4 q = Q[k];
+#pragma unroll
+        for (int j = (k - BC + 1 > 0 ? k - BC + 1 : 0); j <= (k < W - 1 ? k : W - 1); j++) {
+            const int bb = BC - 1 - k + j;
+            if (!CHECK || bb < nv) {
+                const float2 a = __fadd2_rn(lo2(Pt[j]), lo2(q));
+                const float2 b = __fadd2_rn(hi2(q), hi2(Pt[j]));
+                const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.y), 0.0f), fmaxf(fmaxf(a.y, b.x), 0.0f));
+                acc[bb] = __ffma2_rn(mm, mm, acc[bb]);
+            }
+        }
+    }
+}
+
+// qx front padding (entries): windows of the last CSG row's invalid slots start
+// up to BC - 1 positions before the MQ; they are never used, only kept in range
+template <int W> constexpr int x2_pad() { return 8; }
+// qx plus the tile's NT + mmax - 1 columns (sized by the actual halo: more CTAs per SM)
+template <int W> size_t x2_smem(int D) {
+    return (size_t)(x2_pad<W>() + D + (kDiagThreads + D / W - 1) * (W + 1)) * 16;
+}
+
+// The last CSG row with a single valid slot (nv = D mod w + 1 = 1, e.g. D = 128,
+// w = 8): slot 0's W term pairs only (the predicated chunk would issue every
+// pair's instructions for the one that counts).
+template <int W, int BC>
+__device__ __forceinline__ void x2_chunk_slot0(const float4 (&Pt)[W], const float4 *Q, float2 (&acc)[BC]) {
+#pragma unroll
+    for (int j = 0; j < W; j++) {
+        const float4 q = Q[BC - 1 + j];
+        const float2 a = __fadd2_rn(lo2(Pt[j]), lo2(q));
+        const float2 b = __fadd2_rn(hi2(q), hi2(Pt[j]));
+        const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.y), 0.0f), fmaxf(fmaxf(a.y, b.x), 0.0f));
+        acc[0] = __ffma2_rn(mm, mm, acc[0]);
+    }
+}
+
+template <int W>
+__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 : 3))
+    lb_diag_x2_kernel(const float *series, const float *UC, const float *LC, const MQMeta *meta,
+                      const float4 *qtab, const QParams P, float *lb, int32_t *tauc) {
+    constexpr int NT = kDiagThreads;
+    constexpr int BC = W < 8 ? W : 8;
+    constexpr int NCH = W / BC;
+    constexpr int DS = W + 1;  // float4s per tile column
+    constexpr int PAD = x2_pad<W>();
+    extern __shared__ __align__(16) unsigned char dx_smem[];
+    const int D = P.D;
+    const int nl = P.n_len;
+    const int n_sw = D - W + 1;
+    const int mmax = D / W;
+    const int HALO = mmax - 1;
+    const int NC = NT + HALO;
+    float4 *qx = reinterpret_cast<float4 *>(dx_smem) + PAD;  // qx[p], p in [-PAD, D)
+    float4 *tile = qx + D;
+    const int mq = blockIdx.y;
+    const MQMeta m = meta[mq];
+    if ((int)blockIdx.x >= m.nblk) {
+        tau_clear(P, mq, kDiagThreads / 32, 0, P.n_len, tauc);
+        return;
+    }
+    for (int p = (int)threadIdx.x - PAD; p < D; p += NT) {
+        float4 e = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (p >= 0) {
+            const float4 t = qtab[(int64_t)mq * D + p];  // (q, U_Q, L_Q, 0)
+            e = make_float4(-t.y, -t.x, t.x, t.z);
+        }
+        qx[p] = e;
+    }
+    const int64_t Rb = (int64_t)blockIdx.x * NT - 1;
+    const int64_t R0 = Rb - HALO;  // DW of tile column 0
+    constexpr int W4 = W / 4;
+#pragma unroll 2
+    for (int idx = threadIdx.x; idx < NC * W4; idx += NT) {
+        const int col = idx / W4, q = idx % W4;
+        const int64_t rp = R0 + col;
+        float4 c = make_float4(0.f, 0.f, 0.f, 0.f), u = c, l = c;
+        if (rp >= 0 && rp < m.n_dw) {
+            const int64_t g = m.series_off + rp * W + 4 * q;
+            c = __ldg(reinterpret_cast<const float4 *>(series + g));
+            u = __ldg(reinterpret_cast<const float4 *>(UC + g));
+            l = __ldg(reinterpret_cast<const float4 *>(LC + g));
+        }
+        float4 *dst = tile + col * DS + 4 * q;
+        dst[0] = make_float4(c.x, l.x, -u.x, -c.x);
+        dst[1] = make_float4(c.y, l.y, -u.y, -c.y);
+        dst[2] = make_float4(c.z, l.z, -u.z, -c.z);
+        dst[3] = make_float4(c.w, l.w, -u.w, -c.w);
+    }
+    __syncthreads();
+    const int x = threadIdx.x;
+    const int64_t s0 = (Rb + 1 + x) * W;  // e of this thread's slot b = 0
+    float2 acc[W];
+    float saved[W];
+#pragma unroll
+    for (int b = 0; b < W; b++) acc[b] = make_float2(0.f, 0.f), saved[b] = 0.f;
+    uint64_t emit_rows = 0, save_rows = 0;
+    for (int i = 0; i < nl; i++) {
+        const int qi = P.len[i] / W;
+        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
+        if (qi >= 2) save_rows |= 1ull << (qi - 2);
+    }
+    // IQs shorter than W have no full DW anywhere (m = 0, R6): LB_w = 0
+    for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<float, W>(saved, i, s0, m, P, lb, tauc, mq);
+    const float4 *cp = tile + (x + HALO) * DS;  // DW r - j of row j
+    for (int j = 0; j < mmax; j++, cp -= DS) {
+        float4 Pt[W];
+#pragma unroll
+        for (int jj = 0; jj < W; jj++) Pt[jj] = cp[jj];
+        const int nrow = min(W, n_sw - j * W);
+        if constexpr (NCH == 1) {
+            const float4 *Q = qx + (D - W - j * W - (BC - 1));
+            if (nrow >= BC) x2_chunk<W, BC, false>(Pt, Q, nrow, acc);
+            else if (nrow == 1) x2_chunk_slot0<W, BC>(Pt, Q, acc);
+            else x2_chunk<W, BC, true>(Pt, Q, nrow, acc);
+        } else {
+            // two chunks (w = 16): local chunk sums added to slots 0..7 or 8..15 by
+            // one uniform branch (lb_diag_kernel's SPLIT2 association)
+#pragma unroll 1
+            for (int h = 0; h < NCH; h++) {
+                const int b0 = h * BC;
+                const int nv = nrow - b0;
+                float2 t2[BC];
+#pragma unroll
+                for (int b = 0; b < BC; b++) t2[b] = make_float2(0.f, 0.f);
+                const float4 *Q = qx + (D - W - j * W - b0 - (BC - 1));
+                if (nv >= BC) x2_chunk<W, BC, false>(Pt, Q, nv, t2);
+                else if (nv == 1) x2_chunk_slot0<W, BC>(Pt, Q, t2);
+                else if (nv > 0) x2_chunk<W, BC, true>(Pt, Q, nv, t2);
+                if (h == 0) {
+#pragma unroll
+                    for (int b = 0; b < BC; b++) acc[b] = __fadd2_rn(acc[b], t2[b]);
+                } else {
+#pragma unroll
+                    for (int b = 0; b < BC; b++) acc[BC + b] = __fadd2_rn(acc[BC + b], t2[b]);
+                }
+            }
+        }
+        // rows q_i - 1: compose IQ i from the values saved after row q_i - 2
+        // (slots b > r_i) and the current sums (b <= r_i), then write it
+        if (emit_rows >> j & 1ull) {
+            for (int i = 0; i < nl; i++) {
+                const int qi = P.len[i] / W, ri = P.len[i] % W;
+                if (j == qi - 1) {
+                    float v[W];
+#pragma unroll
+                    for (int b = 0; b < W; b++) v[b] = b > ri ? saved[b] : lbpick(P, acc[b].x, acc[b].y);
+                    diag_emit<float, W, (W <= 8)>(v, i, s0, m, P, lb, tauc, mq);
+                }
+            }
+        }
+        if (save_rows >> j & 1ull) {
+#pragma unroll
+            for (int b = 0; b < W; b++) saved[b] = lbpick(P, acc[b].x, acc[b].y);
+        }
     }
 }
 
@@ -1154,6 +1356,16 @@ constexpr int kScanThreads = 256;
 #ifndef SMILER_GS_MINB
 #define SMILER_GS_MINB(W) ((W) <= 8 ? 4 : (W) <= 16 ? 2 : 1)
 #endif
+
+// fp16 ring sums are in units of the ring's storage scale 2^-e: back to the
+// bound itself (exact power-of-two product) before emission
+template <typename V, typename PV, int W>
+__device__ __forceinline__ void ring_unscale(V (&v)[W], const QParams &P) {
+    if constexpr (std::is_same<PV, __half>::value) {
+#pragma unroll
+        for (int b = 0; b < W; b++) v[b] *= P.post_unscale;
+    }
+}
 
 template <int W, bool CHECK, typename PV>
 __device__ __forceinline__ void gs_load_row(PV (&pe)[W], PV (&pc)[W], const PV *pp, uint32_t off, int bw,
@@ -1256,6 +1468,7 @@ __global__ void __launch_bounds__(kScanThreads, SMILER_GS_MINB(W)) group_scan_re
                     V v[W];
 #pragma unroll
                     for (int b = 0; b < W; b++) v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
+                    ring_unscale<V, PV, W>(v, P);
                     diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq);
                 }
             }
@@ -1493,6 +1706,7 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
 #pragma unroll
                         for (int b = 0; b < W; b++)
                             v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
+                        ring_unscale<V, PV, W>(v, P);
                         diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq, bx);
                     }
                 }

@@ -18,6 +18,7 @@
 
 #include <algorithm>
 #include <map>
+#include <mutex>
 #include <string>
 #include <type_traits>
 #include <vector>
@@ -31,15 +32,15 @@ constexpr int kTauMult = 16;  // tau-set size target, multiples of k (R8 reading
 constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previous neighbours)
 // Tile tau-set trim (tau_trim_kernel): keep the kTauKeep* x k smallest-LB_w tile
 // candidates of the scan units' picks (0 = verify them all).  smiler_knn_opts
-// .reserved[2] > 0 overrides the multiple (A/B experiments), < 0 disables.
+// .tau_keep > 0 overrides the multiple, < 0 disables the trim.
 constexpr int kTauKeepOneShot = 8;
 constexpr int kTauKeepCont = 1;
 constexpr int kTrimCap = 16384;   // chunk winners a second bitonic trim may take (two-stage)
 constexpr int kTrimSmall = 1024;  // tile lists sorted whole; longer: radix select (tau_trim_big_kernel)
 static int tau_keep(const smiler_knn_opts &o, int k, bool cont) {
     int mult = cont ? kTauKeepCont : kTauKeepOneShot;
-    if (o.reserved[2] > 0) mult = o.reserved[2];
-    if (o.reserved[2] < 0) mult = 0;
+    if (o.tau_keep > 0) mult = o.tau_keep;
+    if (o.tau_keep < 0) mult = 0;
     return mult * k;
 }
 constexpr int kTauEMax = 8;   // candidates per tau unit (CTA or warp)
@@ -140,9 +141,12 @@ struct smiler_index {
     int64_t *d_soff = nullptr, *d_slen = nullptr;
     std::map<int, std::pair<void *, void *>> env;  // rho -> (U, L)
     int num_sms = 148;
+    float smax = 0.f;          // max |x| over the indexed series (fp16 storage scales, R26)
+    int *qflag_h = nullptr;    // host-mapped sticky flag: an I16 device query outside [-1023, 1023]
+    int *qflag_d = nullptr;    // its device alias (written by query_prep_kernel)
     // workspace
     DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, taulb, tauk, taukey, thr, scount, fcount,
-        taskoff, out_ids, out_d, tmp, tmp2, pred;
+        taskoff, out_ids, out_d, tmp, tmp2, pred, lbs;
     std::vector<cudaEvent_t> events;
     size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
     // pinned staging ring for per-chunk metadata (async H2D without host sync)
@@ -203,19 +207,55 @@ static int meta_stage(smiler_index *idx, int n, MQMeta **out, int *slot) {
 // Opt a kernel in to `bytes` of dynamic shared memory.  Always set (not only
 // above 48 KB): the default cap is 48 KB minus the kernel's STATIC shared
 // memory, so e.g. 34 KB dynamic + 16 KB static fails to launch without it.
+// The attribute is per device, so the record is keyed by (device, kernel) and
+// guarded by a mutex (handles on different devices / threads are independent).
 static void set_smem(const void *kern, size_t bytes) {
-    static std::map<const void *, size_t> done;
+    static std::mutex mu;
+    static std::map<std::pair<int, const void *>, size_t> done;
     if (bytes == 0) return;
-    auto it = done.find(kern);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    const auto key = std::make_pair(dev, kern);
+    auto it = done.find(key);
     if (it != done.end() && it->second >= bytes) return;
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
-    done[kern] = bytes;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) == cudaSuccess)
+        done[key] = bytes;
+    else
+        cudaGetLastError();  // the launch reports the failure
 }
 
 static size_t esize(smiler_dtype t) { return t == SMILER_I16 ? 2 : 4; }
 
 static int set_device(smiler_index *idx) {
     CU(cudaSetDevice(idx->device));
+    return SMILER_OK;
+}
+
+// smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
+constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
+constexpr int kMaxDI16 = 256;  // R17: 2046^2 (2d - 1) < 2^31 for d <= 256
+
+static int check_opts(const smiler_knn_opts &o) {
+    const int v = o.variant;
+    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
+        v != kVarTrimTwoStage)
+        return fail(SMILER_EINVAL, "opts.variant %d is not a known kernel path", v);
+#if !SMILER_EXPERIMENTS
+    if (o.reserved != 0) return fail(SMILER_EINVAL, "opts.reserved must be 0");
+#endif
+    return SMILER_OK;
+}
+
+// The sticky range flag of I16 device queries (query_prep_kernel sets it
+// through the host mapping): reported once, then cleared.
+static int take_qflag(smiler_index *idx) {
+    volatile int *f = idx->qflag_h;
+    if (f && *f) {
+        *f = 0;
+        return fail(SMILER_ERANGE, "an I16 master query in device memory held a value outside [-1023, 1023] "
+                                   "(R17); that call's results are unspecified");
+    }
     return SMILER_OK;
 }
 
@@ -246,13 +286,11 @@ static int ensure_envelope(smiler_index *idx, int rho, void **U, void **L) {
     dim3 grid((unsigned)((nmax + kEnvTile - 1) / kEnvTile), (unsigned)idx->sensors.size());
     size_t smem = (size_t)(kEnvTile + 2 * rho) * esize(idx->dtype);
     if (idx->dtype == SMILER_I16) {
-        if (smem > 48 * 1024)
-            cudaFuncSetAttribute(envelope_kernel<int16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        set_smem((const void *)envelope_kernel<int16_t>, smem);
         envelope_kernel<int16_t><<<grid, 256, smem, idx->stream>>>(
             (const int16_t *)idx->d_series, idx->d_soff, idx->d_slen, rho, (int16_t *)u, (int16_t *)l);
     } else {
-        if (smem > 48 * 1024)
-            cudaFuncSetAttribute(envelope_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        set_smem((const void *)envelope_kernel<float>, smem);
         envelope_kernel<float><<<grid, 256, smem, idx->stream>>>(
             (const float *)idx->d_series, idx->d_soff, idx->d_slen, rho, (float *)u, (float *)l);
     }
@@ -293,19 +331,26 @@ static int upload_series(smiler_index *idx, const void *series, const int64_t *o
     CU(cudaMalloc(&idx->d_slen, sizeof(int64_t) * ns));
     CU(cudaMemcpyAsync(idx->d_soff, so.data(), sizeof(int64_t) * ns, cudaMemcpyHostToDevice, idx->stream));
     CU(cudaMemcpyAsync(idx->d_slen, sl.data(), sizeof(int64_t) * ns, cudaMemcpyHostToDevice, idx->stream));
+    // I16 range (R17) and max |x| (the series bound of the fp16 storage scales, R26)
+    int *chk = nullptr;
+    CU(cudaMalloc(&chk, 2 * sizeof(int)));
+    CU(cudaMemsetAsync(chk, 0, 2 * sizeof(int), idx->stream));
     if (idx->dtype == SMILER_I16) {
-        int *bad = nullptr;
-        CU(cudaMalloc(&bad, sizeof(int)));
-        CU(cudaMemsetAsync(bad, 0, sizeof(int), idx->stream));
-        range_check_kernel<<<idx->num_sms * 4, 256, 0, idx->stream>>>((const int16_t *)idx->d_series,
-                                                                      total, bad);
-        int hb = 0;
-        cudaMemcpyAsync(&hb, bad, sizeof(int), cudaMemcpyDeviceToHost, idx->stream);
-        cudaError_t e = cudaStreamSynchronize(idx->stream);
-        cudaFree(bad);
-        if (e != cudaSuccess) return fail(SMILER_ECUDA, "range check: %s", cudaGetErrorString(e));
-        if (hb) return fail(SMILER_ERANGE, "%d I16 values outside [-1023, 1023] (R17)", hb);
+        range_check_kernel<<<idx->num_sms * 4, 256, 0, idx->stream>>>((const int16_t *)idx->d_series, total, chk);
+        absmax_kernel<int16_t><<<idx->num_sms * 4, 256, 0, idx->stream>>>((const int16_t *)idx->d_series, total,
+                                                                          (unsigned *)chk + 1);
+    } else {
+        absmax_kernel<float><<<idx->num_sms * 4, 256, 0, idx->stream>>>((const float *)idx->d_series, total,
+                                                                        (unsigned *)chk + 1);
     }
+    int hb[2] = {0, 0};
+    cudaMemcpyAsync(hb, chk, sizeof(hb), cudaMemcpyDeviceToHost, idx->stream);
+    cudaError_t e = cudaStreamSynchronize(idx->stream);
+    cudaFree(chk);
+    if (e != cudaSuccess) return fail(SMILER_ECUDA, "series checks: %s", cudaGetErrorString(e));
+    if (hb[0]) return fail(SMILER_ERANGE, "%d I16 values outside [-1023, 1023] (R17)", hb[0]);
+    memcpy(&idx->smax, &hb[1], sizeof(float));
+    if (!isfinite(idx->smax)) return fail(SMILER_EINVAL, "the series holds a non-finite value");
     return SMILER_OK;
 }
 
@@ -323,7 +368,7 @@ static void destroy(smiler_index *idx) {
     DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
                       &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->taulb,  &idx->tauk,
                       &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
-                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred};
+                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred,   &idx->lbs};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
     for (int i = 0; i < kMaxLen; i++) {
@@ -335,6 +380,7 @@ static void destroy(smiler_index *idx) {
         if (idx->h_meta[s]) cudaFreeHost(idx->h_meta[s]);
         if (idx->meta_ev[s]) cudaEventDestroy(idx->meta_ev[s]);
     }
+    if (idx->qflag_h) cudaFreeHost(idx->qflag_h);
     delete idx;
 }
 
@@ -354,6 +400,9 @@ static int common_build(smiler_index *idx, int32_t device, void *stream) {
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) idx->budget = std::min(idx->budget, fr / 2);
     cudaGetLastError();
+    CU(cudaHostAlloc(&idx->qflag_h, sizeof(int), cudaHostAllocMapped));
+    *idx->qflag_h = 0;
+    CU(cudaHostGetDevicePointer(&idx->qflag_d, idx->qflag_h, 0));
     return SMILER_OK;
 }
 
@@ -386,6 +435,10 @@ extern "C" int smiler_index_build(const void *series, smiler_dtype dtype, int64_
         n_sensors = 1;
         offs = {0, n_total};
     }
+    // candidate starts t are 32-bit in the tau / survivor / finalist lists and keys
+    for (int s = 0; s < n_sensors; s++)
+        if (offs[s + 1] - offs[s] - 1 > (int64_t)INT32_MAX)
+            return fail(SMILER_EINVAL, "sensor %d has more than 2^31 points", s);
     smiler_index *idx = new smiler_index();
     int rc = common_build(idx, device, cuda_stream);
     if (rc) {
@@ -484,6 +537,9 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
     }
     pl.D = pl.len[n_len - 1];
     if (pl.D > kMaxD) return fail(SMILER_EINVAL, "D = %d exceeds %d", pl.D, kMaxD);
+    if (idx->dtype == SMILER_I16 && pl.D > kMaxDI16)
+        return fail(SMILER_EINVAL, "I16: D = %d exceeds %d (int32 exactness of every DTW and bound, R17)", pl.D,
+                    kMaxDI16);
     pl.w = idx->window;
     if (pl.w > pl.D) return fail(SMILER_EINVAL, "window %d longer than D = %d", pl.w, pl.D);
     pl.n_len = n_len;
@@ -601,6 +657,7 @@ struct StreamCtx {
     int prows;                 // ring rows per plane
     const CUtensorMap *tmap;   // the ring as one 2-D tensor (tma): w x 256 boxes
     const CUtensorMap *tmap_tail;  // the same tensor, w x (16 bytes) boxes
+    float pscale;              // fp16 ring: entries hold P x pscale (a power of two, R26)
 };
 
 template <typename S>
@@ -615,6 +672,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     smiler_knn_opts o;
     memset(&o, 0, sizeof(o));
     if (opts) o = *opts;
+    TRY(check_opts(o));
     if (!queries) return fail(SMILER_EINVAL, "queries is NULL");
     if (n_mq < 1) return fail(SMILER_EINVAL, "n_mq must be >= 1");
     if (!lengths_in) return fail(SMILER_EINVAL, "lengths is NULL");
@@ -635,7 +693,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     if (pl.direct && (sctx || (lb_only && post_out)))
         return fail(SMILER_EINVAL, "the direct lower bounds have no window level (posting lists / streams)");
     if (pl.direct) pl.fused = false;
-    if (pl.fused && o.reserved[0] == 1 && pl.fused_kind == 0) {  // row-form fused kernel (comparison)
+    if (pl.fused && o.variant == kVarRowFused && pl.fused_kind == 0) {  // row-form fused kernel (comparison)
         const int mmax = pl.D / pl.w, halo = mmax - 1;
         const size_t em = ((size_t)mmax * pl.w * 2 + 15) & ~(size_t)15;
         pl.fused_kind = 1;
@@ -675,6 +733,13 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
 
     const size_t es = sizeof(S);
     const bool q_dev = is_device_ptr(queries);
+    TRY(take_qflag(idx));  // from an earlier call that returned before its kernels ran
+    if (std::is_same<S, int16_t>::value && !q_dev) {  // R17 on the host copy
+        const int16_t *qq = (const int16_t *)queries;
+        for (int64_t x = 0; x < (int64_t)n_mq * D; x++)
+            if (qq[x] > 1023 || qq[x] < -1023)
+                return fail(SMILER_ERANGE, "queries[%lld] = %d outside [-1023, 1023] (R17)", (long long)x, (int)qq[x]);
+    }
     const bool out_dev = lb_only ? (is_device_ptr(lb_out) || (post_out && is_device_ptr(post_out)))
                                  : (is_device_ptr(ids) && is_device_ptr(dists));
     if (!lb_only && (is_device_ptr(ids) != is_device_ptr(dists)))
@@ -785,8 +850,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         P.k = pl.k;
         P.rho_env = pl.rho_env;
         P.E = E;
-        if (o.reserved[1] == 1) P.k = -1;  // timing experiment (results invalid)
-        if (o.reserved[1] == 2) P.E = 0;   // timing experiment: no tau set (no pruning)
+#if SMILER_EXPERIMENTS
+        if (o.reserved == 1) P.k = -1;  // timing experiment (results invalid)
+        if (o.reserved == 2) P.E = 0;   // timing experiment: no tau set (no pruning)
+#endif
         P.LT = LT;
         P.ring_cursor = sctx ? sctx->cursor : 0;
         P.lbsel = pl.lb_kind == SMILER_LB_INDEX_EQ ? 1 : pl.lb_kind == SMILER_LB_INDEX_EC ? 2 : 0;
@@ -806,6 +873,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         ENS(idx->queries.ensure(es * (size_t)B * D));
         ENS(idx->qv.ensure(sizeof(V) * (size_t)B * D));
         ENS(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
+        ENS(idx->lbs.ensure(sizeof(float) * (size_t)B));
         if (!sctx) ENS(idx->post.ensure(sizeof(V) * (size_t)std::max<int64_t>(post_tot, 1)));
         ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
         if (!lb_only) {
@@ -887,11 +955,11 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     };
                     // <= kTrimSmall: one bitonic sort; <= kTrimBigCap: radix select in shared
                     // memory; longer: two-stage (chunk bitonic sorts, then one more trim).
-                    // reserved[0] == 9 (tests): radix, or two-stage with reserved[1] == 9
-                    const bool test_alt = o.reserved[0] == 9;
+                    // variants 9 / 10 (tests): radix / two-stage for any list length
+                    const bool test_alt = o.variant == kVarTrimRadix || o.variant == kVarTrimTwoStage;
                     if (LTt <= kTrimSmall && !test_alt) {
                         trim1(idx->tauc.as<int32_t>(), LT, LTt, tlb);
-                    } else if (two_stage && (LTt > kTrimBigCap || (test_alt && o.reserved[1] == 9))) {
+                    } else if (two_stage && (LTt > kTrimBigCap || o.variant == kVarTrimTwoStage)) {
                         // chunk winners into the survivor buffer (unused until a6), then one more trim
                         // (t in the survivor buffer, their LB_w bits in the finalist buffer:
                         // both unused until a6/a7)
@@ -952,10 +1020,13 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // tau trim, which takes the bounds from P.taulb): half the bytes written by
         // a4 and read by a6.  lb_only (smiler_lower_bounds) and exact_postings keep V.
         P.lb_half = !lb_only && !o.no_prune && diag_emitters && !o.exact_postings;
+        P.lbs = idx->lbs.as<float>();
+        P.post_unscale = (sctx && sctx->post_half) ? 1.0f / sctx->pscale : 1.0f;
         TRY(tm.mark(0));
         // ---- a2 ----------------------------------------------------------
-        query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env,
-                                                         idx->qv.as<V>(), idx->qtab.as<V4>());
+        query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env, idx->qv.as<V>(),
+                                                         idx->qtab.as<V4>(), idx->smax, idx->lbs.as<float>(),
+                                                         idx->qflag_d);
         CHECK_LAUNCH();
         launches++;
         TRY(tm.mark(1));
@@ -996,7 +1067,26 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     idx->lb.as<V>(), idx->tauc.as<int32_t>());
             };
             if (pl.fused_kind == 0) {
-                switch (w) {
+                bool done = false;
+                if constexpr (std::is_same<S, float>::value) {
+                    // f32: the packed fp32x2 form (same sums); variant 2 = the scalar kernel
+                    if (o.variant != kVarScalarDiag) {
+                        auto gx = [&](auto kern, size_t smem) {
+                            set_smem((const void *)kern, smem);
+                            kern<<<grid, kDiagThreads, smem, idx->stream>>>(
+                                (const float *)idx->d_series, (const float *)dUC, (const float *)dLC, d_meta,
+                                reinterpret_cast<const float4 *>(idx->qtab.p), P, idx->lb.as<float>(),
+                                idx->tauc.as<int32_t>());
+                        };
+                        switch (w) {
+                            case 4: gx(lb_diag_x2_kernel<4>, x2_smem<4>(D)); break;
+                            case 8: gx(lb_diag_x2_kernel<8>, x2_smem<8>(D)); break;
+                            default: gx(lb_diag_x2_kernel<16>, x2_smem<16>(D)); break;
+                        }
+                        done = true;
+                    }
+                }
+                if (!done) switch (w) {
                     case 4: go(lb_diag_kernel<S, 4>); break;
                     case 8: go(lb_diag_kernel<S, 8>); break;
                     default: go(lb_diag_kernel<S, 16>); break;
@@ -1032,7 +1122,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           sctx->nrows, sctx->cursor, pb);
+                                                           sctx->nrows, sctx->cursor, pb, sctx->pscale);
                 };
                 if constexpr (std::is_same<S, float>::value) {
                     if (sctx->post_half) {
@@ -1063,7 +1153,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
                                                            (const S *)dLC, d_meta, idx->qtab.as<V4>(), D,
-                                                           w, pb);
+                                                           w, pb, sctx ? sctx->pscale : 1.0f);
                 };
                 bool done_half = false;
                 if constexpr (std::is_same<S, float>::value) {
@@ -1105,8 +1195,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                     int occ = 0;
                     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kScanThreads, smem);
                     const int64_t tiles = (int64_t)nblk_max * B;
-                    // opts.reserved[0] == 8: one tile per CTA (A/B against the persistent grid)
-                    const int g5 = o.reserved[0] == 8 ? (int)tiles
+                    // variant 8: one tile per CTA (A/B against the persistent grid)
+                    const int g5 = o.variant == kVarTmaOneTile ? (int)tiles
                                    : (int)std::min<int64_t>(tiles, (int64_t)idx->num_sms * std::max(occ, 1));
                     kern<<<g5, kScanThreads, smem, idx->stream>>>(*sctx->tmap, *sctx->tmap_tail, d_meta, P,
                                                                   idx->lb.as<V>(), idx->tauc.as<int32_t>(),
@@ -1236,7 +1326,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     unsigned long long acc_h[kMaxLen + 1] = {0};
     if (stats && !lb_only)
         CU(cudaMemcpyAsync(acc_h, idx->tmp.p, 8 * (kMaxLen + 1), cudaMemcpyDeviceToHost, idx->stream));
-    if (!out_dev || stats) CU(cudaStreamSynchronize(idx->stream));
+    if (!out_dev || stats) {
+        CU(cudaStreamSynchronize(idx->stream));
+        TRY(take_qflag(idx));
+    }
     CHECK_LAUNCH();
     if (stats) {
         fin_total = (int64_t)acc_h[0];
@@ -1319,6 +1412,7 @@ struct smiler_stream {
     int64_t pstride = 0;       // ring row stride (elements)
     int prows = 0;             // ring rows per plane
     CUtensorMap tmap, tmap_tail;
+    float pscale = 1.f;        // fp16 ring storage scale (power of two)
     int cursor = 0;
     int64_t steps = 0;
 };
@@ -1350,6 +1444,7 @@ static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_s
     sc.prows = st->prows;
     sc.tmap = &st->tmap;
     sc.tmap_tail = &st->tmap_tail;
+    sc.pscale = st->pscale;
     return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
                        stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
 }
@@ -1412,7 +1507,7 @@ extern "C" int smiler_stream_create_ex(smiler_index *idx, const void *queries, c
     // row stride padded to 8 entries (16-byte rows), first w-1 rows mirrored
     const int pbytes = st->post_half ? 2 : 4;
     st->tma = pl.scan_reg && (pl.w == 4 || pl.w == 8 || pl.w == 16) && same_ndw && ndw0 >= 1 &&
-              !(opts && opts->reserved[0] == 7);  // reserved[0] == 7: A/B without TMA
+              !(opts && opts->variant == kVarRingNoTma);  // variant 7: A/B without TMA
     st->pstride = st->tma ? (ndw0 + 7) / 8 * 8 : 0;
     st->prows = st->tma ? st->n_sw + pl.w - 1 : st->n_sw;
     for (int j = 0; j < n_streams; j++) {
@@ -1430,6 +1525,20 @@ extern "C" int smiler_stream_create_ex(smiler_index *idx, const void *queries, c
         }
     }
     const size_t es = esize(idx->dtype);
+    if (st->post_half) {
+        // fp16 ring scale: entries are sums of w terms, each at most (|q| + max|x|)^2;
+        // the initial master queries bound |q|, with 2x headroom for later points
+        // (an entry above the range saturates at 65504: still a lower bound)
+        std::vector<float> qh((size_t)n_streams * pl.D);
+        if (cudaMemcpy(qh.data(), queries, es * qh.size(), cudaMemcpyDefault) != cudaSuccess) {
+            stream_release(st);
+            return fail(SMILER_ECUDA, "reading the initial queries");
+        }
+        double qm = 0.0;
+        for (float v : qh) qm = std::max(qm, (double)fabsf(v));
+        const double a = 2.0 * (qm + (double)idx->smax);
+        st->pscale = fp16_fit_scale((double)pl.w * a * a);
+    }
     cudaError_t e = cudaMalloc(&st->ring, (size_t)pbytes * (size_t)std::max<int64_t>(tot, 1));
     if (e == cudaSuccess && st->tma) {
         // the mirror rows and the row padding are never read as valid data, but
@@ -1663,6 +1772,8 @@ static int dtw_impl(smiler_index *idx, int32_t sensor, const void *q, int32_t d,
     using V = typename Tr<S>::V;
     const SensorInfo &si = idx->sensors[sensor];
     if (d < 1 || d > kMaxD || d > si.n) return fail(SMILER_EINVAL, "bad d = %d", d);
+    if (std::is_same<S, int16_t>::value && d > kMaxDI16)
+        return fail(SMILER_EINVAL, "I16: d = %d exceeds %d (int32 exactness, R17)", d, kMaxDI16);
     if (rho < 0) return fail(SMILER_EINVAL, "rho < 0");
     rho = std::min(rho, d - 1);
     if (rho > kMaxRhoFast) return fail(SMILER_EINVAL, "rho %d exceeds %d", rho, kMaxRhoFast);
@@ -1692,7 +1803,8 @@ static int dtw_impl(smiler_index *idx, int32_t sensor, const void *q, int32_t d,
     CU(cudaMemcpyAsync(idx->queries.p, q, sizeof(S) * d, cudaMemcpyDefault, idx->stream));
     CU(cudaMemcpyAsync(idx->tauc.p, t32.data(), 4 * n_t, cudaMemcpyHostToDevice, idx->stream));
     query_prep_kernel<S><<<1, 256, 0, idx->stream>>>(idx->queries.as<S>(), d, 0, idx->qv.as<V>(),
-                                                     idx->qtab.as<typename Tr<S>::V4>());
+                                                     idx->qtab.as<typename Tr<S>::V4>(), 0.f, nullptr,
+                                                     idx->qflag_d);
     CHECK_LAUNCH();
     Plan pl;
     pl.n_len = 1;
@@ -1736,9 +1848,19 @@ extern "C" int smiler_merge_topk(const int64_t *ids_in, const void *dists_in, sm
     const size_t nin = (size_t)G * rows * k, nout = (size_t)rows * k;
     const bool in_dev = is_device_ptr(ids_in) && is_device_ptr(dists_in);
     const bool out_dev = is_device_ptr(ids_out) && is_device_ptr(dists_out);
-    void *buf = nullptr;
+    struct Scratch {  // freed on every return path (after the stream has drained it)
+        void *p = nullptr;
+        cudaStream_t st;
+        ~Scratch() {
+            if (p) {
+                cudaStreamSynchronize(st);
+                cudaFree(p);
+            }
+        }
+    } scratch{nullptr, st};
     const size_t need = (in_dev ? 0 : nin * 12) + (out_dev ? 0 : nout * 12);
-    if (need) CU(cudaMalloc(&buf, need));
+    if (need) CU(cudaMalloc(&scratch.p, need));
+    void *buf = scratch.p;
     const int64_t *di = ids_in;
     const void *dd = dists_in;
     char *cur = (char *)buf;
@@ -1766,9 +1888,6 @@ extern "C" int smiler_merge_topk(const int64_t *ids_in, const void *dists_in, sm
         CU(cudaMemcpyAsync(ids_out, io, nout * 8, cudaMemcpyDeviceToHost, st));
         CU(cudaMemcpyAsync(dists_out, doo, nout * 4, cudaMemcpyDeviceToHost, st));
     }
-    if (need) {
-        CU(cudaStreamSynchronize(st));
-        cudaFree(buf);
-    }
+    if (need) CU(cudaStreamSynchronize(st));
     return SMILER_OK;
 }

@@ -50,15 +50,22 @@ def window_shards(n: int, D: int, rho_max: int, window: int, world: int) -> List
 
 
 def all_gather_results(ids, dists, group=None):
-    """All-gather per-rank result tensors [rows, k] into [G, rows, k] (torch)."""
+    """All-gather per-rank result tensors [rows, k] into [G, rows, k] (torch).
+    NCCL gathers the device tensors directly (over NVLink); a gloo group (the
+    CPU tests, or several ranks sharing one GPU, which NCCL refuses) gathers
+    host copies and returns tensors on the inputs' device."""
     import torch
     import torch.distributed as dist
     G = dist.get_world_size(group)
     rows = int(ids.shape[0])
+    dev = ids.device
+    if dev.type == "cuda" and dist.get_backend(group) != "nccl":
+        ids, dists = ids.cpu(), dists.cpu()
     gi = torch.empty((G * rows,) + tuple(ids.shape[1:]), dtype=ids.dtype, device=ids.device)
     gd = torch.empty((G * rows,) + tuple(dists.shape[1:]), dtype=dists.dtype, device=dists.device)
     dist.all_gather_into_tensor(gi, ids.contiguous(), group=group)
     dist.all_gather_into_tensor(gd, dists.contiguous(), group=group)
+    gi, gd = gi.to(dev), gd.to(dev)
     return gi.view((G,) + tuple(ids.shape)), gd.view((G,) + tuple(dists.shape))
 
 
@@ -78,26 +85,56 @@ def merge_gathered(gi, gd, k: int, merge: Optional[Callable] = None):
     return oi, od
 
 
-def window_sharded_knn(series_slice, shard: WindowShard, n_global: int, queries, lengths: Sequence[int],
-                       k: int, window: int, band: float, device: int, stream=None, group=None):
-    """One rank's step of the C4 path: local kNN on its shard, all-gather, merge.
-    `queries` is a CUDA tensor [n_mq, D]; returns (ids, dists) CUDA tensors
-    [n_mq, n_len, k] (identical on every rank)."""
-    import torch
-    from .smiler import Index, smiler_knn
-    idx = Index.shard(series_slice, shard.slice_begin, n_global, shard.t_begin, shard.t_end, window, band,
-                      device=device, stream=stream)
-    try:
+class WindowShardSearch:
+    """One rank's part of the C4 path, kept across calls: the shard index
+    (envelopes of its halo slice) is built once; every `knn` call is the local
+    Suffix kNN over the owned candidates, one all-gather of the (ids, dists)
+    lists and the a9 merge (`smiler_merge_topk`).  With `shared_tau` (NEXT-2)
+    the ranks also prune with each other's running thresholds through a
+    CUDA-IPC buffer (`shared_tau_buffers`)."""
+
+    def __init__(self, series_slice, shard: WindowShard, n_global: int, window: int, band: float, device: int,
+                 stream=None, group=None):
+        from .smiler import Index
+        self.shard, self.group, self.stream = shard, group, stream
+        self.index = Index.shard(series_slice, shard.slice_begin, n_global, shard.t_begin, shard.t_end, window,
+                                 band, device=device, stream=stream)
+
+    def knn(self, queries, lengths: Sequence[int], k: int, shared_tau=None):
+        """`queries`: CUDA tensor [n_mq, D]; returns (ids, dists) CUDA tensors
+        [n_mq, n_len, k], identical on every rank.  shared_tau: a device buffer
+        of n_mq * n_len keys, all ones before the first rank uses it."""
+        import torch
+        from .smiler import KnnOpts, smiler_knn
         n_mq, nl = int(queries.shape[0]), len(lengths)
         ids = torch.empty((n_mq, nl, k), dtype=torch.int64, device=queries.device)
-        dists = torch.empty((n_mq, nl, k), dtype=torch.int32 if idx.dtype == 0 else torch.float32,
+        dists = torch.empty((n_mq, nl, k), dtype=torch.int32 if self.index.dtype == 0 else torch.float32,
                             device=queries.device)
-        smiler_knn(idx.handle, queries, None, lengths, k, ids, dists)
-        gi, gd = all_gather_results(ids.view(n_mq * nl, k), dists.view(n_mq * nl, k), group)
+        op = KnnOpts(shared_tau=shared_tau.data_ptr() if shared_tau is not None else None)
+        smiler_knn(self.index.handle, queries, None, lengths, k, ids, dists, None, op)
+        if self.stream is not None:   # the library runs on `stream`; the collective on torch's
+            torch.cuda.current_stream(queries.device).wait_stream(self.stream)
+        gi, gd = all_gather_results(ids.view(n_mq * nl, k), dists.view(n_mq * nl, k), self.group)
         oi, od = merge_gathered(gi, gd, k)
         return oi.view(n_mq, nl, k), od.view(n_mq, nl, k)
+
+    def close(self):
+        self.index.close()
+
+
+def window_sharded_knn(series_slice, shard: WindowShard, n_global: int, queries, lengths: Sequence[int],
+                       k: int, window: int, band: float, device: int, stream=None, group=None,
+                       search: Optional[WindowShardSearch] = None):
+    """One rank's step of the C4 path (local kNN on its shard, all-gather,
+    merge).  Pass `search` (a WindowShardSearch) to reuse the shard index across
+    calls; without it the index is built for this call and freed."""
+    if search is not None:
+        return search.knn(queries, lengths, k)
+    s = WindowShardSearch(series_slice, shard, n_global, window, band, device, stream, group)
+    try:
+        return s.knn(queries, lengths, k)
     finally:
-        idx.close()
+        s.close()
 
 
 def shared_tau_buffers(rows: int, device, n: int = 2, group=None):

@@ -47,8 +47,12 @@ class KnnOpts(ctypes.Structure):
     _fields_ = [("no_prune", ctypes.c_int32), ("timing", ctypes.c_int32),
                 ("mq_chunk", ctypes.c_int32), ("two_level", ctypes.c_int32),
                 ("lb_kind", ctypes.c_int32), ("horizon", ctypes.c_int32),
-                ("exact_postings", ctypes.c_int32), ("tau_mult", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3),
-                ("shared_tau", ctypes.c_void_p)]
+                ("exact_postings", ctypes.c_int32), ("tau_mult", ctypes.c_int32), ("variant", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("tau_keep", ctypes.c_int32), ("shared_tau", ctypes.c_void_p)]
+
+
+# smiler_knn_opts.variant: kernel paths with the same (exact) result, for tests and A/B timing
+VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
@@ -107,12 +111,81 @@ def _ptr(x: Any) -> Optional[int]:
     if x is None:
         return None
     if isinstance(x, np.ndarray):
-        assert x.flags["C_CONTIGUOUS"], "arrays must be C-contiguous"
+        if not x.flags["C_CONTIGUOUS"]:
+            raise ValueError("arrays must be C-contiguous")
         return x.ctypes.data
     if hasattr(x, "data_ptr"):
-        assert x.is_contiguous(), "tensors must be contiguous"
+        if not x.is_contiguous():
+            raise ValueError("tensors must be contiguous")
         return x.data_ptr()
     raise TypeError(type(x))
+
+
+def _np_or_tensor_dtype(x) -> str:
+    return str(x.dtype).replace("torch.", "")
+
+
+def _check_buf(name: str, x, dtype: str, shape) -> None:
+    """An argument the C side reads or writes as `dtype` with `shape` elements."""
+    if x is None:
+        raise ValueError("%s is None" % name)
+    got = _np_or_tensor_dtype(x)
+    if got != dtype:
+        raise TypeError("%s must be %s, got %s" % (name, dtype, got))
+    if tuple(x.shape) != tuple(shape):
+        raise ValueError("%s must have shape %s, got %s" % (name, tuple(shape), tuple(x.shape)))
+
+
+def _queries_for(index_code: int, queries, lengths):
+    """Queries as the index dtype, [n_mq, D] with D = lengths[-1].  numpy float
+    arrays are cast to float32 for an F32 index, integer arrays to int16 for an
+    I16 index (values are range-checked by the library, R17); tensors must
+    already have the index dtype (no implicit device copy)."""
+    want = "int16" if index_code == SMILER_I16 else "float32"
+    if queries.ndim != 2 or int(queries.shape[1]) != int(lengths[-1]):
+        raise ValueError("queries must be [n_mq, D] with D = lengths[-1] = %d, got shape %s"
+                         % (int(lengths[-1]), tuple(queries.shape)))
+    if isinstance(queries, np.ndarray):
+        if queries.dtype != np.dtype(want):
+            if want == "float32" and np.issubdtype(queries.dtype, np.floating):
+                queries = queries.astype(np.float32)
+            elif want == "int16" and np.issubdtype(queries.dtype, np.integer):
+                if queries.size and (queries.max() > 32767 or queries.min() < -32768):
+                    raise ValueError("I16 queries must satisfy |x| <= 1023")
+                queries = queries.astype(np.int16)
+            else:
+                raise TypeError("queries must be %s for this index, got %s" % (want, queries.dtype))
+        return np.ascontiguousarray(queries)
+    if _np_or_tensor_dtype(queries) != want:
+        raise TypeError("queries must be %s for this index, got %s" % (want, queries.dtype))
+    return queries
+
+
+def _check_knn_args(queries, lengths, k: int, ids, dists) -> None:
+    """Shapes and dtypes the C side relies on: queries [n_mq, D] int16/float32,
+    ids int64 and dists int32/float32 (matching the queries) of [n_mq, n_len, k]."""
+    qd = _np_or_tensor_dtype(queries)
+    if qd not in ("int16", "float32"):
+        raise TypeError("queries must be int16 or float32 (the index dtype), got %s" % qd)
+    if queries.ndim != 2 or int(queries.shape[1]) != int(lengths[-1]):
+        raise ValueError("queries must be [n_mq, D] with D = lengths[-1] = %d, got shape %s"
+                         % (int(lengths[-1]), tuple(queries.shape)))
+    shape = (int(queries.shape[0]), len(lengths), int(k))
+    _check_buf("ids", ids, "int64", shape)
+    _check_buf("dists", dists, "int32" if qd == "int16" else "float32", shape)
+
+
+def _query_sensor(qs, n_mq: int):
+    if qs is None:
+        return None
+    if hasattr(qs, "data_ptr"):
+        if _np_or_tensor_dtype(qs) != "int32" or tuple(qs.shape) != (n_mq,):
+            raise TypeError("query_sensor tensors must be int32 of shape (%d,)" % n_mq)
+        return qs
+    a = np.ascontiguousarray(qs, np.int32)
+    if a.shape != (n_mq,):
+        raise ValueError("query_sensor must have %d entries" % n_mq)
+    return a
 
 
 def _dtype_code(x: Any) -> int:
@@ -163,9 +236,9 @@ def smiler_knn(handle: int, queries, query_sensor, lengths, k: int, ids, dists,
     """Fills ids [n_mq, n_len, k] int64 and dists [n_mq, n_len, k] int32/float32
     (host numpy or device tensors, caller-allocated)."""
     lens = np.ascontiguousarray(lengths, dtype=np.int32)
-    qs = None if query_sensor is None else (
-        query_sensor if hasattr(query_sensor, "data_ptr") else np.ascontiguousarray(query_sensor, np.int32))
+    _check_knn_args(queries, lens, k, ids, dists)
     n_mq = int(queries.shape[0])
+    qs = _query_sensor(query_sensor, n_mq)
     _check("smiler_knn",
            lib().smiler_knn_ex(handle, _ptr(queries), _ptr(qs), n_mq, _ptr(lens), len(lens), k, _ptr(ids),
                                _ptr(dists), ctypes.byref(stats) if stats is not None else None,
@@ -177,9 +250,10 @@ def smiler_knn_step(handle: int, queries, query_sensor, lengths, k: int, prev_id
     """One continuous step: like smiler_knn, with the previous step's ids of the
     same streams seeding each item query's threshold."""
     lens = np.ascontiguousarray(lengths, dtype=np.int32)
-    qs = None if query_sensor is None else (
-        query_sensor if hasattr(query_sensor, "data_ptr") else np.ascontiguousarray(query_sensor, np.int32))
+    _check_knn_args(queries, lens, k, ids, dists)
     n_mq = int(queries.shape[0])
+    _check_buf("prev_ids", prev_ids, "int64", (n_mq, len(lens), int(k)))
+    qs = _query_sensor(query_sensor, n_mq)
     _check("smiler_knn_step",
            lib().smiler_knn_step(handle, _ptr(queries), _ptr(qs), n_mq, _ptr(lens), len(lens), k, _ptr(prev_ids),
                                  shift, _ptr(ids), _ptr(dists), ctypes.byref(stats) if stats is not None else None,
@@ -191,7 +265,8 @@ def smiler_stream_create(handle: int, queries, query_sensor, lengths, k: int, id
     """Create a batch of continuous streams (Remark 1) and run their first search."""
     h = ctypes.c_void_p()
     lens = np.ascontiguousarray(lengths, dtype=np.int32)
-    qs = None if query_sensor is None else np.ascontiguousarray(query_sensor, np.int32)
+    _check_knn_args(queries, lens, k, ids, dists)
+    qs = _query_sensor(query_sensor, int(queries.shape[0]))
     _check("smiler_stream_create",
            lib().smiler_stream_create_ex(handle, _ptr(queries), _ptr(qs), int(queries.shape[0]), _ptr(lens),
                                          len(lens), k, _ptr(ids), _ptr(dists),
@@ -284,11 +359,12 @@ class Stream:
     def __init__(self, index: "Index", queries, lengths: Sequence[int], k: int, query_sensor=None,
                  exact_postings: bool = False):
         self.index, self.lengths, self.k = index, list(lengths), k
+        queries = _queries_for(index.dtype, queries, lengths)
         self.n = int(queries.shape[0])
         self.vt = np.int32 if index.dtype == SMILER_I16 else np.float32
         ids = np.empty((self.n, len(lengths), k), np.int64)
         dists = np.empty((self.n, len(lengths), k), self.vt)
-        self.handle = smiler_stream_create(index.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
+        self.handle = smiler_stream_create(index.handle, queries, query_sensor, lengths, k,
                                            ids, dists, KnnOpts(exact_postings=int(exact_postings)))
         self.first = (ids, dists)
 
@@ -296,7 +372,11 @@ class Stream:
         ids = np.empty((self.n, len(self.lengths), self.k), np.int64)
         dists = np.empty((self.n, len(self.lengths), self.k), self.vt)
         st = KnnStats() if stats else None
-        smiler_stream_step(self.handle, np.ascontiguousarray(new_points), ids, dists, st,
+        new_points = np.asarray(new_points)
+        if new_points.shape != (self.n,):
+            raise ValueError("new_points must have one point per stream (%d)" % self.n)
+        new_points = np.ascontiguousarray(new_points, self.vt if self.vt is np.float32 else np.int16)
+        smiler_stream_step(self.handle, new_points, ids, dists, st,
                            KnnOpts(timing=int(timing), tau_mult=int(tau_mult)))
         if stats:
             return ids, dists, st.as_dict()
@@ -337,21 +417,21 @@ class Index:
 
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
             no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False,
-            lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0, reserved=None):
+            lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0, variant=0,
+            tau_keep: int = 0):
         """kNN of every item query (smiler_knn_ex).  shared_tau: optional device
         buffer (torch int64 tensor of n_mq * n_len entries, all ones = -1 at start)
         shared by the window-range shards of one search (NEXT-2)."""
+        queries = _queries_for(self.dtype, queries, lengths)
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
         op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level),
                      lb_kind=int(lb_kind), horizon=int(horizon), tau_mult=int(tau_mult),
-                     shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
-        if reserved is not None:   # experiment / test switches (include/smiler.h)
-            for j, v in enumerate(reserved):
-                op.reserved[j] = int(v)
-        smiler_knn(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k, ids, dists, st, op)
+                     variant=VARIANTS[variant] if isinstance(variant, str) else int(variant),
+                     tau_keep=int(tau_keep), shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
+        smiler_knn(self.handle, queries, query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()
         return ids, dists
@@ -359,21 +439,23 @@ class Index:
     def predict(self, queries, lengths: Sequence[int], ids, ekv: Sequence[int], horizon: int, theta,
                 query_sensor=None):
         """(ar_mean, ar_var, gp_mean, gp_var), each [n_mq, n_len, len(ekv)] float64."""
+        queries = _queries_for(self.dtype, queries, lengths)
         shape = (queries.shape[0], len(lengths), len(ekv))
         outs = [np.empty(shape, np.float64) for _ in range(4)]
-        smiler_predict(self.handle, np.ascontiguousarray(queries), query_sensor, lengths,
+        smiler_predict(self.handle, queries, query_sensor, lengths,
                        np.ascontiguousarray(ids, dtype=np.int64), ekv, horizon,
                        np.ascontiguousarray(theta, dtype=np.float64), *outs)
         return tuple(outs)
 
     def knn_step(self, queries, lengths: Sequence[int], k: int, prev_ids, shift: int = 1, query_sensor=None,
                  stats: bool = False, timing: bool = False, tau_mult: int = 0):
+        queries = _queries_for(self.dtype, queries, lengths)
         n_mq = queries.shape[0]
         ids = np.empty((n_mq, len(lengths), k), np.int64)
         dists = np.empty((n_mq, len(lengths), k), np.int32 if self.dtype == SMILER_I16 else np.float32)
         st = KnnStats() if stats else None
         op = KnnOpts(timing=int(timing), tau_mult=int(tau_mult))
-        smiler_knn_step(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, k,
+        smiler_knn_step(self.handle, queries, query_sensor, lengths, k,
                         np.ascontiguousarray(prev_ids, dtype=np.int64), shift, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()
@@ -389,25 +471,28 @@ class Index:
     def lower_bounds(self, queries, lengths, n: int, window: int, query_sensor=None, postings: bool = True):
         """postings=True: two-level path (posting lists materialised and returned);
         postings=False: the fused path (returns post=None)."""
+        queries = _queries_for(self.dtype, queries, lengths)
         n_mq, D = queries.shape
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32
         post = np.empty((n_mq, 2, D - window + 1, n // window), vt) if postings else None
         lbw = np.empty((n_mq, len(lengths), n), vt)
-        smiler_lower_bounds(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, post, lbw)
+        smiler_lower_bounds(self.handle, queries, query_sensor, lengths, post, lbw)
         return post, lbw
 
     def lower_bounds_kind(self, queries, lengths, n: int, lb_kind: int, query_sensor=None):
         """The per-candidate bound smiler_knn_ex filters with under `lb_kind`:
         [n_mq][n_len][n] (entries with t > n - d_i unspecified)."""
+        queries = _queries_for(self.dtype, queries, lengths)
         n_mq = queries.shape[0]
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32
         lb = np.empty((n_mq, len(lengths), n), vt)
-        smiler_lower_bounds_ex(self.handle, np.ascontiguousarray(queries), query_sensor, lengths, lb_kind, lb)
+        smiler_lower_bounds_ex(self.handle, queries, query_sensor, lengths, lb_kind, lb)
         return lb
 
     def dtw(self, sensor: int, q, rho: int, ts):
         vt = np.int32 if self.dtype == SMILER_I16 else np.float32
         out = np.empty(len(ts), vt)
+        q = _queries_for(self.dtype, np.asarray(q).reshape(1, -1), [len(q)])[0]
         smiler_dtw(self.handle, sensor, np.ascontiguousarray(q), rho, ts, out)
         return out
 

@@ -132,6 +132,11 @@ def test_dtw_kernel(pkg, orc, dtype, d, rho):
     ts = rng.integers(0, 3000 - d + 1, size=203)   # several warps and a ragged tail
     q = wl.queries[0]
     with pkg.Index(wl.series, None, 1, 1.0) as idx:
+        if dtype == "i16" and d > 256:   # R17: int32 exactness needs d <= 256
+            with pytest.raises(pkg.SmilerError) as ei:
+                idx.dtw(0, q, rho, ts)
+            assert ei.value.code == -1
+            return
         got = idx.dtw(0, q, rho, ts)
     r = min(rho, d - 1)
     if dtype == "i16":
@@ -195,25 +200,25 @@ def test_c4_reduced(pkg, orc, dtype):
 
 # a5 tau-set trim (tau_trim_kernel / tau_trim_big_kernel): any kept subset of
 # verified candidates gives a valid tau, so the kNN must not change; keep = 1 x k
-# is the tightest trim, (9, 0, m) forces the radix-select path, -1 disables it
-@pytest.mark.parametrize("reserved", [(0, 0, 1), (9, 0, 1), (9, 0, 3), (0, 0, -1), (0, 0, 64)])
+# is the tightest trim, variant 9 forces the radix-select path, -1 disables it
+@pytest.mark.parametrize("variant,tau_keep", [(0, 1), (9, 1), (9, 3), (0, -1), (0, 64)])
 @pytest.mark.parametrize("cfg,kw", [("C2", dict(n=20011, mq_per_sensor=4)),
                                     ("C4", dict(n=60013, mq_per_sensor=2))])
-def test_tau_trim(pkg, orc, cfg, kw, reserved):
+def test_tau_trim(pkg, orc, cfg, kw, variant, tau_keep):
     wl = synth.make_workload(cfg, "i16", **kw)
-    ids, dists, st = gpu_knn(pkg, wl, stats=True, reserved=reserved)
+    ids, dists, st = gpu_knn(pkg, wl, stats=True, variant=variant, tau_keep=tau_keep)
     oid, od = orc.knn(wl, threads=THREADS)
     np.testing.assert_array_equal(ids, oid)
     np.testing.assert_array_equal(dists.astype(np.int64), od)
 
 
 # tile lists longer than one chunk (> 8192 scan units per item query): the
-# single bitonic trim (default), the two-stage chunked trim (9, 9, m) and the
-# shared-memory radix trim (9, 0, m)
-@pytest.mark.parametrize("reserved", [(0, 0, 0), (9, 9, 1), (9, 9, 4), (9, 0, 2)])
-def test_tau_trim_long_lists(pkg, orc, reserved):
+# single bitonic trim (default), the two-stage chunked trim (variant 10) and the
+# shared-memory radix trim (variant 9)
+@pytest.mark.parametrize("variant,tau_keep", [(0, 0), (10, 1), (10, 4), (9, 2)])
+def test_tau_trim_long_lists(pkg, orc, variant, tau_keep):
     wl = synth.make_workload("C2", "i16", n=2_200_003, mq_per_sensor=1, lengths=[16, 32])
-    ids, dists = gpu_knn(pkg, wl, reserved=reserved)
+    ids, dists = gpu_knn(pkg, wl, variant=variant, tau_keep=tau_keep)
     oid, od = orc.knn(wl, threads=THREADS)
     np.testing.assert_array_equal(ids, oid)
     np.testing.assert_array_equal(dists.astype(np.int64), od)
@@ -367,7 +372,7 @@ def test_errors_on_gpu(pkg):
     y = np.zeros(100, np.int16)
     with pkg.Index(y, None, 8, 2.0) as idx:
         with pytest.raises(pkg.SmilerError) as ei:
-            idx.knn(np.zeros((1, 32), np.int16), [32, 16], 3)
+            idx.knn(np.zeros((1, 16), np.int16), [32, 16], 3)   # lengths not increasing
         assert ei.value.code == -1
         with pytest.raises(pkg.SmilerError):
             idx.knn(np.zeros((1, 200), np.int16), [200], 3)   # D > N
@@ -474,9 +479,13 @@ def test_forced_chunks_equal_single_chunk(pkg, dtype):
 
 
 def test_limits_long_query_many_lengths_large_k(pkg, orc):
-    """D = 1024 with 16 item queries, k = 1024 (every ABI limit at once, R23)."""
+    """D = 1024 with 16 item queries, k = 1024 (every ABI limit at once, R23;
+    F32: I16 stops at D = 256, R17), and the I16 limit D = 256 itself."""
     lens = [16 * (i + 1) for i in range(15)] + [1024]
-    wl = synth.make_workload("C2", "i16", n=2500, mq_per_sensor=1, lengths=lens, k=1024, window=16, band=0.02)
+    wl = synth.make_workload("C2", "f32", n=2500, mq_per_sensor=1, lengths=lens, k=1024, window=16, band=0.02)
+    check_workload(pkg, orc, wl)
+    lens = [16 * (i + 1) for i in range(15)] + [256]
+    wl = synth.make_workload("C2", "i16", n=2500, mq_per_sensor=1, lengths=lens, k=1024, window=16, band=0.05)
     check_workload(pkg, orc, wl)
 
 
@@ -668,3 +677,105 @@ def test_c4_full_size_sampled(pkg, orc, dtype):
                 for t, v in zip(ts.tolist(), g.tolist()):
                     assert (v, t) >= kth or t in ids[j, i]
     assert st["survivors"] < st["candidates"]
+
+
+# ---------------------------------------------------------------------------
+# ABI hygiene and the storage precision of the bounds (R17, R26)
+# ---------------------------------------------------------------------------
+def test_opts_reserved_and_unknown_variant_are_einval(pkg):
+    wl = synth.make_workload("C1", "i16", n=600)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        n_mq, nl = wl.n_mq, len(wl.lengths)
+        ids = np.empty((n_mq, nl, wl.k), np.int64)
+        dd = np.empty((n_mq, nl, wl.k), np.int32)
+        for kw in (dict(reserved=1), dict(reserved=2), dict(variant=5), dict(variant=-1)):
+            with pytest.raises(pkg.SmilerError) as ei:
+                pkg.smiler_knn(idx.handle, wl.queries, None, wl.lengths, wl.k, ids, dd, None, pkg.KnnOpts(**kw))
+            assert ei.value.code == -1, kw
+        for v in (0, 1, 9, 10):   # every accepted variant gives the brute-force result
+            a = idx.knn(wl.queries, wl.lengths, wl.k, variant=v)
+            np.testing.assert_array_equal(a[0], idx.knn(wl.queries, wl.lengths, wl.k)[0])
+
+
+def test_i16_limits_d_and_query_range(pkg):
+    """R17: I16 needs D <= 256 and |q| <= 1023; host queries are refused before
+    any work, device queries are flagged by the query-prep kernel (ERANGE when
+    the call synchronises) and the handle stays usable."""
+    import torch
+    wl = synth.make_workload("C2", "i16", n=3000, mq_per_sensor=2)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        with pytest.raises(pkg.SmilerError) as ei:
+            idx.knn(np.zeros((1, 300), np.int16), [16, 300], 4)
+        assert ei.value.code == -1 and "R17" in str(ei.value)
+        bad = wl.queries.copy()
+        bad[1, 7] = 1024
+        with pytest.raises(pkg.SmilerError) as ei:
+            idx.knn(bad, wl.lengths, wl.k)
+        assert ei.value.code == -2
+        nl = len(wl.lengths)
+        ids = np.empty((2, nl, wl.k), np.int64)
+        dd = np.empty((2, nl, wl.k), np.int32)
+        with pytest.raises(pkg.SmilerError) as ei:
+            pkg.smiler_knn(idx.handle, torch.from_numpy(bad).cuda(), None, wl.lengths, wl.k, ids, dd)
+        assert ei.value.code == -2
+        good = idx.knn(wl.queries, wl.lengths, wl.k)           # flag cleared, handle usable
+        pkg.smiler_knn(idx.handle, torch.from_numpy(wl.queries).cuda(), None, wl.lengths, wl.k, ids, dd)
+        np.testing.assert_array_equal(ids, good[0])
+
+
+def test_wrapper_rejects_mismatched_buffers(pkg):
+    wl = synth.make_workload("C1", "f32", n=600)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        a = idx.knn(wl.queries.astype(np.float64), wl.lengths, wl.k)   # cast to the index dtype
+        np.testing.assert_array_equal(a[0], idx.knn(wl.queries, wl.lengths, wl.k)[0])
+        ids = np.empty((1, 1, wl.k), np.int64)
+        dd = np.empty((1, 1, wl.k), np.float32)
+        with pytest.raises(TypeError):   # float64 straight into the C ABI
+            pkg.smiler_knn(idx.handle, wl.queries.astype(np.float64), None, wl.lengths, wl.k, ids, dd)
+        with pytest.raises(ValueError):  # narrower than D
+            pkg.smiler_knn(idx.handle, np.ascontiguousarray(wl.queries[:, 1:]), None, wl.lengths, wl.k, ids, dd)
+        with pytest.raises(ValueError):  # wrong output shape
+            pkg.smiler_knn(idx.handle, wl.queries, None, wl.lengths, wl.k + 1, ids, dd)
+
+
+def test_i16_pruning_survives_tau_above_fp16_range(pkg, orc):
+    """R26: the fp16 LB_w array is scaled per MQ by a power of two, so a tau far
+    above 65504 (here i16 series of amplitude ~1000, D = 128) still prunes -- the
+    unscaled array would round tau up to +inf and verify every candidate."""
+    rng = np.random.default_rng(4242)
+    n = 60000
+    x = np.clip(np.cumsum(rng.integers(-60, 61, size=n + 200)), -1000, 1000)
+    x = np.clip(x + rng.integers(-200, 201, size=x.size), -1023, 1023).astype(np.int16)
+    series, tail = x[:n], x[n:]
+    q = np.stack([tail[0:128], tail[50:178]])
+    with pkg.Index(series, None, 8, 0.1) as idx:
+        ids, dists, st = idx.knn(q, [16, 32, 64, 128], 16, stats=True)
+    assert int(dists[:, -1, -1].min()) > 65504 * 2          # tau well above the fp16 range
+    assert st["survivors"] < st["candidates"] // 4, st      # ... and the index still prunes
+    for j in range(2):
+        oid, od = orc.knn_one(series, q[j], [16, 32, 64, 128], [1, 3, 6, 12], 16, threads=THREADS)
+        np.testing.assert_array_equal(ids[j], oid)
+        np.testing.assert_array_equal(dists[j].astype(np.int64), od)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_tight_lb_equals_tau_fp16_inexact(pkg, orc, dtype):
+    """P12 at a bound fp16 cannot represent: constant series a, constant query
+    b, k = 1.  Every candidate has DTW = d (a - b)^2 (a tie), the aligned ones
+    have LB_w = DTW = tau exactly, so t = 0 (aligned, lowest t) is the answer
+    only if the filter keeps a bound equal to tau after the fp16 round-down of
+    the stored bound and the round-up of the threshold."""
+    a, b = (37, -52) if dtype == "i16" else (0.1, -0.73)
+    n, w = 4096, 8
+    vt = np.int16 if dtype == "i16" else np.float32
+    series = np.full(n, a, vt)
+    for d in (16, 48, 128):
+        q = np.full((1, d), b, vt)
+        tau = d * (float(np.float32(a)) - float(np.float32(b))) ** 2
+        with pkg.Index(series, None, w, 3.0) as idx:
+            ids, dists = idx.knn(q, [d], 1)
+        assert ids[0, 0, 0] == 0, (d, ids[0, 0], dists[0, 0])
+        oid, od = orc.knn_one(series, q[0], [d], [3], 1, mode=None if dtype == "i16" else "f32")
+        assert oid[0, 0] == 0 and np.float64(dists[0, 0, 0]) == np.float64(od[0, 0])
+        m_, _ = np.frexp(tau)
+        assert m_ * 2.0 ** 11 != np.floor(m_ * 2.0 ** 11)   # needs > 11 significant bits: fp16-inexact at any scale

@@ -1,10 +1,19 @@
-# build libsmiler.so variants into _build/var/<name>.so: name=flags pairs
+# build libsmiler.so variants into _build/var/<name>.so: name=flags pairs.
+# Only smiler.cu (kernels.cuh / lb.cuh) is recompiled with the extra flags; the
+# other objects are the current build's.
 set -e
 cd "$(dirname "$0")/.."
-mkdir -p paper_conf_sigmod_zhout15_b200/_build/var
+P=paper_conf_sigmod_zhout15_b200
+python -c "from $P.build import build; build()" > /dev/null
+mkdir -p $P/_build/var
+NV="/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -lineinfo -Xcompiler -fPIC \
+    -Xcompiler -fvisibility=hidden --expt-relaxed-constexpr -I include"
+pids=()
 for spec in "$@"; do
   name=${spec%%=*}; flags=${spec#*=}
-  SMILER_EXTRA_NVFLAGS="$flags" python -c "from paper_conf_sigmod_zhout15_b200.build import build; build(force=True)"
-  cp paper_conf_sigmod_zhout15_b200/libsmiler.so paper_conf_sigmod_zhout15_b200/_build/var/$name.so
+  ( $NV $flags -c $P/csrc/smiler.cu -o $P/_build/var/$name.o && \
+    $NV -shared -cudart static -o $P/_build/var/$name.so $P/_build/var/$name.o $P/_build/dtw.o $P/_build/predict.o && \
+    rm $P/_build/var/$name.o && echo "built $name: $flags" ) &
+  pids+=($!)
 done
-python -c "from paper_conf_sigmod_zhout15_b200.build import build; build(force=True)"
+for p in "${pids[@]}"; do wait $p; done

@@ -24,7 +24,7 @@ nl = len(wl.lengths)
 ids = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int64, device=dev)
 dd = torch.empty((wl.n_mq, nl, wl.k), dtype=torch.int32 if dtype == "i16" else torch.float32, device=dev)
 st = pkg.KnnStats()
-op = pkg.KnnOpts(timing=1)
+op = pkg.KnnOpts(timing=1, variant=int(os.environ.get("SMILER_AB", "0")))
 for _ in range(reps):
     pkg.smiler_knn(idx.handle, qd, np.ascontiguousarray(wl.query_sensor), wl.lengths, wl.k, ids, dd, st, op)
 print(cfg, {k: round(v / 1e6, 3) for k, v in st.as_dict().items() if k.startswith("ns_")})
