@@ -41,10 +41,12 @@ __global__ void __launch_bounds__(kThreads) dtw_f32_mix(float *out, long long *c
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
-// DTW cell, int32: diff = q - c; m = min3; x = diff*diff + m
-__global__ void __launch_bounds__(kThreads) dtw_i32_mix(int *out, long long *cyc, int q0) {
-    int a[kChains], b[kChains];
-    int c = threadIdx.x;
+// DTW cell, int32: diff = q - c; m = min3; x = diff*diff + m (IADD, VIMNMX3,
+// IMAD: the kernel's three ops; unsigned, so wrap-around is defined and no
+// masking op is needed to keep the values bounded)
+__global__ void __launch_bounds__(kThreads) dtw_i32_mix(unsigned *out, long long *cyc, unsigned q0) {
+    unsigned a[kChains], b[kChains];
+    unsigned c = threadIdx.x;
 #pragma unroll
     for (int i = 0; i < kChains; i++) {
         a[i] = i * 3 + c;
@@ -52,16 +54,16 @@ __global__ void __launch_bounds__(kThreads) dtw_i32_mix(int *out, long long *cyc
     }
     long long t0 = clock64();
     for (int it = 0; it < kIters; it++) {
-        int q = q0 + it;
+        unsigned q = q0 + it;
 #pragma unroll
         for (int i = 0; i < kChains; i++) {
-            int diff = q - a[i];
-            int m = min(min(b[i], a[i]), c);
-            a[i] = (diff * diff + m) & 0xFFFF;  // keep values small (the AND adds one ALU op)
+            unsigned diff = q - a[i];
+            unsigned m = min(min(b[i], a[i]), c);
+            a[i] = diff * diff + m;
         }
     }
     long long t1 = clock64();
-    int s = 0;
+    unsigned s = 0;
 #pragma unroll
     for (int i = 0; i < kChains; i++) s += a[i];
     out[blockIdx.x * blockDim.x + threadIdx.x] = s;
@@ -156,25 +158,29 @@ __global__ void __launch_bounds__(kThreads) lbterm_i32_mix(int *out, long long *
     if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
-// LB term pair with packed fp32x2 (sm_100): per pair FADD2, FADD2, FMNMX3 x2, FFMA2.
+// LB term pair with packed fp32x2 (sm_100), lb_diag_x2_kernel's form: per pair
+// A = (c, L_C) - (U_Q, q), B = (q, L_Q) - (U_C, c) (two FADD2, the second operand
+// negated), m = (max(A.x, B.y, 0), max(A.y, B.x, 0)) (two FMNMX3, each reading
+// one even and one odd register), acc = fma(m, m, acc) (FFMA2).
 __global__ void __launch_bounds__(kThreads) lbterm_f32x2_mix(float *out, long long *cyc, float q0) {
-    float2 acc[kChains], cc[kChains], ne[kChains];
+    float2 acc[kChains], cl[kChains], uc[kChains];
 #pragma unroll
     for (int i = 0; i < kChains; i++) {
         acc[i] = make_float2(0.f, 0.f);
-        cc[i] = make_float2(i * 0.3f - 1.0f, i * 0.3f - 1.0f);
-        ne[i] = make_float2(-0.5f - threadIdx.x * 1e-3f - i, 0.5f + i);
+        cl[i] = make_float2(i * 0.3f - 1.0f, -0.5f - i);                         // (c, L_C)
+        uc[i] = make_float2(0.5f + threadIdx.x * 1e-3f + i, i * 0.3f - 1.0f);    // (U_C, c)
     }
     long long t0 = clock64();
     for (int it = 0; it < kIters; it++) {
-        const float q = q0 + it * 1e-4f;
-        const float2 nq = make_float2(-q, -q * 0.5f);
-        const float2 qq = make_float2(q, q);
+        // per-thread values (vector registers, as the kernel's LDS-broadcast window)
+        const float q = q0 + it * 1e-4f + threadIdx.x * 1e-7f;
+        const float2 uq = make_float2(q + 0.5f, q);   // (U_Q, q)
+        const float2 ql = make_float2(q, q - 0.5f);   // (q, L_Q)
 #pragma unroll
         for (int i = 0; i < kChains; i++) {
-            float2 d1 = __fadd2_rn(cc[i], nq);
-            float2 d2 = __fadd2_rn(qq, ne[i]);
-            float2 m = make_float2(fmaxf(fmaxf(d1.x, -d1.y), 0.f), fmaxf(fmaxf(d2.x, -d2.y), 0.f));
+            const float2 a = __fadd2_rn(cl[i], make_float2(-uq.x, -uq.y));
+            const float2 b = __fadd2_rn(ql, make_float2(-uc[i].x, -uc[i].y));
+            const float2 m = make_float2(fmaxf(fmaxf(a.x, b.y), 0.f), fmaxf(fmaxf(a.y, b.x), 0.f));
             acc[i] = __ffma2_rn(m, m, acc[i]);
         }
     }
@@ -237,14 +243,22 @@ __global__ void __launch_bounds__(kThreads) dfma_mix(double *out, long long *cyc
 
 struct Rate {
     double per_clk_sm;  // units per SM per SM clock
-    double mhz;         // effective SM clock during the run
+    double mhz;         // SM clock during the run (units per second / per-clock rate)
     double per_s;       // units per second, whole GPU
+    int ctas_per_sm;    // resident CTAs per SM (one full wave is launched)
 };
 
 // Launch `kern` back to back for >= min_ms of device time (sustained clock).
+// The grid is exactly one resident wave (occupancy of this kernel, at most
+// per_sm CTAs per SM), so every CTA runs concurrently and the per-CTA clock64
+// span is the per-SM time of the whole launch.
 template <typename K, typename T>
 static Rate run(K kern, T arg, int sms, int per_sm, double units_per_iter_chain, float min_ms) {
-    int grid = sms * per_sm;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, 0);
+    if (occ < 1) occ = 1;
+    if (occ > per_sm) occ = per_sm;
+    int grid = sms * occ;
     T *out;
     long long *cyc;
     cudaMalloc(&out, sizeof(T) * grid * kThreads);
@@ -276,6 +290,7 @@ static Rate run(K kern, T arg, int sms, int per_sm, double units_per_iter_chain,
     R.per_clk_sm = units_launch / sms / (double)cycles;
     R.per_s = units_launch * reps / (ms * 1e-3);
     R.mhz = R.per_s / (R.per_clk_sm * sms) / 1e6;
+    R.ctas_per_sm = occ;
     return R;
 }
 
@@ -292,7 +307,7 @@ int main(int argc, char **argv) {
         r[1] = run(dtw_f32x2_mix, 1.0f, sms, per_sm, 2.0, min_ms);
         r[2] = run(lbterm_f32_mix, 0.1f, sms, per_sm, 1.0, min_ms);
         r[3] = run(lbterm_f32x2_mix, 0.1f, sms, per_sm, 1.0, min_ms);
-        r[4] = run(dtw_i32_mix, 1, sms, per_sm, 1.0, min_ms);
+        r[4] = run(dtw_i32_mix, 1u, sms, per_sm, 1.0, min_ms);
         r[5] = run(lbterm_i32_mix, 1, sms, per_sm, 1.0, min_ms);
         r[6] = run(lbterm_max3_mix, 0.1f, sms, per_sm, 1.0, min_ms);
         r[7] = run(dfma_mix, 1.0, sms, per_sm, 1.0, min_ms);
@@ -302,11 +317,11 @@ int main(int argc, char **argv) {
                             "lbterm_max3", "dfma"};
     printf("{\"sms\": %d, \"ctas_per_sm\": %d, \"sustained_ms_per_mix\": %.0f", sms, per_sm, min_ms);
     for (int i = 0; i < 8; i++)
-        printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e", names[i], r[i].per_clk_sm,
-               names[i], r[i].mhz, names[i], r[i].per_s);
-    printf(", \"note\": \"units per SM per SM clock and per second over back-to-back full waves (8 CTAs x 256 threads "
-           "per SM, 8 independent chains per thread), sustained for the stated time; dtw cell = FADD+FMNMX3+FFMA (f32), "
-           "f32x2 = FADD2+2 FMNMX3+FFMA2 per 2 cells, i32 = IADD+VIMNMX3+IMAD(+LOP); lbterm = one (SW,DW,j) EQ+EC "
+        printf(", \"%s_per_clk_sm\": %.3f, \"%s_mhz\": %.0f, \"%s_per_s\": %.4e, \"%s_ctas_per_sm\": %d", names[i],
+               r[i].per_clk_sm, names[i], r[i].mhz, names[i], r[i].per_s, names[i], r[i].ctas_per_sm);
+    printf(", \"note\": \"units per SM per SM clock and per second over back-to-back single full waves (the kernel's "
+           "resident CTAs of 256 threads per SM, at most 8; 8 independent chains per thread), sustained for the stated "
+           "time; dtw cell = FADD+FMNMX3+FFMA (f32), f32x2 = FADD2+2 FMNMX3+FFMA2 per 2 cells, i32 = IADD+VIMNMX3+IMAD; lbterm = one (SW,DW,j) EQ+EC "
            "term pair = 2x(FMNMX,FMNMX,FADD,FFMA), lbterm_max3 = 2x(FADD,FADD,FMNMX3,FFMA) (the kernels' form), f32x2 = FADD2,FADD2,FMNMX3,FMNMX3,FFMA2; dfma = one fp64 FMA (2 flops)\", \"cuda\": \"%s\"}\n",
            cudaGetErrorString(e));
     return e == cudaSuccess ? 0 : 1;

@@ -760,7 +760,7 @@ __device__ __forceinline__ __half lb_to_half(int32_t v, float sc) { return __flo
 
 template <typename V, int W, bool FASTMASK = true>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
-                                          V *lb, int32_t *tauc, int mq, int bx = -1) {
+                                          V *lb, int32_t *tauc, int mq, int bx = -1, float lbsc = 0.f) {
     static_assert(W <= 32, "slot mask is 32-bit");
     const int d = P.len[i];
     const int64_t tmin = m.t_lo > 0 ? m.t_lo : 0;
@@ -812,7 +812,7 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     }
     if (P.lb_half) {  // LB_w array as scaled fp16 rounded down (a valid, slightly looser bound)
         __half *oh = reinterpret_cast<__half *>(lb) + m.seg_off + (int64_t)i * m.n + t0;
-        const float sc = P.lbs[mq];
+        const float sc = lbsc > 0.f ? lbsc : P.lbs[mq];
         if (vmask == kAll && W % 8 == 0 && ((reinterpret_cast<uintptr_t>(oh) & 15) == 0)) {
 #pragma unroll
             for (int b = 0; b < W; b += 8) {
@@ -1150,26 +1150,29 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_MINB8 : 3)
 // lb_diag_kernel for f32 with sm_100's packed fp32x2 arithmetic (FADD2 /
 // FFMA2).  The EQ and EC terms of one (SW, DW, j) element share each packed
 // instruction:
-//   A = (c, L_C) + (-U_Q, -q)   = (c - U_Q, L_C - q)      EQ's v - U, EC's L - v
-//   B = (q, L_Q) + (-U_C, -c)   = (q - U_C, L_Q - c)      EC's v - U, EQ's L - v
+//   A = (c, L_C) - (U_Q, q)     = (c - U_Q, L_C - q)      EQ's v - U, EC's L - v
+//   B = (q, L_Q) - (U_C, c)     = (q - U_C, L_Q - c)      EC's v - U, EQ's L - v
 //   m = (max(A.x, B.y, 0), max(A.y, B.x, 0))             two FMNMX3
 // (the halves of B are crossed so that each FMNMX3 reads one even and one odd
 // register of the pairs: no register-bank conflict)
 //   (S_EQ, S_EC) = fma(m, m, (S_EQ, S_EC))               one FFMA2
-// 5 instructions per term pair instead of 8, with exactly the scalar form's
-// roundings (a + (-b) is a - b) and the same per-slot summation order, so
-// every LB_w is bit-identical to lb_diag_kernel<float, W>'s.  The DW tile
-// holds (c, L_C, -U_C, -c) and the MQ table (-U_Q, -q, q, L_Q) per point, so
+// 5 instructions per term pair instead of 8 (FADD2 negates its second operand
+// for free), with exactly the scalar form's roundings and the same per-slot
+// summation order, so every LB_w is bit-identical to lb_diag_kernel<float, W>'s.
+// The DW tile holds (c, L_C, U_C, c) and the MQ table (U_Q, q, q, L_Q) per point, so
 // one LDS.128 yields both operand pairs.  Tile, diagonal walk, emission and
 // tau set are lb_diag_kernel's.
 // smem: qx [x2_pad + D] float4 | tile [kDiagCols][W + 1] float4 (column stride
 // W + 1: the 8 lanes of one LDS.128 phase hit distinct bank quads).
 // ---------------------------------------------------------------------------
 #ifndef SMILER_DIAG_X2_MINB8
-#define SMILER_DIAG_X2_MINB8 6  // 78 registers, no spills: 5 CTAs 9.03 ms, 6: 8.44, 7: 8.49, 8: 8.88 (C2 LB)
+#define SMILER_DIAG_X2_MINB8 7  // 70 registers, no spills; C2 LB 8.25 ms (6: 8.27, 5: 8.58)
 #endif
 __device__ __forceinline__ float2 lo2(const float4 &v) { return make_float2(v.x, v.y); }
 __device__ __forceinline__ float2 hi2(const float4 &v) { return make_float2(v.z, v.w); }
+__device__ __forceinline__ float2 sub2(const float2 &a, const float2 &b) {  // one FADD2 (negated operand)
+    return __fadd2_rn(a, make_float2(-b.x, -b.y));
+}
 
 // Term pairs of chunk slots bb < BC (valid: bb < nv) against the row's DW
 // points Pt[0..W) and the window Q[0..W+BC-1) (element (bb, j) uses
@@ -1184,8 +1187,8 @@ __device__ __forceinline__ void x2_chunk(const float4 (&Pt)[W], const float4 *Q,
         for (int j = (k - BC + 1 > 0 ? k - BC + 1 : 0); j <= (k < W - 1 ? k : W - 1); j++) {
             const int bb = BC - 1 - k + j;
             if (!CHECK || bb < nv) {
-                const float2 a = __fadd2_rn(lo2(Pt[j]), lo2(q));
-                const float2 b = __fadd2_rn(hi2(q), hi2(Pt[j]));
+                const float2 a = sub2(lo2(Pt[j]), lo2(q));
+                const float2 b = sub2(hi2(q), hi2(Pt[j]));
                 const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.y), 0.0f), fmaxf(fmaxf(a.y, b.x), 0.0f));
                 acc[bb] = __ffma2_rn(mm, mm, acc[bb]);
             }
@@ -1209,8 +1212,8 @@ __device__ __forceinline__ void x2_chunk_slot0(const float4 (&Pt)[W], const floa
 #pragma unroll
     for (int j = 0; j < W; j++) {
         const float4 q = Q[BC - 1 + j];
-        const float2 a = __fadd2_rn(lo2(Pt[j]), lo2(q));
-        const float2 b = __fadd2_rn(hi2(q), hi2(Pt[j]));
+        const float2 a = sub2(lo2(Pt[j]), lo2(q));
+        const float2 b = sub2(hi2(q), hi2(Pt[j]));
         const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.y), 0.0f), fmaxf(fmaxf(a.y, b.x), 0.0f));
         acc[0] = __ffma2_rn(mm, mm, acc[0]);
     }
@@ -1244,7 +1247,7 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 :
         float4 e = make_float4(0.f, 0.f, 0.f, 0.f);
         if (p >= 0) {
             const float4 t = qtab[(int64_t)mq * D + p];  // (q, U_Q, L_Q, 0)
-            e = make_float4(-t.y, -t.x, t.x, t.z);
+            e = make_float4(t.y, t.x, t.x, t.z);
         }
         qx[p] = e;
     }
@@ -1263,10 +1266,10 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 :
             l = __ldg(reinterpret_cast<const float4 *>(LC + g));
         }
         float4 *dst = tile + col * DS + 4 * q;
-        dst[0] = make_float4(c.x, l.x, -u.x, -c.x);
-        dst[1] = make_float4(c.y, l.y, -u.y, -c.y);
-        dst[2] = make_float4(c.z, l.z, -u.z, -c.z);
-        dst[3] = make_float4(c.w, l.w, -u.w, -c.w);
+        dst[0] = make_float4(c.x, l.x, u.x, c.x);
+        dst[1] = make_float4(c.y, l.y, u.y, c.y);
+        dst[2] = make_float4(c.z, l.z, u.z, c.z);
+        dst[3] = make_float4(c.w, l.w, u.w, c.w);
     }
     __syncthreads();
     const int x = threadIdx.x;
@@ -1275,65 +1278,80 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 :
     float saved[W];
 #pragma unroll
     for (int b = 0; b < W; b++) acc[b] = make_float2(0.f, 0.f), saved[b] = 0.f;
-    uint64_t emit_rows = 0, save_rows = 0;
-    for (int i = 0; i < nl; i++) {
-        const int qi = P.len[i] / W;
-        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
-        if (qi >= 2) save_rows |= 1ull << (qi - 2);
-    }
+    const float lsc = P.lb_half ? P.lbs[mq] : 0.f;
     // IQs shorter than W have no full DW anywhere (m = 0, R6): LB_w = 0
-    for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<float, W>(saved, i, s0, m, P, lb, tauc, mq);
+    int i0 = 0;
+    for (; i0 < nl && P.len[i0] < W; i0++) diag_emit<float, W>(saved, i0, s0, m, P, lb, tauc, mq, -1, lsc);
     const float4 *cp = tile + (x + HALO) * DS;  // DW r - j of row j
-    for (int j = 0; j < mmax; j++, cp -= DS) {
-        float4 Pt[W];
+    // Rows run in segments that end at the emission rows: IQ i (q_i = d_i / w,
+    // r_i = d_i % w, ascending in i) needs the sums after row q_i - 2 (saved,
+    // slots b > r_i, m_i(b) = q_i - 1) and after row q_i - 1 (slots b <= r_i).
+    // LB_w = max(S_EQ, S_EC) (Eq. 5; the EQ / EC ablations run the scalar kernel).
+    int j = 0;
+    for (int i = i0; i < nl; i++) {
+        const int qi = P.len[i] / W, ri = P.len[i] % W;
+        for (; j < qi; j++, cp -= DS) {
+            if (j == qi - 1) {
 #pragma unroll
-        for (int jj = 0; jj < W; jj++) Pt[jj] = cp[jj];
-        const int nrow = min(W, n_sw - j * W);
-        if constexpr (NCH == 1) {
-            const float4 *Q = qx + (D - W - j * W - (BC - 1));
-            if (nrow >= BC) x2_chunk<W, BC, false>(Pt, Q, nrow, acc);
-            else if (nrow == 1) x2_chunk_slot0<W, BC>(Pt, Q, acc);
-            else x2_chunk<W, BC, true>(Pt, Q, nrow, acc);
-        } else {
-            // two chunks (w = 16): local chunk sums added to slots 0..7 or 8..15 by
-            // one uniform branch (lb_diag_kernel's SPLIT2 association)
-#pragma unroll 1
-            for (int h = 0; h < NCH; h++) {
-                const int b0 = h * BC;
-                const int nv = nrow - b0;
-                float2 t2[BC];
+                for (int b = 0; b < W; b++) saved[b] = fmaxf(acc[b].x, acc[b].y);
+            }
+            float4 Pt[W];
 #pragma unroll
-                for (int b = 0; b < BC; b++) t2[b] = make_float2(0.f, 0.f);
-                const float4 *Q = qx + (D - W - j * W - b0 - (BC - 1));
-                if (nv >= BC) x2_chunk<W, BC, false>(Pt, Q, nv, t2);
-                else if (nv == 1) x2_chunk_slot0<W, BC>(Pt, Q, t2);
-                else if (nv > 0) x2_chunk<W, BC, true>(Pt, Q, nv, t2);
-                if (h == 0) {
-#pragma unroll
-                    for (int b = 0; b < BC; b++) acc[b] = __fadd2_rn(acc[b], t2[b]);
+            for (int jj = 0; jj < W; jj++) Pt[jj] = cp[jj];
+            const int nrow = min(W, n_sw - j * W);
+            if constexpr (NCH == 1) {
+                const float4 *Q = qx + (D - W - j * W - (BC - 1));
+                if (nrow >= BC) {
+                    x2_chunk<W, BC, false>(Pt, Q, nrow, acc);
                 } else {
+                    // the last CSG row (nrow < BC valid slots, a uniform bound): each
+                    // posting element summed on its own, then added (lb_diag_kernel's
+                    // association there: bit-identical LB_w)
 #pragma unroll
-                    for (int b = 0; b < BC; b++) acc[BC + b] = __fadd2_rn(acc[BC + b], t2[b]);
+                    for (int bb = 0; bb < BC; bb++) {
+                        if (bb < nrow) {
+                            float2 t = make_float2(0.f, 0.f);
+#pragma unroll
+                            for (int jj = 0; jj < W; jj++) {
+                                const float4 q = Q[BC - 1 - bb + jj];
+                                const float2 a = sub2(lo2(Pt[jj]), lo2(q));
+                                const float2 b = sub2(hi2(q), hi2(Pt[jj]));
+                                const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.y), 0.0f), fmaxf(fmaxf(a.y, b.x), 0.0f));
+                                t = __ffma2_rn(mm, mm, t);
+                            }
+                            acc[bb] = __fadd2_rn(acc[bb], t);
+                        }
+                    }
+                }
+            } else {
+                // two chunks (w = 16): local chunk sums added to slots 0..7 or 8..15 by
+                // one uniform branch (lb_diag_kernel's SPLIT2 association)
+#pragma unroll 1
+                for (int h = 0; h < NCH; h++) {
+                    const int b0 = h * BC;
+                    const int nv = nrow - b0;
+                    float2 t2[BC];
+#pragma unroll
+                    for (int b = 0; b < BC; b++) t2[b] = make_float2(0.f, 0.f);
+                    const float4 *Q = qx + (D - W - j * W - b0 - (BC - 1));
+                    if (nv >= BC) x2_chunk<W, BC, false>(Pt, Q, nv, t2);
+                    else if (nv == 1) x2_chunk_slot0<W, BC>(Pt, Q, t2);
+                    else if (nv > 0) x2_chunk<W, BC, true>(Pt, Q, nv, t2);
+                    if (h == 0) {
+#pragma unroll
+                        for (int b = 0; b < BC; b++) acc[b] = __fadd2_rn(acc[b], t2[b]);
+                    } else {
+#pragma unroll
+                        for (int b = 0; b < BC; b++) acc[BC + b] = __fadd2_rn(acc[BC + b], t2[b]);
+                    }
                 }
             }
         }
-        // rows q_i - 1: compose IQ i from the values saved after row q_i - 2
-        // (slots b > r_i) and the current sums (b <= r_i), then write it
-        if (emit_rows >> j & 1ull) {
-            for (int i = 0; i < nl; i++) {
-                const int qi = P.len[i] / W, ri = P.len[i] % W;
-                if (j == qi - 1) {
-                    float v[W];
+        // an IQ with the same q_i as the previous one reuses its saved values
+        float v[W];
 #pragma unroll
-                    for (int b = 0; b < W; b++) v[b] = b > ri ? saved[b] : lbpick(P, acc[b].x, acc[b].y);
-                    diag_emit<float, W, (W <= 8)>(v, i, s0, m, P, lb, tauc, mq);
-                }
-            }
-        }
-        if (save_rows >> j & 1ull) {
-#pragma unroll
-            for (int b = 0; b < W; b++) saved[b] = lbpick(P, acc[b].x, acc[b].y);
-        }
+        for (int b = 0; b < W; b++) v[b] = b > ri ? saved[b] : fmaxf(acc[b].x, acc[b].y);
+        diag_emit<float, W, (W <= 8)>(v, i, s0, m, P, lb, tauc, mq, -1, lsc);
     }
 }
 

@@ -1070,7 +1070,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 bool done = false;
                 if constexpr (std::is_same<S, float>::value) {
                     // f32: the packed fp32x2 form (same sums); variant 2 = the scalar kernel
-                    if (o.variant != kVarScalarDiag) {
+                    if (o.variant != kVarScalarDiag && P.lbsel == 0) {
                         auto gx = [&](auto kern, size_t smem) {
                             set_smem((const void *)kern, smem);
                             kern<<<grid, kDiagThreads, smem, idx->stream>>>(
