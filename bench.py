@@ -225,6 +225,17 @@ def oracle_sample(wl, target_s: float):
                              % (len(wl.lengths), wl.name, T, n, 100 * frac, dt))
 
 
+def cpu_model() -> str:
+    """The host CPU's model name (lscpu / /proc/cpuinfo)."""
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.lower().startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 # ---------------------------------------------------------------------------
 CFG_NAMES = {
     "C2": "C2: one sensor, 2^20 points, ELV {16,32,64,128}, band 10%, k=32, w=8, 256 MQs/step/GPU",
@@ -294,17 +305,29 @@ class Runner:
         self.tick = 0
         if self.continuous:
             D = wl.D
-            T = 2 * args.steps + args.warmup + 12
             idx_s = np.asarray(wl.query_sensor)
-            cols = wl.qoff[:, None] + np.arange(D)[None, :]
-            qt = np.empty((T, wl.n_mq, D), wl.queries.dtype)
             tails = np.stack([wl.tails[s_] for s_ in range(len(wl.tails))])
-            for s_ in range(T):
-                qt[s_] = tails[idx_s[:, None], cols + s_]
-            self.qticks_host = torch.from_numpy(qt).pin_memory()
-            self.qticks = self.qticks_host.to(dev)
             self.ids2 = torch.empty_like(self.ids)
             self.have_prev = False
+            if self.streaming:
+                # a tick appends one point per stream: the initial MQs and every later
+                # point of each stream's tail, as far as the tail reaches (no wrap:
+                # a stream only ever sees its own consecutive points)
+                T = tails.shape[1] - int(wl.qoff.max()) - D
+                q0 = tails[idx_s[:, None], wl.qoff[:, None] + np.arange(D)[None, :]]
+                newp = tails[idx_s[:, None], wl.qoff[:, None] + D - 1 + np.arange(T)[None, :]].T  # [T][n_mq]
+                self.q0 = torch.from_numpy(np.ascontiguousarray(q0)).to(dev)
+                self.newp_host = torch.from_numpy(np.ascontiguousarray(newp)).pin_memory()
+                self.newp = self.newp_host.to(dev)
+                self.max_ticks = T - 1
+            else:
+                T = 2 * args.steps + args.warmup + 12
+                cols = wl.qoff[:, None] + np.arange(D)[None, :]
+                qt = np.empty((T, wl.n_mq, D), wl.queries.dtype)
+                for s_ in range(T):
+                    qt[s_] = tails[idx_s[:, None], cols + s_]
+                self.qticks_host = torch.from_numpy(qt).pin_memory()
+                self.qticks = self.qticks_host.to(dev)
 
     def mq_per_step(self):
         """Master queries completed per step on this rank (for the value)."""
@@ -323,13 +346,14 @@ class Runner:
         op = opts if opts is not None else (self.op if stats is not None else self.op_fast)
         if self.streaming:
             if not self.have_prev:
-                self.stream_h = pkg.smiler_stream_create(self.idx.handle, self.qticks[0], self.qs, self.wl.lengths,
+                self.stream_h = pkg.smiler_stream_create(self.idx.handle, self.q0, self.qs, self.wl.lengths,
                                                          self.k, self.ids, self.dd)
                 self.have_prev = True
                 self.tick = 1
-            newp = self.qticks[self.tick % self.qticks.shape[0]][:, -1].contiguous()
+            if self.tick > self.max_ticks:
+                raise RuntimeError("the streams reached the end of their synthetic tails (%d ticks)" % self.max_ticks)
+            pkg.smiler_stream_step(self.stream_h, self.newp[self.tick], self.ids, self.dd, stats, op)
             self.tick += 1
-            pkg.smiler_stream_step(self.stream_h, newp, self.ids, self.dd, stats, op)
             return
         if self.continuous:
             q = self.qticks[self.tick % self.qticks.shape[0]]
@@ -376,12 +400,11 @@ class Runner:
         pkg, torch = self.pkg, self.torch
         if self.streaming:
             # one tick through the public stream API with pinned host buffers
-            if not hasattr(self, "newp_h"):
-                self.newp_h = torch.empty((self.wl.n_mq,), dtype=self.qticks_host.dtype).pin_memory()
-            self.newp_h.copy_(self.qticks_host[self.tick % self.qticks_host.shape[0]][:, -1])
-            self.tick += 1
-            pkg.smiler_stream_step(self.stream_h, self.newp_h, self.ih.view(self.wl.n_mq, self.n_len, self.k),
+            if self.tick > self.max_ticks:
+                raise RuntimeError("the streams reached the end of their synthetic tails (%d ticks)" % self.max_ticks)
+            pkg.smiler_stream_step(self.stream_h, self.newp_host[self.tick], self.ih.view(self.wl.n_mq, self.n_len, self.k),
                                    self.dh.view(self.wl.n_mq, self.n_len, self.k))
+            self.tick += 1
             return
         if self.continuous:
             q = self.qticks_host[self.tick % self.qticks_host.shape[0]]
@@ -432,6 +455,11 @@ def main():
     ap.add_argument("--shared-tau", action="store_true",
                     help="C4: ranks share a running threshold through CUDA IPC / NVLink atomics (NEXT-2)")
     ap.add_argument("--two-level", action="store_true", help="time the paper's two-level path (a3 -> HBM -> a4)")
+    ap.add_argument("--sustain-s", type=float, default=0.0,
+                    help="after the timed steps, run back to back for this many seconds and report the sustained "
+                         "rate and p50/p99 step latency (the C5 protocol uses 60)")
+    ap.add_argument("--prof-steps", type=int, default=10,
+                    help="steps of the separate profiled pass (per-phase events, counters)")
     ap.add_argument("--two-level-steps", type=int, default=3,
                     help="extra steps of the two-level path for the LB-scan (a4) HBM figure; 0 = skip")
     args = ap.parse_args()
@@ -460,8 +488,8 @@ def main():
                           "dtype": "int64" if args.dtype == "i16" else "f64", "data": "synthetic",
                           "impl": "reference",
                           "config": {"workload": cfg_name, "parallelism": "host cores (oracle)"},
-                          "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
-                                           "sample": sample},
+                          "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "cpu_model": cpu_model(),
+                                           "kind": "oracle", "sample": sample},
                           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}))
         return
 
@@ -492,10 +520,10 @@ def main():
     torch.cuda.synchronize(dev)
 
     # ---- timed region: device-resident inputs/outputs ---------------------------
-    # Every call records per-phase CUDA events on the library's stream
-    # (smiler_knn_stats, timing=1); the call synchronises once at its end to
-    # read them (measured cost < 1% of a C2 step).  `value` comes from the two
-    # events around the whole loop; the per-kernel rooflines from the same calls.
+    # The product call exactly as a user makes it (no stats, no per-phase
+    # events, no host synchronisation inside the loop).  One CUDA event pair
+    # around the loop gives `value`; one event per step boundary gives the step
+    # latencies.  The per-phase split comes from a separate profiled pass below.
     gpu_idx = local
     cvd = os.environ.get("CUDA_VISIBLE_DEVICES")
     if cvd:
@@ -503,42 +531,89 @@ def main():
             gpu_idx = int(cvd.split(",")[local])
         except ValueError:
             pass
-    st = pkg.KnnStats()
-    phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_verify",
-                              "ns_select", "ns_total")}
-    acc = {"survivors": 0, "candidates": 0, "dtw_cells": 0.0, "bf_cells": 0.0, "posting_bytes": 0,
-           "lb_bytes": 0, "kernel_launches": 0, "mq_chunks": 0, "tau_verified": 0, "finalists": 0}
     clocks = Clocks(gpu_idx)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)
     clocks.start()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(args.steps):
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    evs[0].record(stream)
+    for s_ in range(args.steps):
+        R.step()
+        evs[s_ + 1].record(stream)
+    torch.cuda.synchronize(dev)
+    ck = clocks.stop()
+    if world > 1:
+        dist.barrier()
+    ms = evs[0].elapsed_time(evs[-1])
+    step_ms = [evs[s_].elapsed_time(evs[s_ + 1]) for s_ in range(args.steps)]
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    mq_step = (R.global_mq if R.global_mq is not None else R.mq_per_step() * world)
+    mq_total = mq_step * args.steps
+    if R.global_mq is None and world > 1:
+        tm = torch.tensor([R.mq_per_step()], dtype=torch.float64, device=dev)
+        dist.all_reduce(tm, op=dist.ReduceOp.SUM)
+        mq_step = float(tm.item())
+        mq_total = mq_step * args.steps
+    value = mq_total / (ms_max / 1000.0)
+
+    prof_steps_planned = max(1, min(args.steps, args.prof_steps)) + args.steps + 1  # profiled pass + e2e ticks
+    # ---- sustained run (C5 protocol: >= 60 s, p50 / p99 step latency)
+    sustained = None
+    if args.sustain_s > 0:
+        ck_s = Clocks(gpu_idx)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        ck_s.start()
+        t_wall0 = time.perf_counter()
+        lat = []
+        n_sus = 0
+        dev_ms = 0.0
+        while time.perf_counter() - t_wall0 < args.sustain_s and \
+                (not R.streaming or R.tick + 32 + 2 * prof_steps_planned <= R.max_ticks):
+            batch = [torch.cuda.Event(enable_timing=True) for _ in range(33)]
+            batch[0].record(stream)
+            for b_ in range(32):
+                R.step()
+                batch[b_ + 1].record(stream)
+            batch[-1].synchronize()
+            lat += [batch[b_].elapsed_time(batch[b_ + 1]) for b_ in range(32)]
+            dev_ms += batch[0].elapsed_time(batch[-1])
+            n_sus += 32
+        torch.cuda.synchronize(dev)
+        ck2 = ck_s.stop()
+        lat.sort()
+        tl = torch.tensor([dev_ms], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tl, op=dist.ReduceOp.MAX)
+        sustained = {"seconds": time.perf_counter() - t_wall0, "steps": n_sus,
+                     "value": mq_step * n_sus / (float(tl.item()) / 1000.0), "unit": UNIT,
+                     "p50_step_ms": lat[len(lat) // 2], "p99_step_ms": lat[min(len(lat) - 1, int(0.99 * len(lat)))],
+                     "max_step_ms": lat[-1], "clocks": ck2,
+                     "timing": "device time per step (CUDA events between back-to-back steps on the library "
+                               "stream), rank-0 distribution; value = MQs / max-over-ranks device time"}
+
+    # ---- profiled pass: per-phase CUDA events and counters (smiler_knn_stats) --
+    st = pkg.KnnStats()
+    phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_verify",
+                              "ns_select", "ns_total")}
+    acc = {"survivors": 0, "candidates": 0, "dtw_cells": 0.0, "bf_cells": 0.0, "posting_bytes": 0,
+           "lb_bytes": 0, "kernel_launches": 0, "mq_chunks": 0, "tau_verified": 0, "finalists": 0}
+    prof_steps = max(1, min(args.steps, args.prof_steps))
+    ck_p = Clocks(gpu_idx)
+    ck_p.start()
+    for _ in range(prof_steps):
         R.step(st)
         for f in phase:
             phase[f] += getattr(st, f)
         for f in acc:
             acc[f] += getattr(st, f)
-    e1.record(stream)
     torch.cuda.synchronize(dev)
-    ck = clocks.stop()
-    if world > 1:
-        dist.barrier()
-    ms = e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
-    mq_total = (R.global_mq if R.global_mq is not None else R.mq_per_step() * world) * args.steps
-    if R.global_mq is None and world > 1:
-        tm = torch.tensor([R.mq_per_step() * args.steps], dtype=torch.float64, device=dev)
-        dist.all_reduce(tm, op=dist.ReduceOp.SUM)
-        mq_total = float(tm.item())
-    value = mq_total / (ms_max / 1000.0)
-    prof_steps = args.steps
+    ck_prof = ck_p.stop()
     launches_per_step = acc["kernel_launches"] / prof_steps + (1 if R.sharded_window else 0)
 
     # ---- e2e: the same public call with pinned host buffers ------------------
@@ -591,15 +666,26 @@ def main():
     alu = load_alu_peaks()
     steps = prof_steps
     sm_mhz = ck.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    if alu:
-        term_peak = alu["lbterm_per_clk_sm"] * alu["sms"] * sm_mhz * 1e6
-        cell_peak = alu["dtw_cell_f32_per_clk_sm" if args.dtype == "f32" else "dtw_cell_i32_per_clk_sm"] * \
-            alu["sms"] * sm_mhz * 1e6
-        alu_src = "profiles/alu_peaks.json (alu_bench) x median SM clock under load"
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    # ALU rooflines from unit counts: per SM per clock a Blackwell SM
+    # issues 4 warp-instructions (128 lane-instructions) and its FP32 (FMA) pipe
+    # retires 128 lanes (a packed f32x2 instruction takes two of its cycles).
+    #   LB term pair, f32 packed (lb_diag_x2): 6 FP32 lane-ops (4 subtractions in
+    #     2 FADD2, 2 FMAs in 1 FFMA2) -> 128 / 6 = 21.33 pairs/clk (5 instructions:
+    #     issue bound 25.6); scalar f32 forms (8 instructions): 128 / 8 = 16
+    #   DTW cell f32: FADD, FMNMX3, FFMA -> issue bound 128 / 3 = 42.67 cells/clk
+    #   i16 (int32) mixes: the alu_bench measurement (profiles/alu_peaks.json)
+    if args.dtype == "f32":
+        term_pclk = 128.0 / 6.0 if (wl.window in (4, 8, 16) and not R.streaming and not args.two_level) else 16.0
+        cell_pclk = 128.0 / 3.0
+        alu_src = ("unit counts (128 FP32 lanes / 4 issues per SM per clock; DESIGN.md §6) x median SM clock "
+                   "sampled during the timed region")
     else:
-        term_peak = 148 * 16 * sm_mhz * 1e6
-        cell_peak = 148 * 42.7 * sm_mhz * 1e6
-        alu_src = "issue-rate estimate (no alu_peaks.json) x median SM clock"
+        term_pclk = alu["lbterm_i32_per_clk_sm"] if alu else 16.0
+        cell_pclk = alu["dtw_cell_i32_per_clk_sm"] if alu else 128.0 / 3.0
+        alu_src = "profiles/alu_peaks.json (alu_bench int32 mixes) x median SM clock sampled during the timed region"
+    term_peak = term_pclk * sms * sm_mhz * 1e6
+    cell_peak = cell_pclk * sms * sm_mhz * 1e6
     n_sw = wl.D - wl.window + 1
     if R.sharded_window:
         pts = [R.index_points] * wl.n_mq
@@ -658,18 +744,16 @@ def main():
     rf = dict(kernels[dom])
     rf["kernel"] = dom
     rf["traffic"] = None
-    tfile = os.path.join(ROOT, "profiles", "r01", "prof_c2_traffic_per_mq.json")
+    tfile = os.path.join(ROOT, "profiles", "r02", "prof_c2_traffic_per_mq.json")
     if args.config == "C2" and os.path.exists(tfile):
-        tname = {"lb_fused": "lb_diag_kernel<%s, %d>", "window_lb_a3": "window_lb_kernel<%s, %d>",
-                 "group_scan_a4": "group_scan_kernel<%s, %d>"}.get(dom)
+        tname = {"lb_fused": ("lb_diag_x2_kernel<%d>" % wl.window) if args.dtype == "f32"
+                 else ("lb_diag_kernel<short, %d>" % wl.window)}.get(dom)
         tmap = json.load(open(tfile))
-        if tname:
-            key = tname % ("float" if args.dtype == "f32" else "short", wl.window)
-            if key in tmap:
-                # DRAM bytes per launch = ncu per-MQ traffic x MQs per launch (one chunk per step)
-                rf["traffic"] = tmap[key] * wl.n_mq
-                rf["traffic_source"] = "profiles/r01/prof_c2_traffic_per_mq.json (ncu --set full, %s)" % key
-                rf["algorithmic_bytes_per_launch"] = lb_bytes_step
+        if tname and tname in tmap:
+            # DRAM bytes per launch = ncu per-MQ traffic x MQs per launch (one chunk per step)
+            rf["traffic"] = tmap[tname] * wl.n_mq
+            rf["traffic_source"] = "profiles/r02/prof_c2_traffic_per_mq.json (ncu --set full, %s)" % tname
+            rf["algorithmic_bytes_per_launch"] = lb_bytes_step
     rf["peak_source"] = ("MEASURED_PEAKS.json hbm_gbs (%s)" % peak_kind if rf["bound"] == "hbm" else alu_src)
     two_level = None
     if two is not None:
@@ -683,7 +767,8 @@ def main():
     cpu = None
     if world == 1 and not args.no_cpu:
         v, cores, dt, sample = oracle_sample(wl, args.oracle_seconds)
-        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "cpu_model": cpu_model(), "kind": "oracle",
+               "sample": sample}
 
     par = {"C2": "dp%d (independent MQ batches)" % world, "C3": "sensor sharding x%d" % world,
            "C5": "sensor sharding x%d" % world, "C4": "window-range sharding x%d + NCCL all-gather merge" % world}
@@ -709,8 +794,13 @@ def main():
         "phase_ms_per_step": ph_ms,
         "roofline": rf, "kernels": kernels, "two_level": two_level,
         "gpu_launches": int(round(launches_per_step * args.steps)),
-        "phase_timing": "per-phase CUDA events of every timed call (same timed region as value)",
+        "phase_timing": ("per-phase CUDA events (smiler_knn_stats) of a separate profiled pass of %d steps right "
+                         "after the timed region (the timed loop itself records no phase events and never syncs)"
+                         % prof_steps),
+        "step_ms": {"p50": sorted(step_ms)[len(step_ms) // 2], "max": max(step_ms)},
+        "sustained": sustained,
         "clocks": ck,
+        "clocks_profiled_pass": ck_prof,
         "cpu_baseline": cpu,
         "e2e": e2e,
     }
