@@ -100,6 +100,8 @@ typedef struct smiler_knn_opts {
     int32_t variant;  /* kernel-path selector for tests and A/B timing; every variant computes
                          the same (exact) result: 0 = automatic, 1 = row-form fused LB kernel,
                          2 = scalar (not fp32x2-packed) diagonal LB kernel for F32,
+                         3 = the anti-diagonal wavefront DTW kernel for every warping width
+                         (by default it runs only for rho > 32, the register band below),
                          7 = stream ring scanned without TMA, 8 = one tile per ring-scan CTA,
                          9 = radix-select tau-set trim, 10 = two-stage tau-set trim.  Any other
                          value is EINVAL */

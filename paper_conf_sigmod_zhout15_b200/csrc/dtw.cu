@@ -299,7 +299,147 @@ static bool dispatch(int rho, const DtwParams<S> &p, int grid, cudaStream_t st,
     return done;
 }
 
+// ---------------------------------------------------------------------------
+// Any rho (the generic path for rho > kMaxRhoFast, and an A/B variant for
+// smaller bands): one warp per candidate, anti-diagonal wavefront.  Cells of
+// anti-diagonal k = i + j depend only on diagonals k-1 and k-2 (Eq. 21), so
+// all of them are computed at once by the warp's lanes.  Indexing the band by
+// delta = i - j in [-rho, rho], diagonal k holds the deltas with the parity of
+// k, so ONE shared array g[delta] suffices: while diagonal k is computed, the
+// slots of the other parity hold diagonal k-1 (the (i-1, j) and (i, j-1)
+// predecessors at delta -/+ 1) and its own slots still hold diagonal k-2 (the
+// (i-1, j-1) predecessor at delta) -- each cell reads only slots no lane writes
+// in this step.  Only valid cells (1 <= i, j <= d, |i - j| <= rho) are
+// computed; every read of a never-written slot is the boundary g(0, j) =
+// g(i, 0) = inf of Eq. 22, and g[0] starts as g(0, 0) = 0.  The cell is the
+// register-band kernel's (f32: fmaf(q - c, q - c, min3), R16), so results are
+// bit-identical to it and to the oracle.  The item query and the candidate
+// are staged per warp in shared memory.
+// ---------------------------------------------------------------------------
+constexpr int kWaveWarps = 4;
+__host__ __device__ inline int wave_pad(int n) { return (n + 3) & ~3; }
+// per-warp shared elements: q [d] | c [d] | g [2 rho + 1]
+__host__ __device__ inline size_t wave_smem_elems(int d, int rho) {
+    return (size_t)wave_pad(d) * 2 + wave_pad(2 * rho + 1);
+}
+
+template <typename S>
+__global__ void __launch_bounds__(kWaveWarps * 32) dtw_wave_kernel(const DtwParams<S> p, int rho) {
+    using V = typename Tr<S>::V;
+    const V INF = Tr<S>::inf();
+    extern __shared__ __align__(16) unsigned char wv_smem[];
+    const int lane = threadIdx.x & 31;
+    const int wib = threadIdx.x >> 5;
+    const int d = p.d;
+    V *sq = reinterpret_cast<V *>(wv_smem) + (size_t)wib * wave_smem_elems(d, rho);  // q_i at sq[i - 1]
+    V *sc = sq + wave_pad(d);                                                        // c_j at sc[j - 1]
+    V *g = sc + wave_pad(d);                                                         // g[delta + rho]
+    const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nw = (gridDim.x * blockDim.x) >> 5;
+    const int total = p.task_off[p.n_mq];
+    int cur_mq = -1;
+    for (int task = gw; task < total; task += nw) {
+        int lo = 0, hi = p.n_mq;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (p.task_off[mid] <= task) lo = mid; else hi = mid;
+        }
+        const int mq = lo;
+        const int chunk = task - p.task_off[mq];
+        const MQMeta m = p.meta[mq];
+        const int seg = mq * p.n_len + p.li;
+        int cnt;
+        int64_t lbase;
+        if (p.mode == 0) {
+            cnt = p.LTc;
+            lbase = (int64_t)seg * p.LT;
+        } else {
+            cnt = p.counts[seg];
+            lbase = m.seg_off + (int64_t)p.li * m.n;
+        }
+        const int idx = chunk * 32 + lane;
+        const int my_t = idx < cnt ? p.list[lbase + idx] : -1;
+        if (mq != cur_mq) {
+            __syncwarp();
+            const V *q = p.qv + (int64_t)mq * p.D + (p.D - d);
+            for (int x = lane; x < d; x += 32) sq[x] = q[x];
+            cur_mq = mq;
+        }
+        const S *cs = p.series + m.series_off;
+        V my_dist = INF;
+        for (int l = 0; l < 32; l++) {  // the task's candidates, one per pass of the warp
+            const int t = __shfl_sync(0xffffffffu, my_t, l);
+            if (t < 0) continue;  // warp-uniform
+            __syncwarp();
+            for (int x = lane; x < d; x += 32) sc[x] = (V)__ldg(cs + t + x);
+            for (int x = lane; x < 2 * rho + 1; x += 32) g[x] = x == rho ? (V)0 : INF;
+            __syncwarp();
+            for (int k = 2; k <= 2 * d; k++) {
+                // valid deltas of diagonal k: |delta| <= rho, 1 <= (k + delta) / 2 <= d,
+                // 1 <= (k - delta) / 2 <= d, delta = k (mod 2)
+                int dlo = max(-rho, max(2 - k, k - 2 * d));
+                const int dhi = min(rho, min(2 * d - k, k - 2));
+                dlo += (dlo - k) & 1;
+                for (int delta = dlo + 2 * lane; delta <= dhi; delta += 64) {
+                    const int i = (k + delta) >> 1, j = (k - delta) >> 1;
+                    const V up = delta - 1 >= -rho ? g[delta - 1 + rho] : INF;  // (i-1, j)
+                    const V lf = delta + 1 <= rho ? g[delta + 1 + rho] : INF;   // (i, j-1)
+                    const V dg = g[delta + rho];                                // (i-1, j-1)
+                    g[delta + rho] = cell(sq[i - 1], sc[j - 1], vmin3<V>(up, lf, dg));
+                }
+                __syncwarp();
+            }
+            const V dist = g[rho];  // (d, d)
+            if (lane == l) my_dist = dist;
+        }
+        const uint64_t key = my_t >= 0 ? (((uint64_t)vbits<V>(my_dist) << 32) | (uint32_t)my_t) : kKeyMax;
+        if (p.mode == 0) {
+            if (idx < cnt) p.keys_out[lbase + idx] = key;
+        } else {
+            const bool fin = my_t >= 0 && key <= p.tau_key[seg];
+            const unsigned bal = __ballot_sync(0xffffffffu, fin);
+            if (bal) {
+                int base = 0;
+                if (lane == 0) base = atomicAdd(&p.fin_count[seg], __popc(bal));
+                base = __shfl_sync(0xffffffffu, base, 0);
+                if (fin) p.fin[m.seg_off + (int64_t)p.li * m.n + base + __popc(bal & ((1u << lane) - 1))] = key;
+            }
+        }
+    }
+}
+
+template <typename S>
+static void launch_wave(int rho, const DtwParams<S> &p, int grid, cudaStream_t st) {
+    using V = typename Tr<S>::V;
+    static std::mutex mu;
+    static std::map<int, int> sms_of;  // device -> SM count
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int sms;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = sms_of.find(dev);
+        if (it == sms_of.end()) {
+            int n = 0;
+            cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+            cudaFuncSetAttribute(dtw_wave_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)(kWaveWarps * wave_smem_elems(kMaxD, kMaxD) * sizeof(V)));
+            it = sms_of.emplace(dev, n > 0 ? n : 1).first;
+        }
+        sms = it->second;
+    }
+    const size_t smem = kWaveWarps * wave_smem_elems(p.d, rho) * sizeof(V);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, dtw_wave_kernel<S>, kWaveWarps * 32, smem);
+    if (grid <= 0) grid = sms * (occ > 0 ? occ : 1);
+    dtw_wave_kernel<S><<<grid, kWaveWarps * 32, smem, st>>>(p, rho);
+}
+
 template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st) {
+    if (p.wave || rho > kMaxRhoFast) {
+        launch_wave<S>(rho, p, grid, st);
+        return;
+    }
     dispatch<S>(rho, p, grid, st, std::make_integer_sequence<int, kMaxRhoFast + 1>{});
 }
 

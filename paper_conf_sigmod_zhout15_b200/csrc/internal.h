@@ -86,6 +86,7 @@ template <typename S> struct DtwParams {
     const uint64_t *tau_key;      // survivors mode: per-segment key threshold
     uint64_t *fin;                // survivors mode: finalist keys (segment layout)
     int32_t *fin_count;
+    int wave;                     // 1: anti-diagonal wavefront kernel for any rho (else only rho > kMaxRhoFast)
 };
 
 template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st);

@@ -233,12 +233,12 @@ static int set_device(smiler_index *idx) {
 }
 
 // smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
-constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
+constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
 constexpr int kMaxDI16 = 256;  // R17: 2046^2 (2d - 1) < 2^31 for d <= 256
 
 static int check_opts(const smiler_knn_opts &o) {
     const int v = o.variant;
-    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
+    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
         v != kVarTrimTwoStage)
         return fail(SMILER_EINVAL, "opts.variant %d is not a known kernel path", v);
 #if !SMILER_EXPERIMENTS
@@ -524,6 +524,7 @@ struct Plan {
     int lb_kind;     // smiler_knn_opts.lb_kind (SMILER_LB_*)
     bool direct;     // SMILER_LB_DIRECT*: lb_direct_kernel, no window level
     int RTf;         // fused: tile DWs per CTA
+    bool wave = false;  // opts.variant 3: the wavefront DTW kernel for every rho (A/B)
     size_t smem_gs, smem_fz;
 };
 
@@ -550,9 +551,7 @@ static int validate_query(smiler_index *idx, const int32_t *lengths_h, int n_len
         int r = rho_for(idx->band, pl.len[i]);
         pl.rho_env = std::max(pl.rho_env, r);  // R4: envelopes use rho_max
         pl.rho[i] = std::min(r, pl.len[i] - 1);  // rho >= d-1 is unconstrained DTW
-        if (pl.rho[i] > kMaxRhoFast)
-            return fail(SMILER_EINVAL, "warping width %d for d=%d exceeds the supported %d", r, pl.len[i],
-                        kMaxRhoFast);
+        // rho > kMaxRhoFast: the anti-diagonal wavefront kernel (any rho)
     }
     const size_t vs = 4;
     const int mmax = pl.D / pl.w;
@@ -619,6 +618,7 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
     p.tau_key = tau_key;
     p.fin = fin;
     p.fin_count = fin_count;
+    p.wave = pl.wave ? 1 : 0;
     launch_dtw<S>(pl.rho[li], p, 0, st);
     CHECK_LAUNCH();
     return SMILER_OK;
@@ -688,6 +688,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     if (o.lb_kind < SMILER_LB_INDEX || o.lb_kind > SMILER_LB_DIRECT_SHARED)
         return fail(SMILER_EINVAL, "lb_kind %d is not a SMILER_LB_* value", o.lb_kind);
     pl.lb_kind = o.lb_kind;
+    pl.wave = o.variant == kVarWaveDtw;
     if (o.horizon < 0) return fail(SMILER_EINVAL, "horizon must be >= 0");
     pl.direct = o.lb_kind >= SMILER_LB_DIRECT;
     if (pl.direct && (sctx || (lb_only && post_out)))
@@ -1776,7 +1777,7 @@ static int dtw_impl(smiler_index *idx, int32_t sensor, const void *q, int32_t d,
         return fail(SMILER_EINVAL, "I16: d = %d exceeds %d (int32 exactness, R17)", d, kMaxDI16);
     if (rho < 0) return fail(SMILER_EINVAL, "rho < 0");
     rho = std::min(rho, d - 1);
-    if (rho > kMaxRhoFast) return fail(SMILER_EINVAL, "rho %d exceeds %d", rho, kMaxRhoFast);
+    // rho > kMaxRhoFast runs the anti-diagonal wavefront kernel
     if (n_t < 1 || n_t > INT32_MAX / 2) return fail(SMILER_EINVAL, "bad n_t");
     std::vector<int64_t> th(n_t);
     if (is_device_ptr(ts)) CU(cudaMemcpy(th.data(), ts, 8 * n_t, cudaMemcpyDeviceToHost));

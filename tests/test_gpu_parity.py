@@ -125,7 +125,9 @@ def test_postings_and_lbw(pkg, orc, dtype, cfg, n, lengths, window, band):
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
 @pytest.mark.parametrize("d,rho", [(1, 0), (2, 1), (7, 3), (16, 1), (32, 4), (33, 8), (64, 6), (96, 8),
-                                   (128, 12), (128, 25), (100, 32), (20, 32), (300, 30), (1024, 5)])
+                                   (128, 12), (128, 25), (100, 32), (20, 32), (300, 30), (1024, 5),
+                                   # rho > 32: the anti-diagonal wavefront kernel (R23: any band)
+                                   (70, 33), (200, 60), (256, 255), (640, 100), (1024, 400)])
 def test_dtw_kernel(pkg, orc, dtype, d, rho):
     wl = synth.make_workload("C2", dtype, n=3000, mq_per_sensor=1, lengths=[max(d, 1)], window=1, band=1.0)
     rng = np.random.default_rng(d * 100 + rho)
@@ -779,3 +781,20 @@ def test_tight_lb_equals_tau_fp16_inexact(pkg, orc, dtype):
         assert oid[0, 0] == 0 and np.float64(dists[0, 0, 0]) == np.float64(od[0, 0])
         m_, _ = np.frexp(tau)
         assert m_ * 2.0 ** 11 != np.floor(m_ * 2.0 ** 11)   # needs > 11 significant bits: fp16-inexact at any scale
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_wide_band_knn(pkg, orc, dtype):
+    """A 50% band (rho_i = floor(0.5 d_i) up to 128 > 32): the wavefront DTW path
+    end to end, against the oracle."""
+    wl = synth.make_workload("C2", dtype, n=2500, mq_per_sensor=2, lengths=[64, 256], k=8, window=16, band=0.5)
+    assert max(wl.rhos()) == 128
+    check_workload(pkg, orc, wl)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_wavefront_variant_equals_register_band(pkg, orc, dtype):
+    """opts.variant 3 runs the wavefront DTW kernel for every rho (A/B): C5-shaped
+    bands {3, 6, 12, 25}, bit-exact with the oracle (the same cells, R16)."""
+    wl = synth.make_workload("C5", dtype, n=6007, n_sensors=2, mq_per_sensor=2)
+    check_workload(pkg, orc, wl, variant=3)
