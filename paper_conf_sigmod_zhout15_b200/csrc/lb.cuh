@@ -757,6 +757,9 @@ constexpr int kDiagCols = kDiagThreads + kDiagHaloMax;  // compile-time tile str
 // so that no bound of the MQ exceeds 65504 after scaling, R26).
 __device__ __forceinline__ __half lb_to_half(float v, float sc) { return __float2half_rd(v * sc); }
 __device__ __forceinline__ __half lb_to_half(int32_t v, float sc) { return __float2half_rd(__int2float_rd(v) * sc); }
+// LB x sc in f32, never above the exact product (the f32 product of a power of two is exact)
+__device__ __forceinline__ float lb_scaled_rd(float v, float sc) { return v * sc; }
+__device__ __forceinline__ float lb_scaled_rd(int32_t v, float sc) { return __int2float_rd(v) * sc; }
 
 template <typename V, int W, bool FASTMASK = true>
 __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, const MQMeta &m, const QParams &P,
@@ -814,12 +817,17 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
         __half *oh = reinterpret_cast<__half *>(lb) + m.seg_off + (int64_t)i * m.n + t0;
         const float sc = lbsc > 0.f ? lbsc : P.lbs[mq];
         if (vmask == kAll && W % 8 == 0 && ((reinterpret_cast<uintptr_t>(oh) & 15) == 0)) {
+            // bounds are >= 0, so rounding toward zero is rounding down: one packed
+            // conversion (cvt.rz.f16x2.f32) per two bounds
 #pragma unroll
             for (int b = 0; b < W; b += 8) {
-                __align__(16) __half hv[8];
+                uint32_t hw[4];
 #pragma unroll
-                for (int q = 0; q < 8; q++) hv[q] = lb_to_half(v[b + q], sc);
-                *reinterpret_cast<int4 *>(oh + b) = *reinterpret_cast<const int4 *>(hv);
+                for (int q = 0; q < 4; q++) {
+                    const float lo = lb_scaled_rd(v[b + 2 * q], sc), hi = lb_scaled_rd(v[b + 2 * q + 1], sc);
+                    asm("cvt.rz.f16x2.f32 %0, %1, %2;" : "=r"(hw[q]) : "f"(hi), "f"(lo));
+                }
+                *reinterpret_cast<int4 *>(oh + b) = make_int4((int)hw[0], (int)hw[1], (int)hw[2], (int)hw[3]);
             }
         } else {
 #pragma unroll
@@ -1651,25 +1659,33 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
     __syncthreads();
     if (x == 0)
         for (int g = 0; g < kTmaStages && g < g_end; g++) issue(g);
-    uint64_t emit_rows = 0, save_rows = 0;
-    for (int i = 0; i < nl; i++) {
-        const int qi = P.len[i] / W;
-        if (qi >= 1) emit_rows |= 1ull << (qi - 1);
-        if (qi >= 2) save_rows |= 1ull << (qi - 2);
+    // LB_w = max(S_EQ, S_EC) (Eq. 5) or one sum (Table 3 ablations): max(S_EQ fa, S_EC fb)
+    // with fa, fb in {0, 1} (sums are non-negative), times the fp16 ring's
+    // unscale factor 2^e (exact), all folded into the two factors
+    const V one = (V)1;
+    V fa = P.lbsel == 2 ? (V)0 : one, fb = P.lbsel == 1 ? (V)0 : one;
+    if constexpr (std::is_same<PV, __half>::value) {
+        fa *= P.post_unscale;
+        fb *= P.post_unscale;
     }
+    auto pick = [&](V a, V b) { return vmax(a * fa, b * fb); };
+    int i0 = 0;  // IQs shorter than W: no full DW (R6), emitted as LB_w = 0 after the rows
+    while (i0 < nl && P.len[i0] < W) i0++;
     int g = 0;
     for (int k = 0; k < my_tiles; k++) {
         const int tile = (int)blockIdx.x + k * (int)gridDim.x;
         const int mq = tile / nb, bx = tile - mq * nb;
-        // first used at the first emission row: the load overlaps the row loop
+        // first used at the first emission: the load overlaps the rows
         const MQMeta m = meta[mq];
+        const float lsc = P.lb_half ? P.lbs[mq] : 0.f;
         const int64_t Rb = (int64_t)bx * NT - 1;
-        const int64_t r = Rb + x;
-        const int64_t s0 = (r + 1) * W;  // e of slot b = 0
+        const int64_t s0 = (Rb + x + 1) * W;  // e of slot b = 0
         V se[W], sc[W];
 #pragma unroll
         for (int b = 0; b < W; b++) se[b] = sc[b] = (V)0;
-        for (int j = 0; j < mmax; j++, g++) {
+        // One CSG row: wait for its stage, add this thread's column, release the
+        // stage (one CTA barrier per two rows; thread 0 refills both stages).
+        auto row = [&](int j) {
             const int st = g & (kTmaStages - 1);
             mbar_wait(&s_full[st], (uint32_t)(g / kTmaStages) & 1u);
             const int nrow = n_sw - j * W;  // SWs of this CSG row (< W only in the last row)
@@ -1685,8 +1701,6 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
                 tma_row_add<V, PV, W, A, TP, false>(sb + 2 * W * NT + (xo - NT), nrow, se, sc);
             }
 #if SMILER_TMA_EMPTYBAR
-            // each warp releases stage st once its reads are done; thread 0 alone
-            // waits for all of them before refilling it (no CTA-wide barrier)
             __syncwarp();
             if ((x & 31) == 0) mbar_arrive(&s_empty[st]);
             if (x == 0 && g + kTmaStages < g_end) {
@@ -1696,51 +1710,57 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
             }
 #else
             if (SMILER_TMA_SYNC2 && kTmaStages >= 4) {
-            // one CTA barrier per two rows: after odd rows (and the CTA's last row)
-            // the stages of rows g-1 and g are free and are refilled together
-            if ((g & 1) || g + 1 == g_end) {
-                __syncthreads();  // every thread has read the stages of rows g-1, g
-                if (x == 0) {
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    if ((g & 1) && g - 1 + kTmaStages < g_end) issue(g - 1 + kTmaStages);
-                    if (g + kTmaStages < g_end) issue(g + kTmaStages);
-                }
-            }
-            } else {
-            __syncthreads();  // every thread has read stage st
-            if (x == 0 && g + kTmaStages < g_end) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                issue(g + kTmaStages);
-            }
-            }
-#endif
-            const bool live = bx < m.nblk;  // grids are sized for the longest sensor of the chunk
-            if (!live) continue;
-            if (emit_rows >> j & 1ull) {
-                for (int i = 0; i < nl; i++) {
-                    const int qi = P.len[i] / W, ri = P.len[i] % W;
-                    if (j == qi - 1) {
-                        V v[W];
-#pragma unroll
-                        for (int b = 0; b < W; b++)
-                            v[b] = b > ri ? (qi >= 2 ? s_saved[b][x] : (V)0) : lbpick(P, se[b], sc[b]);
-                        ring_unscale<V, PV, W>(v, P);
-                        diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq, bx);
+                if ((g & 1) || g + 1 == g_end) {
+                    __syncthreads();  // every thread has read the stages of rows g-1, g
+                    if (x == 0) {
+                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                        if ((g & 1) && g - 1 + kTmaStages < g_end) issue(g - 1 + kTmaStages);
+                        if (g + kTmaStages < g_end) issue(g + kTmaStages);
                     }
                 }
+            } else {
+                __syncthreads();
+                if (x == 0 && g + kTmaStages < g_end) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    issue(g + kTmaStages);
+                }
             }
-            if (save_rows >> j & 1ull) {
+#endif
+            g++;
+        };
+        // Rows run in segments ending at the emission rows (lengths ascending):
+        // IQ i (q_i = d_i / w, r_i = d_i % w) needs the sums after row q_i - 2
+        // (saved in shared memory, slots b > r_i: m_i(b) = q_i - 1) and after row
+        // q_i - 1 (slots b <= r_i).  An IQ with the q of the previous one reuses
+        // its saved values; q_i = 1 saves the zero sums.
+        int j = 0;
+        const bool live = bx < m.nblk;  // grids are sized for the longest sensor of the chunk
+        for (int i = i0; i < nl; i++) {
+            const int qi = P.len[i] / W, ri = P.len[i] % W;
+            for (; j < qi; j++) {
+                if (j == qi - 1) {
 #pragma unroll
-                for (int b = 0; b < W; b++) s_saved[b][x] = lbpick(P, se[b], sc[b]);
+                    for (int b = 0; b < W; b++) s_saved[b][x] = pick(se[b], sc[b]);
+                }
+                row(j);
+            }
+            if (live) {
+                V v[W];
+#pragma unroll
+                for (int b = 0; b < W; b++) {
+                    const V sv = s_saved[b][x];
+                    v[b] = b > ri ? sv : pick(se[b], sc[b]);
+                }
+                diag_emit<V, W>(v, i, s0, m, P, lb, tauc, mq, bx, lsc);
             }
         }
-        if (bx >= m.nblk) {
+        if (!live) {
             tau_clear(P, mq, NT / 32, 0, P.n_len, tauc, bx);
-        } else if (nl > 0 && P.len[0] < W) {  // IQs shorter than W: no full DW (R6), LB_w = 0
+        } else if (i0 > 0) {
             V z[W];
 #pragma unroll
             for (int b = 0; b < W; b++) z[b] = (V)0;
-            for (int i = 0; i < nl && P.len[i] < W; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq, bx);
+            for (int i = 0; i < i0; i++) diag_emit<V, W>(z, i, s0, m, P, lb, tauc, mq, bx, lsc);
         }
     }
 }

@@ -418,7 +418,7 @@ class Index:
     def knn(self, queries, lengths: Sequence[int], k: int, query_sensor=None, stats: bool = False,
             no_prune: bool = False, timing: bool = False, mq_chunk: int = 0, two_level: bool = False,
             lb_kind: int = 0, horizon: int = 0, shared_tau=None, tau_mult: int = 0, variant=0,
-            tau_keep: int = 0):
+            tau_keep: int = 0, exact_postings: bool = False):
         """kNN of every item query (smiler_knn_ex).  shared_tau: optional device
         buffer (torch int64 tensor of n_mq * n_len entries, all ones = -1 at start)
         shared by the window-range shards of one search (NEXT-2)."""
@@ -430,7 +430,8 @@ class Index:
         op = KnnOpts(no_prune=int(no_prune), timing=int(timing), mq_chunk=mq_chunk, two_level=int(two_level),
                      lb_kind=int(lb_kind), horizon=int(horizon), tau_mult=int(tau_mult),
                      variant=VARIANTS[variant] if isinstance(variant, str) else int(variant),
-                     tau_keep=int(tau_keep), shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
+                     tau_keep=int(tau_keep), exact_postings=int(exact_postings),
+                     shared_tau=_ptr(shared_tau) if shared_tau is not None else None)
         smiler_knn(self.handle, queries, query_sensor, lengths, k, ids, dists, st, op)
         if stats:
             return ids, dists, st.as_dict()

@@ -752,8 +752,14 @@ def test_i16_pruning_survives_tau_above_fp16_range(pkg, orc):
     q = np.stack([tail[0:128], tail[50:178]])
     with pkg.Index(series, None, 8, 0.1) as idx:
         ids, dists, st = idx.knn(q, [16, 32, 64, 128], 16, stats=True)
+        # the same search with the LB_w array in int32 (exact_postings: no fp16 storage)
+        ids_x, dists_x, st_x = idx.knn(q, [16, 32, 64, 128], 16, stats=True, exact_postings=True)
     assert int(dists[:, -1, -1].min()) > 65504 * 2          # tau well above the fp16 range
-    assert st["survivors"] < st["candidates"] // 4, st      # ... and the index still prunes
+    np.testing.assert_array_equal(ids, ids_x)
+    # the fp16 array prunes (almost) as well as the exact one: the unscaled array
+    # saturated and kept every candidate once tau passed 65504
+    assert st["survivors"] <= st_x["survivors"] * 1.02 + 64, (st, st_x)
+    assert st_x["survivors"] < 0.9 * st_x["candidates"], st_x
     for j in range(2):
         oid, od = orc.knn_one(series, q[j], [16, 32, 64, 128], [1, 3, 6, 12], 16, threads=THREADS)
         np.testing.assert_array_equal(ids[j], oid)
