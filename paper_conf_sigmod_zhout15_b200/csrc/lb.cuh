@@ -1173,6 +1173,9 @@ __global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_MINB8 : 3)
 // smem: qx [x2_pad + D] float4 | tile [kDiagCols][W + 1] float4 (column stride
 // W + 1: the 8 lanes of one LDS.128 phase hit distinct bank quads).
 // ---------------------------------------------------------------------------
+#ifndef SMILER_DIAG_X2_MINB16
+#define SMILER_DIAG_X2_MINB16 3
+#endif
 #ifndef SMILER_DIAG_X2_MINB8
 #define SMILER_DIAG_X2_MINB8 7  // 70 registers, no spills; C2 LB 8.25 ms (6: 8.27, 5: 8.58)
 #endif
@@ -1228,7 +1231,7 @@ __device__ __forceinline__ void x2_chunk_slot0(const float4 (&Pt)[W], const floa
 }
 
 template <int W>
-__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 : 3))
+__global__ void __launch_bounds__(kDiagThreads, (W <= 8 ? SMILER_DIAG_X2_MINB8 : SMILER_DIAG_X2_MINB16))
     lb_diag_x2_kernel(const float *series, const float *UC, const float *LC, const MQMeta *meta,
                       const float4 *qtab, const QParams P, float *lb, int32_t *tauc) {
     constexpr int NT = kDiagThreads;

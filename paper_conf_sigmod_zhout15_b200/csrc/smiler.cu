@@ -12,6 +12,7 @@
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <math.h>
+#include <nvtx3/nvToolsExt.h>
 #include <stdarg.h>
 #include <stdio.h>
 #include <string.h>
@@ -624,12 +625,26 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
     return SMILER_OK;
 }
 
+// NVTX ranges (host timeline; nsys / ncu attribute the kernels launched inside
+// them): one range per smiler_knn chunk phase, opened at each phase boundary.
+// Without an attached tool the NVTX calls are no-ops.
+static const char *const kPhaseName[8] = {"smiler a2 query prep", "smiler a3/a4 lower bounds",
+                                          "smiler a4 group scan", "smiler a5 tau",
+                                          "smiler a6 filter", "smiler a7 verify",
+                                          "smiler a8 select", nullptr};
 struct PhaseTimer {
     smiler_index *idx;
     bool on;
     std::vector<std::pair<int, int>> marks;  // (phase, event index)
     int next = 0;
+    bool nvtx_open = false;
+    ~PhaseTimer() {
+        if (nvtx_open) nvtxRangePop();
+    }
     int mark(int phase) {
+        if (nvtx_open) nvtxRangePop();
+        nvtx_open = phase < 7 && kPhaseName[phase];
+        if (nvtx_open) nvtxRangePushA(kPhaseName[phase]);
         if (!on) return SMILER_OK;
         if (next >= (int)idx->events.size()) {
             cudaEvent_t ev;
@@ -876,7 +891,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         ENS(idx->qtab.ensure(sizeof(V4) * (size_t)B * D));
         ENS(idx->lbs.ensure(sizeof(float) * (size_t)B));
         if (!sctx) ENS(idx->post.ensure(sizeof(V) * (size_t)std::max<int64_t>(post_tot, 1)));
-        ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
+        {
+            // the filter's 16-byte vector loads also touch the unwritten row tails
+            // (t > N - d_i) of the LB_w array (masked, never used): zero the buffer
+            // once when it grows so no read is of never-initialised memory
+            const void *before = idx->lb.p;
+            ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
+            if (idx->lb.p != before) CU(cudaMemsetAsync(idx->lb.p, 0, idx->lb.cap, idx->stream));
+        }
         if (!lb_only) {
             ENS(idx->surv.ensure(4 * (size_t)seg_tot));
             ENS(idx->fin.ensure(8 * (size_t)seg_tot));
@@ -1364,9 +1386,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     return SMILER_OK;
 }
 
+struct NvtxRange {
+    explicit NvtxRange(const char *n) { nvtxRangePushA(n); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 extern "C" int smiler_knn_ex(smiler_index *idx, const void *queries, const int32_t *query_sensor,
                              int32_t n_mq, const int32_t *lengths, int32_t n_len, int32_t k, int64_t *ids,
                              void *dists, smiler_knn_stats *stats, const smiler_knn_opts *opts) {
+    NvtxRange nr("smiler_knn");
     if (!idx) return fail(SMILER_EINVAL, "index is NULL");
     if (idx->dtype == SMILER_I16)
         return knn_impl<int16_t>(idx, queries, query_sensor, n_mq, lengths, n_len, k, ids, dists, stats,
@@ -1609,6 +1637,7 @@ extern "C" int smiler_stream_create(smiler_index *idx, const void *queries, cons
 
 extern "C" int smiler_stream_step(smiler_stream *st, const void *new_points, int64_t *ids, void *dists,
                                   smiler_knn_stats *stats, const smiler_knn_opts *opts) {
+    NvtxRange nr("smiler_stream_step");
     if (!st) return fail(SMILER_EINVAL, "stream is NULL");
     if (!new_points || !ids || !dists) return fail(SMILER_EINVAL, "NULL argument");
     smiler_index *idx = st->idx;
