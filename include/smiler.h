@@ -60,7 +60,7 @@ typedef enum {
 typedef struct smiler_knn_stats {
     int64_t candidates;   /* sum over (MQ, item query) of candidate starts t      */
     int64_t tau_verified; /* DTWs computed to set the thresholds tau_i (a5)       */
-    int64_t survivors;    /* candidates with LB_w <= tau_i, verified by DTW (a7)  */
+    int64_t survivors;    /* candidates with LB_w <= tau_i that a7 verified by DTW */
     int64_t finalists;    /* verified candidates with key <= tau key (a8 input)   */
     double dtw_cells;     /* banded-DTW cells evaluated (a5 + a7)                 */
     double bf_cells;      /* cells a brute-force scan of every candidate needs    */
@@ -70,6 +70,9 @@ typedef struct smiler_knn_stats {
     int32_t mq_chunks;
     double ns_prep, ns_window_lb, ns_group_scan, ns_tau, ns_filter, ns_verify, ns_select;
     double ns_total;
+    int64_t cascade_pruned;/* survivors of the index bound (a6) that the LB_Keogh cascade
+                              (LB_EQ with IQ_i's own envelope of width rho_i) dropped before
+                              a7; `survivors` counts the candidates a7 verified */
 } smiler_knn_stats;
 
 typedef struct smiler_knn_opts {
@@ -102,6 +105,7 @@ typedef struct smiler_knn_opts {
                          2 = scalar (not fp32x2-packed) diagonal LB kernel for F32,
                          3 = the anti-diagonal wavefront DTW kernel for every warping width
                          (by default it runs only for rho > 32, the register band below),
+                         4 = no LB_Keogh cascade between the filter and the verification,
                          7 = stream ring scanned without TMA, 8 = one tile per ring-scan CTA,
                          9 = radix-select tau-set trim, 10 = two-stage tau-set trim.  Any other
                          value is EINVAL */

@@ -60,6 +60,15 @@ __device__ __forceinline__ int32_t cell(int32_t q, int32_t c, int32_t m) {
     int32_t diff = q - c;
     return diff * diff + m;
 }
+// e(v; U, L) of Eq. 26 accumulated (the same arithmetic as the LB kernels' lb_term)
+__device__ __forceinline__ void lb_term(float v, float U, float L, float &acc) {
+    const float m = fmaxf(fmaxf(v - U, L - v), 0.0f);
+    acc = fmaf(m, m, acc);
+}
+__device__ __forceinline__ void lb_term(int32_t v, int32_t U, int32_t L, int32_t &acc) {
+    const int32_t dd = v - min(max(v, L), U);
+    acc += dd * dd;
+}
 template <typename V> __device__ __forceinline__ uint32_t vbits(V v);
 template <> __device__ __forceinline__ uint32_t vbits(float v) { return __float_as_uint(v); }
 template <> __device__ __forceinline__ uint32_t vbits(int32_t v) { return (uint32_t)v; }
@@ -442,6 +451,119 @@ template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, 
     }
     dispatch<S>(rho, p, grid, st, std::make_integer_sequence<int, kMaxRhoFast + 1>{});
 }
+
+// ---------------------------------------------------------------------------
+// LB_Keogh cascade (between a6 and a7).  The index bound LB_w (Thm 4.3) uses the
+// master query's envelope of width rho_max for every item query (R4, R20) and
+// only the candidate's full disjoint windows; LB_EQ(IQ_i, C_t) with IQ_i's own
+// envelope of width rho_i over all d_i points (Eq. 26, Keogh's bound for band
+// rho_i) is another lower bound of the same DTW, tighter for the short
+// item queries.  A survivor whose LB_EQ exceeds the admission threshold cannot be
+// among the k nearest (the same argument as the filter), so it is
+// dropped before its DTW.  Warp task = 32 survivors (one per lane), candidate
+// rows staged through shared memory exactly as the DTW kernel stages them; the
+// warp stops early once every lane's partial sum exceeds the threshold.
+// ---------------------------------------------------------------------------
+template <typename S>
+__global__ void __launch_bounds__(kDtwThreads) cascade_kernel(const CascadeParams<S> p) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    extern __shared__ __align__(16) unsigned char cz_smem[];
+    const int lane = threadIdx.x & 31;
+    const int wib = threadIdx.x >> 5;
+    const int d = p.d;
+    V2 *senv = reinterpret_cast<V2 *>(cz_smem) + (size_t)wib * (d + 32 * 33 / 2 + 1);
+    V (*s_c)[33] = reinterpret_cast<V (*)[33]>(senv + d);
+    const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nw = (gridDim.x * blockDim.x) >> 5;
+    const int total = p.task_off[p.n_mq];
+    int cur_mq = -1;
+    for (int task = gw; task < total; task += nw) {
+        int lo = 0, hi = p.n_mq;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (p.task_off[mid] <= task) lo = mid; else hi = mid;
+        }
+        const int mq = lo;
+        const int chunk = task - p.task_off[mq];
+        const MQMeta m = p.meta[mq];
+        const int seg = mq * p.n_len + p.li;
+        const int cnt = p.counts[seg];
+        const int64_t lbase = m.seg_off + (int64_t)p.li * m.n;
+        const int idx = chunk * 32 + lane;
+        const int t = idx < cnt ? p.list[lbase + idx] : -1;
+        V thr;
+        if constexpr (std::is_same<V, float>::value) thr = __uint_as_float(p.thr[seg]);
+        else thr = (int32_t)p.thr[seg];
+        if (mq != cur_mq) {  // IQ_li's own envelope, positions D - d .. D - 1
+            __syncwarp();
+            const V2 *e = p.qenv + ((int64_t)mq * p.n_len + p.li) * p.D + (p.D - d);
+            for (int x = lane; x < d; x += 32) senv[x] = e[x];
+            cur_mq = mq;
+        }
+        const S *cs = p.series + m.series_off;
+        V acc = (V)0;
+        for (int j0 = 0; j0 < d; j0 += 32) {
+            __syncwarp();
+            const bool in_row = (j0 + lane) < d;
+#pragma unroll 1
+            for (int l0 = 0; l0 < 32; l0 += 16) {
+                S vals[16];
+#pragma unroll
+                for (int q = 0; q < 16; q++) {
+                    const int tl = __shfl_sync(0xffffffffu, t, l0 + q);
+                    vals[q] = (tl >= 0 && in_row) ? __ldg(cs + tl + j0 + lane) : (S)0;
+                }
+#pragma unroll
+                for (int q = 0; q < 16; q++) s_c[lane][l0 + q] = (V)vals[q];
+            }
+            __syncwarp();
+            const int jn = min(32, d - j0);
+            for (int r = 0; r < jn; r++) {
+                const V2 e = senv[j0 + r];  // (U, L) at IQ position j0 + r
+                lb_term(s_c[r][lane], e.x, e.y, acc);
+            }
+            if (__all_sync(0xffffffffu, t < 0 || acc > thr)) break;  // every lane's bound already exceeds it
+        }
+        const bool keep = t >= 0 && acc <= thr;
+        const unsigned bal = __ballot_sync(0xffffffffu, keep);
+        if (bal) {
+            int base = 0;
+            if (lane == 0) base = atomicAdd(&p.out_counts[seg], __popc(bal));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (keep) p.out_list[lbase + base + __popc(bal & ((1u << lane) - 1))] = t;
+        }
+    }
+}
+
+template <typename S> void launch_cascade(const CascadeParams<S> &p, cudaStream_t st) {
+    using V = typename Tr<S>::V;
+    using V2 = typename Tr<S>::V2;
+    static std::mutex mu;
+    static std::map<int, int> sms_of;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int sms;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = sms_of.find(dev);
+        if (it == sms_of.end()) {
+            int n = 0;
+            cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+            cudaFuncSetAttribute(cascade_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)((size_t)kDtwWarps * (kMaxD * sizeof(V2) + (32 * 33 + 2) * sizeof(V))));
+            it = sms_of.emplace(dev, n > 0 ? n : 1).first;
+        }
+        sms = it->second;
+    }
+    const size_t smem = (size_t)kDtwWarps * (p.d + 32 * 33 / 2 + 1) * sizeof(V2);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, cascade_kernel<S>, kDtwThreads, smem);
+    cascade_kernel<S><<<sms * (occ > 0 ? occ : 1), kDtwThreads, smem, st>>>(p);
+}
+
+template void launch_cascade<int16_t>(const CascadeParams<int16_t> &, cudaStream_t);
+template void launch_cascade<float>(const CascadeParams<float> &, cudaStream_t);
 
 template void launch_dtw<int16_t>(int, const DtwParams<int16_t> &, int, cudaStream_t);
 template void launch_dtw<float>(int, const DtwParams<float> &, int, cudaStream_t);

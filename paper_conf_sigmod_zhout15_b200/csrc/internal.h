@@ -91,6 +91,31 @@ template <typename S> struct DtwParams {
 
 template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st);
 
+// LB_Keogh cascade between the filter (a6) and the DTW verification (a7) of one
+// item-query index li: every survivor of the index bound is re-bounded by
+// LB_EQ with the item query's own envelope (width rho_i, clipped to the item
+// query) over all d_i points, and kept only if that bound is <= the segment's
+// admission threshold.
+template <typename S> struct CascadeParams {
+    const S *series;
+    const MQMeta *meta;
+    const typename Tr<S>::V2 *qenv;  // [n_mq][n_len][D] (U, L) of IQ_i's own envelope (positions >= D - d_i)
+    int D, n_len, li, d, n_mq;
+    const int32_t *list;             // survivor t lists (segment layout)
+    const int32_t *counts;           // per segment
+    const int32_t *task_off;         // [n_mq + 1] prefix of warp tasks (32 survivors each)
+    const uint32_t *thr;             // per-segment admission bound (tau_select_kernel)
+    int32_t *out_list;               // kept t (segment layout)
+    int32_t *out_counts;             // per segment (zeroed by the caller)
+};
+template <typename S> void launch_cascade(const CascadeParams<S> &p, cudaStream_t st);
+
+// Item-query envelopes of the cascade: IQ_i's own envelope, width rho_i.
+struct IQTab {
+    int len[kMaxLen];
+    int rho[kMaxLen];
+};
+
 // Largest power of two 2^e (|e| <= 60) with bound x 2^e <= 65504 (fp16 max):
 // the storage scale of bounds that never exceed `bound` (R26).  Scaling by a
 // power of two is exact, so rounding the scaled value down to fp16 keeps it a

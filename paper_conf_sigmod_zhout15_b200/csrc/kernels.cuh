@@ -207,7 +207,8 @@ template <typename S>
 __global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D, int rho,
                                                         typename Tr<S>::V *qv,
                                                         typename Tr<S>::V4 *qtab, float smax,
-                                                        float *lbs, int *qflag) {
+                                                        float *lbs, int *qflag, const IQTab tab, int n_len,
+                                                        typename Tr<S>::V2 *qenv) {
     using V = typename Tr<S>::V;
     using V4 = typename Tr<S>::V4;
     __shared__ V s[kMaxD];
@@ -250,6 +251,27 @@ __global__ void __launch_bounds__(256) query_prep_kernel(const S *queries, int D
         e.z = mn;
         e.w = (V)0;
         qtab[(int64_t)mq * D + p] = e;
+    }
+    // the cascade's item-query envelopes: IQ_i = MQ[D - d_i, D) with width rho_i,
+    // clipped to the item query (Eq. 25 over IQ_i itself, R3)
+    if (qenv) {
+        for (int i = 0; i < n_len; i++) {
+            const int a = D - tab.len[i], r = tab.rho[i];
+            typename Tr<S>::V2 *o = qenv + ((int64_t)mq * n_len + i) * D;
+            for (int p = a + threadIdx.x; p < D; p += blockDim.x) {
+                const int lo = p - r < a ? a : p - r;
+                const int hi = p + r > D - 1 ? D - 1 : p + r;
+                V mx = s[lo], mn = s[lo];
+                for (int y = lo + 1; y <= hi; y++) {
+                    mx = s[y] > mx ? s[y] : mx;
+                    mn = s[y] < mn ? s[y] : mn;
+                }
+                typename Tr<S>::V2 e2;
+                e2.x = mx;
+                e2.y = mn;
+                o[p] = e2;
+            }
+        }
     }
 }
 
@@ -796,12 +818,14 @@ __global__ void prev_tau_kernel(const int64_t *prev, int shift, const MQMeta *me
     }
 }
 
-// Stats: acc[0] += finalists, acc[1 + i] += survivors of item query i.
-__global__ void accum_counts_kernel(const int32_t *scount, const int32_t *fcount, int nseg, int n_len,
-                                    unsigned long long *acc) {
+// Stats: acc[0] += finalists, acc[1 + i] += candidates DTW-verified for item
+// query i (a7), acc[1 + kMaxLen + i] += survivors of a6 the cascade dropped.
+__global__ void accum_counts_kernel(const int32_t *vcount, const int32_t *scount, const int32_t *fcount, int nseg,
+                                    int n_len, unsigned long long *acc) {
     for (int s = threadIdx.x; s < nseg; s += blockDim.x) {
         atomicAdd(&acc[0], (unsigned long long)fcount[s]);
-        atomicAdd(&acc[1 + s % n_len], (unsigned long long)scount[s]);
+        atomicAdd(&acc[1 + s % n_len], (unsigned long long)vcount[s]);
+        atomicAdd(&acc[1 + kMaxLen + s % n_len], (unsigned long long)(scount[s] - vcount[s]));
     }
 }
 

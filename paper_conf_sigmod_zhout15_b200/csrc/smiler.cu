@@ -147,7 +147,7 @@ struct smiler_index {
     int *qflag_d = nullptr;    // its device alias (written by query_prep_kernel)
     // workspace
     DevBuf queries, qv, qtab, meta, post, lb, surv, fin, tauc, taulb, tauk, taukey, thr, scount, fcount,
-        taskoff, out_ids, out_d, tmp, tmp2, pred, lbs;
+        taskoff, out_ids, out_d, tmp, tmp2, pred, lbs, qenv, surv2, scount2;
     std::vector<cudaEvent_t> events;
     size_t budget = (size_t)24 << 30;  // workspace bytes per chunk (set at build)
     // pinned staging ring for per-chunk metadata (async H2D without host sync)
@@ -234,12 +234,13 @@ static int set_device(smiler_index *idx) {
 }
 
 // smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
-constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
+constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarNoCascade = 4, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
 constexpr int kMaxDI16 = 256;  // R17: 2046^2 (2d - 1) < 2^31 for d <= 256
 
 static int check_opts(const smiler_knn_opts &o) {
     const int v = o.variant;
-    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
+    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarNoCascade &&
+        v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
         v != kVarTrimTwoStage)
         return fail(SMILER_EINVAL, "opts.variant %d is not a known kernel path", v);
 #if !SMILER_EXPERIMENTS
@@ -369,7 +370,8 @@ static void destroy(smiler_index *idx) {
     DevBuf *bufs[] = {&idx->queries, &idx->qv,     &idx->qtab,   &idx->meta,   &idx->post,
                       &idx->lb,      &idx->surv,   &idx->fin,    &idx->tauc,   &idx->taulb,  &idx->tauk,
                       &idx->taukey,  &idx->thr,    &idx->scount, &idx->fcount, &idx->taskoff,
-                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred,   &idx->lbs};
+                      &idx->out_ids, &idx->out_d,  &idx->tmp,    &idx->tmp2,   &idx->pred,   &idx->lbs,
+                      &idx->qenv,    &idx->surv2,  &idx->scount2};
     for (DevBuf *b : bufs) b->release();
     for (auto ev : idx->events) cudaEventDestroy(ev);
     for (int i = 0; i < kMaxLen; i++) {
@@ -775,14 +777,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
 
     if (stats) {
         memset(stats, 0, sizeof(*stats));
-        TRY(idx->tmp.ensure(8 * (kMaxLen + 1)));
-        CU(cudaMemsetAsync(idx->tmp.p, 0, 8 * (kMaxLen + 1), idx->stream));
+        TRY(idx->tmp.ensure(8 * (2 * kMaxLen + 1)));
+        CU(cudaMemsetAsync(idx->tmp.p, 0, 8 * (2 * kMaxLen + 1), idx->stream));
     }
     PhaseTimer tm{idx, stats != nullptr && o.timing != 0};
     int launches = 0;
     int64_t tau_slots_total = 0;
     double cells_acc = 0, bf_cells = 0;
-    int64_t cand_total = 0, surv_total = 0, fin_total = 0, post_bytes = 0, lb_bytes = 0;
+    int64_t cand_total = 0, surv_total = 0, fin_total = 0, post_bytes = 0, lb_bytes = 0, casc_total = 0;
     int n_chunks = 0;
 
     for (int c0 = 0; c0 < n_mq;) {
@@ -843,6 +845,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                                                                      : 1;
         int E = 0;
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
+        // LB_Keogh cascade between a6 and a7 (launch_cascade); variant 4 skips it (A/B)
+        const bool cascade = !lb_only && !o.no_prune && o.variant != kVarNoCascade;
         if (!lb_only && !o.no_prune) {
             const int umin = nblk_min * units_per_blk;
             // tau set ~ mult * k tile candidates per IQ (plus k shifted previous
@@ -899,6 +903,11 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             ENS(idx->lb.ensure(sizeof(V) * (size_t)seg_tot));
             if (idx->lb.p != before) CU(cudaMemsetAsync(idx->lb.p, 0, idx->lb.cap, idx->stream));
         }
+        if (cascade) {
+            ENS(idx->qenv.ensure(sizeof(V2) * (size_t)B * nl * D));
+            ENS(idx->surv2.ensure(4 * (size_t)seg_tot));
+            ENS(idx->scount2.ensure(4 * (size_t)nseg));
+        }
         if (!lb_only) {
             ENS(idx->surv.ensure(4 * (size_t)seg_tot));
             ENS(idx->fin.ensure(8 * (size_t)seg_tot));
@@ -909,7 +918,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             ENS(idx->thr.ensure(4 * (size_t)nseg));
             ENS(idx->scount.ensure(4 * (size_t)nseg));
             ENS(idx->fcount.ensure(4 * (size_t)nseg));
-            ENS(idx->taskoff.ensure(4 * (size_t)(B + 1) * nl * 2));
+            ENS(idx->taskoff.ensure(4 * (size_t)(B + 1) * nl * 3));
             ENS(idx->out_ids.ensure(8 * (size_t)nseg * pl.k));
             ENS(idx->out_d.ensure(4 * (size_t)nseg * pl.k));
         }
@@ -1047,9 +1056,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         P.post_unscale = (sctx && sctx->post_half) ? 1.0f / sctx->pscale : 1.0f;
         TRY(tm.mark(0));
         // ---- a2 ----------------------------------------------------------
+        IQTab iqt;
+        for (int i = 0; i < nl; i++) {
+            iqt.len[i] = pl.len[i];
+            iqt.rho[i] = pl.rho[i];
+        }
         query_prep_kernel<S><<<B, 256, 0, idx->stream>>>(idx->queries.as<S>(), D, pl.rho_env, idx->qv.as<V>(),
                                                          idx->qtab.as<V4>(), idx->smax, idx->lbs.as<float>(),
-                                                         idx->qflag_d);
+                                                         idx->qflag_d, iqt, nl,
+                                                         cascade ? idx->qenv.as<V2>() : nullptr);
         CHECK_LAUNCH();
         launches++;
         TRY(tm.mark(1));
@@ -1314,13 +1329,43 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
         }
         TRY(tm.mark(5));
-        // ---- a7 ----------------------------------------------------------
+        // ---- a6b cascade + a7 (per item query on its side stream) ---------
         int32_t *taskoff2 = taskoff + (size_t)nl * (B + 1);
+        int32_t *taskoff3 = taskoff + (size_t)2 * nl * (B + 1);
+        const int32_t *vlist = idx->surv.as<int32_t>();
+        const int32_t *vcnt = scount;
+        if (cascade) {
+            CU(cudaMemsetAsync(idx->scount2.p, 0, 4 * (size_t)nseg, idx->stream));
+            vlist = idx->surv2.as<int32_t>();
+            vcnt = idx->scount2.as<int32_t>();
+        }
         TRY(side_fork(idx, nl));
         for (int i = 0; i < nl; i++) {
-            TRY(run_dtw_list<S>(idx, pl, i, B, 1, idx->surv.as<int32_t>(), 0, scount,
-                                taskoff2 + (size_t)i * (B + 1), nullptr, taukey, idx->fin.as<uint64_t>(),
-                                fcount, d_meta, idx->qv.as<V>(), D, idx->side[i]));
+            if (cascade) {
+                int32_t *to = taskoff3 + (size_t)i * (B + 1);
+                task_prefix_kernel<<<1, 1024, 0, idx->side[i]>>>(scount, -1, B, nl, i, to);
+                CHECK_LAUNCH();
+                CascadeParams<S> cp;
+                cp.series = (const S *)idx->d_series;
+                cp.meta = d_meta;
+                cp.qenv = idx->qenv.as<V2>();
+                cp.D = D;
+                cp.n_len = nl;
+                cp.li = i;
+                cp.d = pl.len[i];
+                cp.n_mq = B;
+                cp.list = idx->surv.as<int32_t>();
+                cp.counts = scount;
+                cp.task_off = to;
+                cp.thr = thr;
+                cp.out_list = idx->surv2.as<int32_t>();
+                cp.out_counts = idx->scount2.as<int32_t>();
+                launch_cascade<S>(cp, idx->side[i]);
+                CHECK_LAUNCH();
+                launches += 2;
+            }
+            TRY(run_dtw_list<S>(idx, pl, i, B, 1, vlist, 0, vcnt, taskoff2 + (size_t)i * (B + 1), nullptr, taukey,
+                                idx->fin.as<uint64_t>(), fcount, d_meta, idx->qv.as<V>(), D, idx->side[i]));
             launches += 2;
         }
         TRY(side_join(idx, nl));
@@ -1340,15 +1385,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             CU(cudaMemcpyAsync(sctx->d_prev_out + (size_t)c0 * nl * pl.k, idx->out_ids.p, 8 * ob,
                                cudaMemcpyDeviceToDevice, idx->stream));
         if (stats) {
-            accum_counts_kernel<<<1, 256, 0, idx->stream>>>(scount, fcount, nseg, nl,
+            accum_counts_kernel<<<1, 256, 0, idx->stream>>>(vcnt, scount, fcount, nseg, nl,
                                                             idx->tmp.as<unsigned long long>());
             CHECK_LAUNCH();
         }
         c0 = c1;
     }
-    unsigned long long acc_h[kMaxLen + 1] = {0};
+    unsigned long long acc_h[2 * kMaxLen + 1] = {0};
     if (stats && !lb_only)
-        CU(cudaMemcpyAsync(acc_h, idx->tmp.p, 8 * (kMaxLen + 1), cudaMemcpyDeviceToHost, idx->stream));
+        CU(cudaMemcpyAsync(acc_h, idx->tmp.p, 8 * (2 * kMaxLen + 1), cudaMemcpyDeviceToHost, idx->stream));
     if (!out_dev || stats) {
         CU(cudaStreamSynchronize(idx->stream));
         TRY(take_qflag(idx));
@@ -1358,11 +1403,13 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         fin_total = (int64_t)acc_h[0];
         for (int i = 0; i < nl; i++) {
             surv_total += (int64_t)acc_h[1 + i];
+            casc_total += (int64_t)acc_h[1 + kMaxLen + i];
             cells_acc += (double)acc_h[1 + i] * (double)dtw_cells(pl.len[i], pl.rho[i]);
         }
         stats->candidates = cand_total;
         stats->tau_verified = tau_slots_total;
         stats->survivors = surv_total;
+        stats->cascade_pruned = casc_total;
         stats->finalists = fin_total;
         stats->dtw_cells = cells_acc;
         stats->bf_cells = bf_cells;
@@ -1834,7 +1881,7 @@ static int dtw_impl(smiler_index *idx, int32_t sensor, const void *q, int32_t d,
     CU(cudaMemcpyAsync(idx->tauc.p, t32.data(), 4 * n_t, cudaMemcpyHostToDevice, idx->stream));
     query_prep_kernel<S><<<1, 256, 0, idx->stream>>>(idx->queries.as<S>(), d, 0, idx->qv.as<V>(),
                                                      idx->qtab.as<typename Tr<S>::V4>(), 0.f, nullptr,
-                                                     idx->qflag_d);
+                                                     idx->qflag_d, IQTab{}, 0, nullptr);
     CHECK_LAUNCH();
     Plan pl;
     pl.n_len = 1;

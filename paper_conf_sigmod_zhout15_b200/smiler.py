@@ -37,7 +37,8 @@ class KnnStats(ctypes.Structure):
                 ("ns_prep", ctypes.c_double), ("ns_window_lb", ctypes.c_double),
                 ("ns_group_scan", ctypes.c_double), ("ns_tau", ctypes.c_double),
                 ("ns_filter", ctypes.c_double), ("ns_verify", ctypes.c_double),
-                ("ns_select", ctypes.c_double), ("ns_total", ctypes.c_double)]
+                ("ns_select", ctypes.c_double), ("ns_total", ctypes.c_double),
+                ("cascade_pruned", ctypes.c_int64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -52,7 +53,7 @@ class KnnOpts(ctypes.Structure):
 
 
 # smiler_knn_opts.variant: kernel paths with the same (exact) result, for tests and A/B timing
-VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
+VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "no_cascade": 4, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
