@@ -12,18 +12,20 @@ cfg = sys.argv[1] if len(sys.argv) > 1 else "C5"
 dtype = sys.argv[2] if len(sys.argv) > 2 else "f32"
 ns = int(sys.argv[3]) if len(sys.argv) > 3 else 256
 steps = int(sys.argv[4]) if len(sys.argv) > 4 else 4
-wl = synth.make_workload(cfg, dtype, n_sensors=ns, consecutive=True)
-nxt = synth.make_workload(cfg, dtype, n_sensors=ns, consecutive=True, step=steps)
+wl = synth.make_workload(cfg, dtype, n_sensors=ns)
 idx = pkg.Index(wl.series, wl.offsets, wl.window, wl.band)
 exact = len(sys.argv) > 5 and sys.argv[5] == "exact"
 st = pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor, exact_postings=exact)
 D = wl.D
 acc = {}
-for s in range(steps):
+chunks = 1
+for s in range(1, steps + 1):
     # the next point of every stream (a real feed would supply it)
-    newp = np.ascontiguousarray(nxt.queries[:, D - steps + s]) if s < steps else None
-    _, _, stt = st.step(newp, stats=True, timing=True)
+    _, _, stt = st.step(wl.new_points(s), stats=True, timing=True)
+    chunks = stt["mq_chunks"]
     for k, v in stt.items():
         if k.startswith("ns_"):
             acc[k] = acc.get(k, 0) + v / 1e6 / steps
 print(cfg, dtype, ns, {k: round(v, 3) for k, v in acc.items()})
+# master queries per launch of the per-chunk kernels (ncu traffic normalisation)
+print("MQ_PER_LAUNCH=%d" % ((wl.n_mq + chunks - 1) // chunks))
