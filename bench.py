@@ -699,8 +699,9 @@ def main():
     post_bytes_step = pair_bytes * n_sw * sum(p // wl.window for p in pts)
     # LB_w array entry: fp16 rounded down on the product path (one direction of the
     # library's lb_bytes stat, which counts the a4 write and the a6 read), else 4 B
-    lb_entry = (acc["lb_bytes"] / (2.0 * n_len * sum(pts) * steps)) if acc["lb_bytes"] else 4.0
-    lb_bytes_step = lb_entry * n_len * sum(pts)
+    # (the library's lb_bytes counts the a4 write and the a6 read; 0 when the filter
+    # runs inside the scan and no LB_w array exists: lagged stream steps, fused a4+a6)
+    lb_bytes_step = acc["lb_bytes"] / 2.0 / steps
 
     # continuous streams recompute only SW_0 (EQ + EC) and SW_1..SW_rho_max (EQ):
     # (rho_max + 2) / 2 term-pair equivalents per (DW, j) instead of n_sw
@@ -709,6 +710,7 @@ def main():
 
     def rooflines(ph, ac, nsteps, fused):
         ks = {}
+        lbb = ac["lb_bytes"] / 2.0 / nsteps  # the LB_w array written by a4 / read by a6 (0 if fused)
         win_s = ph["ns_window_lb"] / 1e9 / nsteps
         if win_s > 0:
             terms = inc_terms if R.streaming else win_terms
@@ -720,7 +722,7 @@ def main():
                                                                      // wl.n_mq)}
         gs_s = ph["ns_group_scan"] / 1e9 / nsteps
         if not fused and gs_s > 0:
-            byts = post_bytes_step + lb_bytes_step
+            byts = post_bytes_step + lbb
             gbs = byts / gs_s / 1e9
             ks["group_scan_a4"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                                    "frac": gbs / peaks["hbm_gbs"], "ms": gs_s * 1e3,
@@ -731,8 +733,8 @@ def main():
             ks["dtw_verify_a7"] = {"bound": "alu", "achieved": cr / 1e12, "peak": cell_peak / 1e12,
                                    "unit": "T DTW cells/s", "frac": cr / cell_peak, "ms": v_s * 1e3}
         f_s = ph["ns_filter"] / 1e9 / nsteps
-        if f_s > 0:
-            gbs = lb_bytes_step / f_s / 1e9
+        if f_s > 0 and lbb > 0:
+            gbs = lbb / f_s / 1e9
             ks["filter_a6"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                                "frac": gbs / peaks["hbm_gbs"], "ms": f_s * 1e3}
         return ks

@@ -106,6 +106,8 @@ typedef struct smiler_knn_opts {
                          3 = the anti-diagonal wavefront DTW kernel for every warping width
                          (by default it runs only for rho > 32, the register band below),
                          4 = no LB_Keogh cascade between the filter and the verification,
+                         5 = stream steps without the lagged tile tau set (thresholds after
+                         the scan, LB_w array + filter pass),
                          7 = stream ring scanned without TMA, 8 = one tile per ring-scan CTA,
                          9 = radix-select tau-set trim, 10 = two-stage tau-set trim.  Any other
                          value is EINVAL */

@@ -818,6 +818,26 @@ __global__ void prev_tau_kernel(const int64_t *prev, int shift, const MQMeta *me
     }
 }
 
+// Lagged tile tau set (stream steps): the previous call's scan-unit candidates
+// of each (stream, item query), shifted by the one-point advance, become the
+// tile part [0, LTt) of this step's tau list with their (previous) LB_w bits as
+// trim keys; a shifted t outside the owned range is dropped (-1).
+__global__ void lag_tau_kernel(const int32_t *lag_t, const uint32_t *lag_lb, int LTt, const MQMeta *meta,
+                               const QParams P, int32_t *tauc, uint32_t *taulb) {
+    const int seg = blockIdx.y;
+    const int x = blockIdx.x * blockDim.x + threadIdx.x;
+    if (x >= LTt) return;
+    const int mq = seg / P.n_len, i = seg % P.n_len;
+    const MQMeta m = meta[mq];
+    const int64_t tb = m.t_lo > 0 ? m.t_lo : 0;
+    const int64_t te = min(m.t_hi, m.n - m.hz - P.len[i] + 1);
+    const int32_t t = lag_t[(int64_t)seg * LTt + x];
+    const int64_t t1 = t >= 0 ? (int64_t)t + 1 : -1;
+    const bool ok = t1 >= tb && t1 < te;
+    tauc[(int64_t)seg * P.LT + x] = ok ? (int32_t)t1 : -1;
+    taulb[(int64_t)seg * P.LT + x] = ok ? lag_lb[(int64_t)seg * LTt + x] : 0xFFFFFFFFu;
+}
+
 // Stats: acc[0] += finalists, acc[1 + i] += candidates DTW-verified for item
 // query i (a7), acc[1 + kMaxLen + i] += survivors of a6 the cascade dropped.
 __global__ void accum_counts_kernel(const int32_t *vcount, const int32_t *scount, const int32_t *fcount, int nseg,

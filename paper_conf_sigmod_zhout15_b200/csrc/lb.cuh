@@ -794,26 +794,27 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
             keep |= (uint32_t)k_ << b;
         }
         keep &= vmask;
-        const int lane = threadIdx.x & 31;
-        const int cnt = __popc(keep);
-        int x = cnt;
+        if (__any_sync(0xffffffffu, keep)) {  // survivors are rare: most warps skip the append
+            const int lane = threadIdx.x & 31;
+            const int cnt = __popc(keep);
+            int x = cnt;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= o) x += y;
+            }
+            const int total = __shfl_sync(0xffffffffu, x, 31);
+            int base = 0;
+            if (lane == 31 && total) base = atomicAdd(&P.scount[seg], total);
+            base = __shfl_sync(0xffffffffu, base, 31);
+            int o = base + x - cnt;
+            int32_t *dst = P.surv + m.seg_off + (int64_t)i * m.n;
+#pragma unroll
+            for (int b = 0; b < W; b++)
+                if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
         }
-        const int total = __shfl_sync(0xffffffffu, x, 31);
-        int base = 0;
-        if (lane == 31 && total) base = atomicAdd(&P.scount[seg], total);
-        base = __shfl_sync(0xffffffffu, base, 31);
-        int o = base + x - cnt;
-        int32_t *dst = P.surv + m.seg_off + (int64_t)i * m.n;
-#pragma unroll
-        for (int b = 0; b < W; b++)
-            if (keep >> b & 1u) dst[o++] = (int32_t)(t0 + b);
-        return;
-    }
-    if (P.lb_half) {  // LB_w array as scaled fp16 rounded down (a valid, slightly looser bound)
+        if (P.E <= 0) return;  // a lagged stream step still picks the next step's tile tau set
+    } else if (P.lb_half) {  // LB_w array as scaled fp16 rounded down (a valid, slightly looser bound)
         __half *oh = reinterpret_cast<__half *>(lb) + m.seg_off + (int64_t)i * m.n + t0;
         const float sc = lbsc > 0.f ? lbsc : P.lbs[mq];
         if (vmask == kAll && W % 8 == 0 && ((reinterpret_cast<uintptr_t>(oh) & 15) == 0)) {

@@ -234,12 +234,13 @@ static int set_device(smiler_index *idx) {
 }
 
 // smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
-constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarNoCascade = 4, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
+constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarNoCascade = 4, kVarNoLag = 5,
+              kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
 constexpr int kMaxDI16 = 256;  // R17: 2046^2 (2d - 1) < 2^31 for d <= 256
 
 static int check_opts(const smiler_knn_opts &o) {
     const int v = o.variant;
-    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarNoCascade &&
+    if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarNoCascade && v != kVarNoLag &&
         v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
         v != kVarTrimTwoStage)
         return fail(SMILER_EINVAL, "opts.variant %d is not a known kernel path", v);
@@ -675,6 +676,11 @@ struct StreamCtx {
     const CUtensorMap *tmap;   // the ring as one 2-D tensor (tma): w x 256 boxes
     const CUtensorMap *tmap_tail;  // the same tensor, w x (16 bytes) boxes
     float pscale;              // fp16 ring: entries hold P x pscale (a power of two, R26)
+    // lagged tile tau set (stream steps): this step's scan-unit candidates are kept
+    // per stream and, shifted by one point, form the next step's tile tau set, so
+    // the thresholds exist before the next scan and the filter runs inside it
+    DevBuf *lag_t, *lag_lb;    // [n_streams][n_len][lag_LTt] t and LB_w bits
+    int *lag_LTt;              // entries per (stream, item query) saved by the last call; -1 = none
 };
 
 template <typename S>
@@ -785,6 +791,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
     int64_t tau_slots_total = 0;
     double cells_acc = 0, bf_cells = 0;
     int64_t cand_total = 0, surv_total = 0, fin_total = 0, post_bytes = 0, lb_bytes = 0, casc_total = 0;
+    int lag_LTt_seen = -2;  // -2: no chunk saved yet; -1: chunks differ (no lagged set next step)
     int n_chunks = 0;
 
     for (int c0 = 0; c0 < n_mq;) {
@@ -1047,7 +1054,20 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // each LB_w with tau_i as it is produced and appends the survivors; the
         // LB_w array is never written or re-read (P:1437-1448 in one pass).
         const bool diag_emitters = pl.direct || (pl.fused && pl.fused_kind == 0) || (!pl.fused && pl.scan_reg);
-        const bool fuse = use_prev && E == 0 && !lb_only && !o.no_prune && diag_emitters;
+        // Stream calls keep this scan's tile tau candidates (lag_save); a stream step
+        // whose previous call saved them (same list shape) verifies them, shifted by
+        // the one-point advance (the continuation of a good candidate, as R9 shifts
+        // the previous neighbours), with the previous neighbours BEFORE its scan:
+        // any >= k verified candidates give a valid tau (R8), so the thresholds
+        // exist before the scan and the filter runs inside it (lagged fuse).
+        const bool lag_save = sctx && !lb_only && !o.no_prune && E > 0 && diag_emitters &&
+                              o.variant != kVarNoLag;
+        const bool lagged = lag_save && sctx->mode == 1 && use_prev && *sctx->lag_LTt == LTt;
+        const bool fuse = (use_prev && E == 0 && !lb_only && !o.no_prune && diag_emitters) || lagged;
+        if (lag_save) {
+            TRY(sctx->lag_t->ensure(4 * (size_t)n_mq * nl * LTt));
+            TRY(sctx->lag_lb->ensure(4 * (size_t)n_mq * nl * LTt));
+        }
         // LB_w array as fp16 rounded down for the filter (its only reader besides the
         // tau trim, which takes the bounds from P.taulb): half the bytes written by
         // a4 and read by a6.  lb_only (smiler_lower_bounds) and exact_postings keep V.
@@ -1069,6 +1089,14 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         launches++;
         TRY(tm.mark(1));
         if (fuse) {
+            if (lagged) {  // the previous call's tile candidates, shifted by one point
+                dim3 g((unsigned)((LTt + 255) / 256), (unsigned)nseg);
+                lag_tau_kernel<<<g, 256, 0, idx->stream>>>(sctx->lag_t->as<int32_t>() + (size_t)c0 * nl * LTt,
+                                                          sctx->lag_lb->as<uint32_t>() + (size_t)c0 * nl * LTt, LTt,
+                                                          d_meta, P, idx->tauc.as<int32_t>(), idx->taulb.as<uint32_t>());
+                CHECK_LAUNCH();
+                launches++;
+            }
             TRY(do_a5());
             TRY(tm.mark(4));
             P.fuse = 1;
@@ -1301,6 +1329,15 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             c0 = c1;
             continue;
         }
+        if (lag_save) {  // this scan's tile candidates (before a5's trim reorders them)
+            CU(cudaMemcpy2DAsync(sctx->lag_t->as<int32_t>() + (size_t)c0 * nl * LTt, 4 * (size_t)LTt,
+                                 idx->tauc.p, 4 * (size_t)LT, 4 * (size_t)LTt, (size_t)nseg, cudaMemcpyDeviceToDevice,
+                                 idx->stream));
+            CU(cudaMemcpy2DAsync(sctx->lag_lb->as<uint32_t>() + (size_t)c0 * nl * LTt, 4 * (size_t)LTt,
+                                 idx->taulb.p, 4 * (size_t)LT, 4 * (size_t)LTt, (size_t)nseg, cudaMemcpyDeviceToDevice,
+                                 idx->stream));
+            lag_LTt_seen = lag_LTt_seen == -2 ? LTt : (lag_LTt_seen == LTt ? LTt : -1);
+        }
         if (!fuse) TRY(do_a5());
         TRY(tm.mark(4));
         // ---- a6 ----------------------------------------------------------
@@ -1391,6 +1428,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         }
         c0 = c1;
     }
+    if (sctx) *sctx->lag_LTt = lag_LTt_seen >= 0 ? lag_LTt_seen : -1;  // the next step may use the saved lists
     unsigned long long acc_h[2 * kMaxLen + 1] = {0};
     if (stats && !lb_only)
         CU(cudaMemcpyAsync(acc_h, idx->tmp.p, 8 * (2 * kMaxLen + 1), cudaMemcpyDeviceToHost, idx->stream));
@@ -1489,6 +1527,8 @@ struct smiler_stream {
     int prows = 0;             // ring rows per plane
     CUtensorMap tmap, tmap_tail;
     float pscale = 1.f;        // fp16 ring storage scale (power of two)
+    DevBuf lag_t, lag_lb;      // lagged tile tau set (StreamCtx)
+    int lag_LTt = -1;
     int cursor = 0;
     int64_t steps = 0;
 };
@@ -1501,6 +1541,8 @@ static void stream_release(smiler_stream *st) {
     if (st->d_new) cudaFree(st->d_new);
     if (st->ring) cudaFree(st->ring);
     if (st->d_prev) cudaFree(st->d_prev);
+    st->lag_t.release();
+    st->lag_lb.release();
     delete st;
 }
 
@@ -1521,6 +1563,9 @@ static int stream_run(smiler_stream *st, int64_t *ids, void *dists, smiler_knn_s
     sc.tmap = &st->tmap;
     sc.tmap_tail = &st->tmap_tail;
     sc.pscale = st->pscale;
+    sc.lag_t = &st->lag_t;
+    sc.lag_lb = &st->lag_lb;
+    sc.lag_LTt = &st->lag_LTt;
     return knn_impl<S>(st->idx, st->d_mq, st->qsens.data(), st->n, st->lens.data(), st->n_len, st->k, ids, dists,
                        stats, opts, false, nullptr, nullptr, mode == 1 ? st->d_prev : nullptr, 1, &sc);
 }

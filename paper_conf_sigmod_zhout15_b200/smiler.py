@@ -53,7 +53,7 @@ class KnnOpts(ctypes.Structure):
 
 
 # smiler_knn_opts.variant: kernel paths with the same (exact) result, for tests and A/B timing
-VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "no_cascade": 4, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
+VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "no_cascade": 4, "no_lag": 5, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates
@@ -369,7 +369,7 @@ class Stream:
                                            ids, dists, KnnOpts(exact_postings=int(exact_postings)))
         self.first = (ids, dists)
 
-    def step(self, new_points, stats: bool = False, timing: bool = False, tau_mult: int = 0):
+    def step(self, new_points, stats: bool = False, timing: bool = False, tau_mult: int = 0, variant=0):
         ids = np.empty((self.n, len(self.lengths), self.k), np.int64)
         dists = np.empty((self.n, len(self.lengths), self.k), self.vt)
         st = KnnStats() if stats else None
@@ -378,7 +378,8 @@ class Stream:
             raise ValueError("new_points must have one point per stream (%d)" % self.n)
         new_points = np.ascontiguousarray(new_points, self.vt if self.vt is np.float32 else np.int16)
         smiler_stream_step(self.handle, new_points, ids, dists, st,
-                           KnnOpts(timing=int(timing), tau_mult=int(tau_mult)))
+                           KnnOpts(timing=int(timing), tau_mult=int(tau_mult),
+                                   variant=VARIANTS[variant] if isinstance(variant, str) else int(variant)))
         if stats:
             return ids, dists, st.as_dict()
         return ids, dists

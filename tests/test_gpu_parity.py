@@ -559,7 +559,7 @@ def test_device_buffers_and_streams(pkg):
 # ---------------------------------------------------------------------------
 # continuous streams with the reused window-level index (Remark 1)
 # ---------------------------------------------------------------------------
-def _stream_case(pkg, orc, dtype, name, steps, exact_postings=False, tau_mult=0, **kw):
+def _stream_case(pkg, orc, dtype, name, steps, exact_postings=False, tau_mult=0, variant=0, **kw):
     wl = synth.make_workload(name, dtype, step=0, **kw)
     D = wl.D
     with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
@@ -570,7 +570,7 @@ def _stream_case(pkg, orc, dtype, name, steps, exact_postings=False, tau_mult=0,
                 if s > 0:
                     newp = np.ascontiguousarray(ws.queries[:, D - 1])   # the point appended at step s
                     assert (ws.queries[:, :D - 1] == prev_q[:, 1:]).all()
-                    ids, dists, stt = st.step(newp, stats=True, tau_mult=tau_mult)
+                    ids, dists, stt = st.step(newp, stats=True, tau_mult=tau_mult, variant=variant)
                     assert stt["posting_bytes"] > 0
                 prev_q = ws.queries
                 if s % 3 and s != steps:
@@ -583,6 +583,13 @@ def _stream_case(pkg, orc, dtype, name, steps, exact_postings=False, tau_mult=0,
                     oid, od = orc.knn(ws, mode="f32", threads=THREADS)
                     np.testing.assert_array_equal(ids, oid)
                     np.testing.assert_array_equal(dists, od)
+
+
+@pytest.mark.parametrize("dtype", ["i16", "f32"])
+def test_stream_steps_without_lagged_tau_set(pkg, orc, dtype):
+    """opts.variant 5: stream steps with the tile tau set taken after the scan
+    (LB_w array + filter pass) -- the path the lagged tau set replaces."""
+    _stream_case(pkg, orc, dtype, "C5", 7, variant=5, n=3001, n_sensors=2, mq_per_sensor=2)
 
 
 # f32 streams store their postings as fp16 rounded toward zero unless
