@@ -101,7 +101,12 @@ constexpr int kStageUnroll = SMILER_DTW_STAGE_UNROLL;
 #define SMILER_DTW_CPASYNC 0  // 1: f32 candidate rows staged with cp.async, double-buffered (measured slower: occupancy)
 #endif
 // shared-memory row buffers per warp for the candidate staging
-template <typename S> constexpr int dtw_cbufs() { return (std::is_same<S, float>::value && SMILER_DTW_CPASYNC) ? 2 : 1; }
+#ifndef SMILER_DTW_CPASYNC_MINRHO
+#define SMILER_DTW_CPASYNC_MINRHO 1000  // cp.async double buffering only for rho >= this (A/B knob)
+#endif
+template <typename S, int RHO> constexpr int dtw_cbufs() {
+    return (std::is_same<S, float>::value && (SMILER_DTW_CPASYNC || RHO >= SMILER_DTW_CPASYNC_MINRHO)) ? 2 : 1;
+}
 
 __device__ __forceinline__ void cp_async4(void *dst, const void *src, bool ok) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
@@ -123,7 +128,7 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
     const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5;
     const int qs = dtw_qstage(p.d, RHO);
-    constexpr int NB = dtw_cbufs<S>();
+    constexpr int NB = dtw_cbufs<S, RHO>();
     constexpr bool ASYNC = NB == 2;
     V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (qs + NB * 32 * 33);
     V (*s_cb)[33] = reinterpret_cast<V (*)[33]>(sq + qs);  // NB buffers of [32][33]
@@ -270,7 +275,7 @@ struct DtwLaunchCfg {
 template <typename S, int RHO>
 static DtwLaunchCfg dtw_cfg() {
     using V = typename Tr<S>::V;
-    constexpr int NB = dtw_cbufs<S>();
+    constexpr int NB = dtw_cbufs<S, RHO>();
     static std::mutex mu;
     static std::map<int, DtwLaunchCfg> per_dev;
     int dev = 0;
@@ -293,7 +298,7 @@ static DtwLaunchCfg dtw_cfg() {
 template <typename S, int RHO>
 static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
     using V = typename Tr<S>::V;
-    constexpr int NB = dtw_cbufs<S>();
+    constexpr int NB = dtw_cbufs<S, RHO>();
     size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + NB * 32 * 33) * sizeof(V);
     const DtwLaunchCfg c = dtw_cfg<S, RHO>();
     if (grid <= 0) grid = c.sms * c.occ;

@@ -783,18 +783,19 @@ __device__ __forceinline__ void diag_emit(const V (&v)[W], int i, int64_t s0, co
     if (P.fuse) {  // a6 here: keep LB <= thr (ties survive), warp-aggregated append
         const int seg = mq * P.n_len + i;
         const uint32_t th = P.thr[seg];
-        uint32_t keep = 0;
+        auto passes = [&](V x) {
+            if constexpr (std::is_same<V, float>::value) return x <= __uint_as_float(th);
+            else return x <= (int32_t)th;
+        };
+        // survivors are rare: one test of the thread's smallest bound decides for most warps
+        V vmin = v[0];
 #pragma unroll
-        for (int b = 0; b < W; b++) {
-            bool k_;
-            if constexpr (std::is_same<V, float>::value)
-                k_ = v[b] <= __uint_as_float(th);
-            else
-                k_ = v[b] <= (int32_t)th;
-            keep |= (uint32_t)k_ << b;
-        }
-        keep &= vmask;
-        if (__any_sync(0xffffffffu, keep)) {  // survivors are rare: most warps skip the append
+        for (int b = 1; b < W; b++) vmin = vmin < v[b] ? vmin : v[b];
+        if (__any_sync(0xffffffffu, passes(vmin))) {
+            uint32_t keep = 0;
+#pragma unroll
+            for (int b = 0; b < W; b++) keep |= (uint32_t)passes(v[b]) << b;
+            keep &= vmask;
             const int lane = threadIdx.x & 31;
             const int cnt = __popc(keep);
             int x = cnt;

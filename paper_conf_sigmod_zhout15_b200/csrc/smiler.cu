@@ -1366,7 +1366,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
         }
         TRY(tm.mark(5));
-        // ---- a6b cascade + a7 (per item query on its side stream) ---------
+        // ---- a6b: LB_Keogh cascade (R27), per item query on its side stream -----
         int32_t *taskoff2 = taskoff + (size_t)nl * (B + 1);
         int32_t *taskoff3 = taskoff + (size_t)2 * nl * (B + 1);
         const int32_t *vlist = idx->surv.as<int32_t>();
@@ -1375,10 +1375,8 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             CU(cudaMemsetAsync(idx->scount2.p, 0, 4 * (size_t)nseg, idx->stream));
             vlist = idx->surv2.as<int32_t>();
             vcnt = idx->scount2.as<int32_t>();
-        }
-        TRY(side_fork(idx, nl));
-        for (int i = 0; i < nl; i++) {
-            if (cascade) {
+            TRY(side_fork(idx, nl));
+            for (int i = 0; i < nl; i++) {
                 int32_t *to = taskoff3 + (size_t)i * (B + 1);
                 task_prefix_kernel<<<1, 1024, 0, idx->side[i]>>>(scount, -1, B, nl, i, to);
                 CHECK_LAUNCH();
@@ -1401,6 +1399,12 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                 CHECK_LAUNCH();
                 launches += 2;
             }
+            TRY(side_join(idx, nl));
+        }
+        TRY(tm.mark(5));  // the cascade is timed with the filter (ns_filter)
+        // ---- a7: DTW verification ------------------------------------------
+        TRY(side_fork(idx, nl));
+        for (int i = 0; i < nl; i++) {
             TRY(run_dtw_list<S>(idx, pl, i, B, 1, vlist, 0, vcnt, taskoff2 + (size_t)i * (B + 1), nullptr, taukey,
                                 idx->fin.as<uint64_t>(), fcount, d_meta, idx->qv.as<V>(), D, idx->side[i]));
             launches += 2;

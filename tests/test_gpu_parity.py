@@ -697,7 +697,7 @@ def test_opts_reserved_and_unknown_variant_are_einval(pkg):
         n_mq, nl = wl.n_mq, len(wl.lengths)
         ids = np.empty((n_mq, nl, wl.k), np.int64)
         dd = np.empty((n_mq, nl, wl.k), np.int32)
-        for kw in (dict(reserved=1), dict(reserved=2), dict(variant=5), dict(variant=-1)):
+        for kw in (dict(reserved=1), dict(reserved=2), dict(variant=6), dict(variant=-1)):
             with pytest.raises(pkg.SmilerError) as ei:
                 pkg.smiler_knn(idx.handle, wl.queries, None, wl.lengths, wl.k, ids, dd, None, pkg.KnnOpts(**kw))
             assert ei.value.code == -1, kw
