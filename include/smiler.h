@@ -108,6 +108,8 @@ typedef struct smiler_knn_opts {
                          4 = no LB_Keogh cascade between the filter and the verification,
                          5 = stream steps without the lagged tile tau set (thresholds after
                          the scan, LB_w array + filter pass),
+                         6 = F32 register-band DTW with rows in pairs and fp32x2-packed
+                         cells (same cells, bit-identical; measured no faster: A/B only),
                          7 = stream ring scanned without TMA, 8 = one tile per ring-scan CTA,
                          9 = radix-select tau-set trim, 10 = two-stage tau-set trim.  Any other
                          value is EINVAL */

@@ -93,6 +93,97 @@ __device__ __forceinline__ void dp_row(V (&band)[2 * RHO + 1], const V *qrow, V 
     }
 }
 
+// Five DP rows j .. j+4 (f32, opts.variant 6) with fp32x2-packed cells: two
+// paired-row passes (rows j, j+1 and j+2, j+3) whose step k computes (r, k) and
+// (r+1, k-2) -- independent: (r+1, k-2) needs (r+1, k-3), (r, k-2), (r, k-1),
+// all from earlier steps -- with one FADD2 and one FFMA2 (per lane exactly q - c
+// and fmaf(diff, diff, m), R16: bit-identical to the scalar cell) and one FMNMX3
+// each, and one scalar row (j+4), interleaved with a skew of 3
+// steps: a pass's step k needs the previous row's slots k and k+1, which
+// the stage before writes at its steps k+2 and k+3 (the scalar row's step k:
+// k+1 and k+2).  The three stages are independent chains (ILP).  The row carried
+// to the next block (j+4) comes from scalar cells: a packed result's halves are
+// a register pair, and a long-lived half would pin its pair.  11 instructions
+// per 5 cells (2.2) instead of 15 (the unpaired edge cells of each pass run
+// scalar).  Measured: the same time as the scalar band (C5 rho = 25: 15% fewer
+// instructions, FMA / ALU pipes equally busy, more dispatch and pipe-throttle
+// stalls; profiles/r02/ab_dtw_packed.txt), so it is the A/B path, not the default.
+// tq[i] = (q_{j+i-rho}, q_{j+i-rho-1}) = (q of (r, k), q of (r+1, k-2)) for
+// i = k (pass 1) or k + 2 (pass 2); the scalar row's step u reads
+// q_{j+4+u-rho} = tq[u+4].x.  Entries are loaded in groups of
+// G, each group AH steps before its first use: ptxas hoists every shared load of
+// an unrolled block to its top (the whole table live), so each group's address
+// carries a zero computed from a cell value of the step before (a cell is >= 0
+// or +inf: its sign bit is 0), which pins the loads in place.  All rows live in
+// `band` in place (a slot is overwritten only after its last reader).
+#ifndef SMILER_DTW_X2_GROUP
+#define SMILER_DTW_X2_GROUP 8  // pair-table entries per load group (even)
+#endif
+#ifndef SMILER_DTW_X2_AHEAD
+#define SMILER_DTW_X2_AHEAD 4  // steps between a group's load and its first use
+#endif
+constexpr int kX2Rows = 5;
+template <int RHO>
+__device__ __forceinline__ void dp_rows5(float (&band)[2 * RHO + 1], const float4 *tq, float c0, float c1,
+                                         float c2, float c3, float c4, const float INF) {
+    constexpr int W = 2 * RHO + 1;
+    constexpr int NT = W + 4;  // entries tq[0 .. W + 3]
+    constexpr int G = SMILER_DTW_X2_GROUP, AH = SMILER_DTW_X2_AHEAD;
+    static_assert(W >= 3, "paired rows need rho >= 1");
+    static_assert(G % 2 == 0 && AH >= 1 && AH < G, "load groups");
+    float A[W], E[W];  // rows j and j+2
+    float2 T[NT + 2];
+    const float2 n01 = make_float2(-c0, -c1), n23 = make_float2(-c2, -c3);
+    auto load_group = [&](int g0, uint32_t zero) {
+        const float4 *p = tq + (g0 >> 1) + zero;
+#pragma unroll
+        for (int i = 0; i < G; i += 2) {
+            if (g0 + i < NT) {
+                const float4 v = p[i >> 1];
+                T[g0 + i] = make_float2(v.x, v.y);
+                T[g0 + i + 1] = make_float2(v.z, v.w);
+            }
+        }
+    };
+    // step k of a pass with row r in X, row r+1 written to band, c pair (cA, cB),
+    // pair-table offset o (pass 1: 0, pass 2: 2)
+    auto step = [&](float (&X)[W], int k, int o, float cA, float cB, const float2 &nc) {
+        if (k == 0) {
+            X[0] = cell(T[o].x, cA, fminf(band[0], band[1]));
+        } else if (k == 1) {
+            X[1] = cell(T[o + 1].x, cA, vmin3<float>(X[0], band[1], band[2]));
+        } else if (k < W) {
+            const float ma = vmin3<float>(X[k - 1], band[k], k + 1 < W ? band[k + 1] : INF);
+            const float mb = k >= 3 ? vmin3<float>(band[k - 3], X[k - 2], X[k - 1]) : fminf(X[k - 2], X[k - 1]);
+            const float2 dq = __fadd2_rn(T[o + k], nc);
+            const float2 r = __ffma2_rn(dq, dq, make_float2(ma, mb));
+            X[k] = r.x;
+            band[k - 2] = r.y;
+        } else if (k == W) {
+            band[W - 2] = cell(T[o + W - 1].x, cB, vmin3<float>(band[W - 3], X[W - 2], X[W - 1]));
+        } else {
+            band[W - 1] = cell(T[o + W].x, cB, fminf(band[W - 2], X[W - 1]));
+        }
+    };
+    // scalar row j+4, step u: left = its slot u-1 (band[u-1], written at step
+    // u-1), diag / up = row j+3's slots u, u+1 (band[u], band[u+1])
+    float left = INF;
+    auto srow = [&](int u) {
+        const float nv = cell(T[u + 4].x, c4, vmin3<float>(left, band[u], u + 1 < W ? band[u + 1] : INF));
+        band[u] = nv;
+        left = nv;
+    };
+    load_group(0, 0u);
+#pragma unroll
+    for (int s = 0; s <= W + 7; s++) {
+        if (s >= 1 && (s + AH) % G == 0 && s + AH < NT)
+            load_group(s + AH, __float_as_uint(A[s - 1 < W ? s - 1 : W - 1]) >> 31);
+        if (s <= W + 1) step(A, s, 0, c0, c1, n01);
+        if (s >= 3 && s - 3 <= W + 1) step(E, s - 3, 2, c2, c3, n23);
+        if (s >= 6 && s - 6 < W) srow(s - 6);
+    }
+}
+
 #ifndef SMILER_DTW_STAGE_UNROLL
 #define SMILER_DTW_STAGE_UNROLL 16  // candidate-row loads in flight per lane before their stores
 #endif
@@ -117,11 +208,19 @@ __device__ __forceinline__ void cp_async4(void *dst, const void *src, bool ok) {
 #ifndef SMILER_DTW_MINB_WIDE
 #define SMILER_DTW_MINB_WIDE 1  // CTAs per SM the compiler must fit for rho > 12 (register cap)
 #endif
-template <typename S, int RHO>
-__global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE : 1)) dtw_kernel(const DtwParams<S> p) {
+// X2: f32 rows run in pairs with fp32x2-packed cells (dp_rows2); the query is
+// staged as the pair table sqp[e] = (q_{e+1-rho}, q_{e-rho}) (two floats per entry).
+#ifndef SMILER_DTW_X2_MINB
+#define SMILER_DTW_X2_MINB 1  // CTAs per SM the packed kernels must fit (register cap)
+#endif
+template <typename S, int RHO, bool X2>
+__global__ void __launch_bounds__(kDtwThreads, (X2 ? SMILER_DTW_X2_MINB : RHO > 12 ? SMILER_DTW_MINB_WIDE : 1))
+    dtw_kernel(const DtwParams<S> p) {
     using V = typename Tr<S>::V;
     constexpr int W = 2 * RHO + 1;
     constexpr int kRows = dtw_krows<RHO>();
+    static_assert(!X2 || (std::is_same<S, float>::value && RHO >= 1 && kRows % 4 == 0), "X2: f32, rho >= 1");
+    constexpr int QF = X2 ? 4 : 1;  // floats per staged query entry (X2: two pair tables)
     constexpr bool IS_F = std::is_same<S, float>::value;
     const V INF = Tr<S>::inf();
     extern __shared__ __align__(16) unsigned char dtw_smem[];
@@ -130,8 +229,9 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
     const int qs = dtw_qstage(p.d, RHO);
     constexpr int NB = dtw_cbufs<S, RHO>();
     constexpr bool ASYNC = NB == 2;
-    V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (qs + NB * 32 * 33);
-    V (*s_cb)[33] = reinterpret_cast<V (*)[33]>(sq + qs);  // NB buffers of [32][33]
+    V *sq = reinterpret_cast<V *>(dtw_smem) + wib * (QF * qs + NB * 32 * 33);
+    V (*s_cb)[33] = reinterpret_cast<V (*)[33]>(sq + QF * qs);  // NB buffers of [32][33]
+    float2 *sqp = reinterpret_cast<float2 *>(sq);  // X2: the pair table
     const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int nw = (gridDim.x * blockDim.x) >> 5;
     const int total = p.task_off[p.n_mq];
@@ -164,11 +264,21 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
         if (mq != cur_mq) {  // stage IQ_li of this MQ: sq[x] = q_{x-rho+1}
             __syncwarp();
             const V *q = p.qv + (int64_t)mq * p.D + (p.D - d);
-            for (int x = lane; x < d + W + kRows; x += 32) {
-                int i = x - RHO + 1;
-                V v = IS_F ? INF : (V)0;
-                if (i >= 1 && i <= d) v = q[i - 1];
-                sq[x] = v;
+            if constexpr (X2) {
+                for (int x = lane; x < qs + 1; x += 32) {  // sqp[x] and the shifted copy sqp[qs + x - 1]
+                    const int i = x - RHO + 1;
+                    const float v1 = (i >= 1 && i <= d) ? q[i - 1] : INF;
+                    const float v0 = (i - 1 >= 1 && i - 1 <= d) ? q[i - 2] : INF;
+                    if (x < qs) sqp[x] = make_float2(v1, v0);
+                    if (x >= 1) sqp[qs + x - 1] = make_float2(v1, v0);
+                }
+            } else {
+                for (int x = lane; x < d + W + kRows; x += 32) {
+                    int i = x - RHO + 1;
+                    V v = IS_F ? INF : (V)0;
+                    if (i >= 1 && i <= d) v = q[i - 1];
+                    sq[x] = v;
+                }
             }
             cur_mq = mq;
             __syncwarp();
@@ -223,7 +333,24 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
             }
             const int jn = min(32, d - j0);
             int r = 0;
-            for (; r + kRows <= jn; r += kRows) {
+            if constexpr (X2) {
+                // blocks of 5 rows from pair-table entry o = j - 1 = j0 + r: the table
+                // (even o) or its copy shifted by one entry (odd o), 16-byte aligned
+                for (; r + kX2Rows <= jn; r += kX2Rows) {
+                    const int o = j0 + r;
+                    const float4 *tq = reinterpret_cast<const float4 *>((o & 1) ? sqp + qs + (o - 1) : sqp + o);
+                    dp_rows5<RHO>(band, tq, s_c[r][lane], s_c[r + 1][lane], s_c[r + 2][lane], s_c[r + 3][lane],
+                                  s_c[r + 4][lane], INF);
+                }
+                for (; r < jn; r++) {
+                    const int j = j0 + r + 1;
+                    V qr[W];
+#pragma unroll
+                    for (int x = 0; x < W; x++) qr[x] = sqp[j - 1 + x].x;
+                    dp_row<V, RHO, false>(band, qr, s_c[r][lane], j, d, INF);
+                }
+            }
+            for (; !X2 && r + kRows <= jn; r += kRows) {
                 const int j = j0 + r + 1;
                 V qr[W + kRows - 1];
 #pragma unroll
@@ -239,7 +366,7 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
                         dp_row<V, RHO, true>(band, qr + rr, s_c[r + rr][lane], j + rr, d, INF);
                 }
             }
-            for (; r < jn; r++) {
+            for (; !X2 && r < jn; r++) {
                 const int j = j0 + r + 1;
                 V qr[W];
 #pragma unroll
@@ -272,10 +399,11 @@ __global__ void __launch_bounds__(kDtwThreads, (RHO > 12 ? SMILER_DTW_MINB_WIDE 
 struct DtwLaunchCfg {
     int occ = 0, sms = 0;
 };
-template <typename S, int RHO>
+template <typename S, int RHO, bool X2>
 static DtwLaunchCfg dtw_cfg() {
     using V = typename Tr<S>::V;
     constexpr int NB = dtw_cbufs<S, RHO>();
+    constexpr int QF = X2 ? 4 : 1;
     static std::mutex mu;
     static std::map<int, DtwLaunchCfg> per_dev;
     int dev = 0;
@@ -284,25 +412,41 @@ static DtwLaunchCfg dtw_cfg() {
     auto it = per_dev.find(dev);
     if (it != per_dev.end()) return it->second;
     DtwLaunchCfg c;
-    cudaFuncSetAttribute(dtw_kernel<S, RHO>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)((size_t)kDtwWarps * (dtw_qstage(kMaxD, RHO) + NB * 32 * 33) * sizeof(V)));
+    cudaFuncSetAttribute(dtw_kernel<S, RHO, X2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)((size_t)kDtwWarps * (QF * dtw_qstage(kMaxD, RHO) + NB * 32 * 33) * sizeof(V)));
     cudaDeviceGetAttribute(&c.sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c.occ, dtw_kernel<S, RHO>, kDtwThreads,
-                                                  (size_t)kDtwWarps * (dtw_qstage(256, RHO) + NB * 32 * 33) * sizeof(V));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c.occ, dtw_kernel<S, RHO, X2>, kDtwThreads,
+                                                  (size_t)kDtwWarps * (QF * dtw_qstage(256, RHO) + NB * 32 * 33) * sizeof(V));
     if (c.occ < 1) c.occ = 1;
     if (c.sms < 1) c.sms = 1;
     per_dev[dev] = c;
     return c;
 }
 
-template <typename S, int RHO>
-static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
+template <typename S, int RHO, bool X2>
+static void launch_cfg(const DtwParams<S> &p, int grid, cudaStream_t st) {
     using V = typename Tr<S>::V;
     constexpr int NB = dtw_cbufs<S, RHO>();
-    size_t smem = (size_t)kDtwWarps * (dtw_qstage(p.d, RHO) + NB * 32 * 33) * sizeof(V);
-    const DtwLaunchCfg c = dtw_cfg<S, RHO>();
+    constexpr int QF = X2 ? 4 : 1;
+    size_t smem = (size_t)kDtwWarps * (QF * dtw_qstage(p.d, RHO) + NB * 32 * 33) * sizeof(V);
+    const DtwLaunchCfg c = dtw_cfg<S, RHO, X2>();
     if (grid <= 0) grid = c.sms * c.occ;
-    dtw_kernel<S, RHO><<<grid, kDtwThreads, smem, st>>>(p);
+    dtw_kernel<S, RHO, X2><<<grid, kDtwThreads, smem, st>>>(p);
+}
+
+#ifndef SMILER_DTW_X2_MINRHO
+#define SMILER_DTW_X2_MINRHO 4  // f32 bands with rho >= this run the packed row pairs (narrower: the unpaired edge cells dominate)
+#endif
+template <typename S, int RHO>
+static void launch_one(const DtwParams<S> &p, int grid, cudaStream_t st) {
+    constexpr bool CAN_X2 = std::is_same<S, float>::value && RHO >= SMILER_DTW_X2_MINRHO && RHO >= 1;
+    if constexpr (CAN_X2) {
+        if (p.packed) {
+            launch_cfg<S, RHO, true>(p, grid, st);
+            return;
+        }
+    }
+    launch_cfg<S, RHO, false>(p, grid, st);
 }
 
 template <typename S, int... Rs>

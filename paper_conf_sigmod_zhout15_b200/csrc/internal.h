@@ -87,6 +87,7 @@ template <typename S> struct DtwParams {
     uint64_t *fin;                // survivors mode: finalist keys (segment layout)
     int32_t *fin_count;
     int wave;                     // 1: anti-diagonal wavefront kernel for any rho (else only rho > kMaxRhoFast)
+    int packed = 0;               // 1: f32 rows in pairs with fp32x2-packed cells (A/B of the scalar register band)
 };
 
 template <typename S> void launch_dtw(int rho, const DtwParams<S> &p, int grid, cudaStream_t st);

@@ -235,13 +235,13 @@ static int set_device(smiler_index *idx) {
 
 // smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
 constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarNoCascade = 4, kVarNoLag = 5,
-              kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
+              kVarPackedDtw = 6, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
 constexpr int kMaxDI16 = 256;  // R17: 2046^2 (2d - 1) < 2^31 for d <= 256
 
 static int check_opts(const smiler_knn_opts &o) {
     const int v = o.variant;
     if (v != 0 && v != kVarRowFused && v != kVarScalarDiag && v != kVarWaveDtw && v != kVarNoCascade && v != kVarNoLag &&
-        v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
+        v != kVarPackedDtw && v != kVarRingNoTma && v != kVarTmaOneTile && v != kVarTrimRadix &&
         v != kVarTrimTwoStage)
         return fail(SMILER_EINVAL, "opts.variant %d is not a known kernel path", v);
 #if !SMILER_EXPERIMENTS
@@ -529,6 +529,7 @@ struct Plan {
     bool direct;     // SMILER_LB_DIRECT*: lb_direct_kernel, no window level
     int RTf;         // fused: tile DWs per CTA
     bool wave = false;  // opts.variant 3: the wavefront DTW kernel for every rho (A/B)
+    bool packed_dtw = false;  // opts.variant 6: f32 register band with fp32x2-packed row pairs (A/B)
     size_t smem_gs, smem_fz;
 };
 
@@ -623,6 +624,7 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
     p.fin = fin;
     p.fin_count = fin_count;
     p.wave = pl.wave ? 1 : 0;
+    p.packed = pl.packed_dtw ? 1 : 0;
     launch_dtw<S>(pl.rho[li], p, 0, st);
     CHECK_LAUNCH();
     return SMILER_OK;
@@ -712,6 +714,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         return fail(SMILER_EINVAL, "lb_kind %d is not a SMILER_LB_* value", o.lb_kind);
     pl.lb_kind = o.lb_kind;
     pl.wave = o.variant == kVarWaveDtw;
+    pl.packed_dtw = o.variant == kVarPackedDtw;
     if (o.horizon < 0) return fail(SMILER_EINVAL, "horizon must be >= 0");
     pl.direct = o.lb_kind >= SMILER_LB_DIRECT;
     if (pl.direct && (sctx || (lb_only && post_out)))

@@ -53,7 +53,7 @@ class KnnOpts(ctypes.Structure):
 
 
 # smiler_knn_opts.variant: kernel paths with the same (exact) result, for tests and A/B timing
-VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "no_cascade": 4, "no_lag": 5, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
+VARIANTS = {"auto": 0, "row_fused": 1, "scalar_diag": 2, "wave_dtw": 3, "no_cascade": 4, "no_lag": 5, "packed_dtw": 6, "ring_no_tma": 7, "tma_one_tile": 8, "trim_radix": 9, "trim_two_stage": 10}
 
 
 # smiler_knn_opts.lb_kind (include/smiler.h): the lower bound that filters candidates

@@ -125,7 +125,7 @@ def test_postings_and_lbw(pkg, orc, dtype, cfg, n, lengths, window, band):
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("dtype", ["i16", "f32"])
 @pytest.mark.parametrize("d,rho", [(1, 0), (2, 1), (7, 3), (16, 1), (32, 4), (33, 8), (64, 6), (96, 8),
-                                   (128, 12), (128, 25), (100, 32), (20, 32), (300, 30), (1024, 5),
+                                   (128, 12), (128, 25), (100, 32), (20, 32), (300, 30), (1024, 5), (45, 2), (37, 7), (130, 16),
                                    # rho > 32: the anti-diagonal wavefront kernel (R23: any band)
                                    (70, 33), (200, 60), (256, 255), (640, 100), (1024, 400)])
 def test_dtw_kernel(pkg, orc, dtype, d, rho):
@@ -697,11 +697,11 @@ def test_opts_reserved_and_unknown_variant_are_einval(pkg):
         n_mq, nl = wl.n_mq, len(wl.lengths)
         ids = np.empty((n_mq, nl, wl.k), np.int64)
         dd = np.empty((n_mq, nl, wl.k), np.int32)
-        for kw in (dict(reserved=1), dict(reserved=2), dict(variant=6), dict(variant=-1)):
+        for kw in (dict(reserved=1), dict(reserved=2), dict(variant=11), dict(variant=-1)):
             with pytest.raises(pkg.SmilerError) as ei:
                 pkg.smiler_knn(idx.handle, wl.queries, None, wl.lengths, wl.k, ids, dd, None, pkg.KnnOpts(**kw))
             assert ei.value.code == -1, kw
-        for v in (0, 1, 9, 10):   # every accepted variant gives the brute-force result
+        for v in (0, 1, 6, 9, 10):   # every accepted variant gives the brute-force result
             a = idx.knn(wl.queries, wl.lengths, wl.k, variant=v)
             np.testing.assert_array_equal(a[0], idx.knn(wl.queries, wl.lengths, wl.k)[0])
 
@@ -811,3 +811,11 @@ def test_wavefront_variant_equals_register_band(pkg, orc, dtype):
     bands {3, 6, 12, 25}, bit-exact with the oracle (the same cells, R16)."""
     wl = synth.make_workload("C5", dtype, n=6007, n_sensors=2, mq_per_sensor=2)
     check_workload(pkg, orc, wl, variant=3)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C5"])
+def test_packed_dtw_variant(pkg, orc, cfg):
+    """opts.variant 6 runs the f32 register band with rows in pairs and fp32x2-packed
+    cells (the A/B of the default scalar cells): bit-exact with the oracle."""
+    wl = synth.make_workload(cfg, "f32", n=6007, n_sensors=2, mq_per_sensor=2)
+    check_workload(pkg, orc, wl, variant=6)

@@ -1,4 +1,4 @@
-"""Continuous-stream run shaped like C3/C5 for ncu (argv: config dtype n_sensors steps)."""
+"""Continuous-stream run shaped like C3/C5 for ncu (argv: config dtype n_sensors steps; env SMILER_AB = opts.variant)."""
 import os
 import sys
 
@@ -21,7 +21,7 @@ acc = {}
 chunks = 1
 for s in range(1, steps + 1):
     # the next point of every stream (a real feed would supply it)
-    _, _, stt = st.step(wl.new_points(s), stats=True, timing=True)
+    _, _, stt = st.step(wl.new_points(s), stats=True, timing=True, variant=int(os.environ.get("SMILER_AB", "0")))
     chunks = stt["mq_chunks"]
     for k, v in stt.items():
         if k.startswith("ns_"):
