@@ -32,6 +32,9 @@
 #ifndef SMILER_DIAG_SPLIT2
 #define SMILER_DIAG_SPLIT2 1  // lb_diag w = 16: local chunk sums + one uniform branch instead of slot rotation
 #endif
+#ifndef SMILER_INC_X2
+#define SMILER_INC_X2 1  // f32 continuous-step EQ rows with fp32x2-packed terms (posting_chunk_eq_x2)
+#endif
 #ifndef SMILER_INC_TILES
 #define SMILER_INC_TILES 4  // 128-DW tiles per CTA of the incremental a3 kernel (1: 7.79 ms, 4: 7.00 ms on C5)
 #endif
@@ -48,7 +51,8 @@
 #define SMILER_EXPERIMENTS 0  // 1: timing-only switches (smiler_knn_opts.reserved != 0, results invalid)
 #endif
 #ifndef SMILER_TMA_EMPTYBAR
-#define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower)
+#define SMILER_TMA_EMPTYBAR 0  // 1: stages freed by per-warp arrivals, thread 0 waits (measured slower; so
+                               // was the last warp to finish a stage refilling it: C5 scan 13.96 -> 17.3 ms)
 #endif
 
 // The bound of a candidate from its EQ and EC sums: LB = max(EQ, EC) (Eq. 5,
@@ -422,6 +426,52 @@ __global__ void __launch_bounds__(128) window_lb_kernel(const S *series, const S
     }
 }
 
+// EQ-only chunk of the continuous step, f32, with fp32x2-packed terms: slots
+// (bb, bb+1) of one DW point j are MQ positions p and p-1 (consecutive SWs
+// overlap shifted by one), so the pair table T[p] = (U_Q[p], U_Q[p-1], L_Q[p],
+// L_Q[p-1]) gives both envelope pairs in one 16-byte load and cc[j] = (c_j, c_j):
+// A = cc - (U, U'), B = (L, L') - cc (two FADD2, negated operand), m = max3 per
+// lane (two FMNMX3), acc = fma(m, m, acc) (one FFMA2): 5 instructions per two
+// terms instead of 8, every lane's arithmetic exactly lb_term's (bit-identical).
+// Window-position-outer order (one table entry live at a time); each slot still
+// receives its terms in increasing j.  CHECK: the last chunk (nvalid < BC
+// slots); positions of invalid slots are clamped (never stored).
+template <int W, int BC, bool CHECK, typename F>
+__device__ __forceinline__ void posting_chunk_eq_x2(const float2 (&cc)[W], const float4 *T, int pb, int nvalid,
+                                                    F &&store) {
+    static_assert(BC % 2 == 0, "slot pairs");
+    float2 acc[BC / 2];
+#pragma unroll
+    for (int pp = 0; pp < BC / 2; pp++) acc[pp] = make_float2(0.f, 0.f);
+#pragma unroll
+    for (int k0 = 0; k0 < W + BC - 1; k0++) {
+        // pairs (pp, j) with k0 = BC - 1 - 2 pp + j
+        bool any = false;
+#pragma unroll
+        for (int pp = 0; pp < BC / 2; pp++) {
+            const int j = k0 - (BC - 1) + 2 * pp;
+            any |= (j >= 0 && j < W);
+        }
+        if (!any) continue;
+        const float4 t = T[CHECK ? max(pb + k0, 0) : pb + k0];
+#pragma unroll
+        for (int pp = 0; pp < BC / 2; pp++) {
+            const int j = k0 - (BC - 1) + 2 * pp;
+            if (j >= 0 && j < W && (!CHECK || 2 * pp < nvalid)) {
+                const float2 a = __fadd2_rn(cc[j], make_float2(-t.x, -t.y));
+                const float2 b = __fadd2_rn(make_float2(t.z, t.w), make_float2(-cc[j].x, -cc[j].y));
+                const float2 mm = make_float2(fmaxf(fmaxf(a.x, b.x), 0.0f), fmaxf(fmaxf(a.y, b.y), 0.0f));
+                acc[pp] = __ffma2_rn(mm, mm, acc[pp]);
+            }
+        }
+    }
+#pragma unroll
+    for (int pp = 0; pp < BC / 2; pp++) {
+        if (!CHECK || 2 * pp < nvalid) store(2 * pp, acc[pp].x);
+        if (!CHECK || 2 * pp + 1 < nvalid) store(2 * pp + 1, acc[pp].y);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // Continuous step, static w (Remark 1): rows b in [0, nrows) of the
 // ring (physical row (b + cursor) mod n_sw).  SW_0 gets P_EQ and P_EC; SW_1 ..
@@ -437,8 +487,11 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
                                                            int cursor, PV *post, float pscale) {
     using V = typename Tr<S>::V;
     constexpr int BC = W < 8 ? W : 8;
+    constexpr bool X2 = std::is_same<V, float>::value && SMILER_INC_X2;
     extern __shared__ __align__(16) unsigned char wi_smem[];
-    V *sqq = reinterpret_cast<V *>(wi_smem);
+    // X2 (f32): the EQ pair table T[p] = (U_Q[p], U_Q[p-1], L_Q[p], L_Q[p-1]) first
+    float4 *sT = reinterpret_cast<float4 *>(wi_smem);
+    V *sqq = reinterpret_cast<V *>(wi_smem + (X2 ? (size_t)D * sizeof(float4) : 0));
     V *squ = sqq + D;
     V *sql = squ + D;
     const int mq = blockIdx.y;
@@ -452,6 +505,10 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
         sqq[p] = e.x;
         squ[p] = e.y;
         sql[p] = e.z;
+        if constexpr (X2) {
+            const typename Tr<S>::V4 e1 = qtab[(int64_t)mq * D + (p > 0 ? p - 1 : 0)];
+            sT[p] = make_float4(e.y, e1.y, e.z, e1.z);
+        }
     }
     __syncthreads();
     for (int tt = 0; tt < SMILER_INC_TILES; tt++) {
@@ -483,12 +540,24 @@ __global__ void __launch_bounds__(128) window_lb_inc_kernel(const S *series, con
         put(0, 1, ec);
     });
     int b0 = 1;
-    for (; b0 + BC <= n_sw; b0 += BC)
-        posting_chunk<V, W, BC, false, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
-                                             [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
-    if (b0 < n_sw)
-        posting_chunk<V, W, BC, true, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
-                                            [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
+    if constexpr (X2 && BC % 2 == 0) {
+        float2 cc[W];
+#pragma unroll
+        for (int j = 0; j < W; j++) cc[j] = make_float2(c[j], c[j]);
+        for (; b0 + BC <= n_sw; b0 += BC)
+            posting_chunk_eq_x2<W, BC, false>(cc, sT, D - W - b0 - (BC - 1), BC,
+                                              [&](int bb, float eq) { put(b0 + bb, 0, eq); });
+        if (b0 < n_sw)
+            posting_chunk_eq_x2<W, BC, true>(cc, sT, D - W - b0 - (BC - 1), n_sw - b0,
+                                             [&](int bb, float eq) { put(b0 + bb, 0, eq); });
+    } else {
+        for (; b0 + BC <= n_sw; b0 += BC)
+            posting_chunk<V, W, BC, false, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), BC,
+                                                 [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
+        if (b0 < n_sw)
+            posting_chunk<V, W, BC, true, true>(c, U, L, sqq, squ, sql, D - W - b0 - (BC - 1), n_sw - b0,
+                                                [&](int bb, V eq, V) { put(b0 + bb, 0, eq); });
+    }
     }
 }
 
@@ -1634,16 +1703,33 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
     const int ntiles = n_mq * nb;
     const int my_tiles = (int)blockIdx.x < ntiles ? (ntiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
     const int g_end = my_tiles * mmax;  // rows of this CTA (32-bit: a few thousand)
-    auto issue = [&](int g) {  // global row g -> stage g % kTmaStages
-        const int k = g / mmax, j = g - k * mmax;
-        const int tile = (int)blockIdx.x + k * (int)gridDim.x;
-        const int mq = tile / nb, bx = tile - mq * nb;
+    // Issue cursor (the thread that refills): rows are issued in increasing g,
+    // so (tile, mq, bx, j, physical SW row) advance incrementally -- a division
+    // only when a tile starts (the issuing warp is the one every other warp waits
+    // for at the next barrier: 240 instructions per issue with divisions per row).
+    struct IssueCursor {
+        int j, tile, mq, bx, pr;
+    } ic;
+    ic.j = 0;
+    ic.tile = (int)blockIdx.x;
+    ic.mq = ic.tile / nb;
+    ic.bx = ic.tile - ic.mq * nb;
+    ic.pr = P.ring_cursor;  // physical row of SW_0 (< n_sw)
+    auto issue = [&](int g) {  // global row g (the next one in order) -> stage g % kTmaStages
+        const int j = ic.j, mq = ic.mq, bx = ic.bx, pr = ic.pr;
+        if (++ic.j == mmax) {
+            ic.j = 0;
+            ic.tile += (int)gridDim.x;
+            ic.mq = ic.tile / nb;
+            ic.bx = ic.tile - ic.mq * nb;
+            ic.pr = P.ring_cursor;
+        } else {
+            ic.pr += W;  // j W < n_sw, cursor < n_sw: one wrap at most
+            ic.pr -= ic.pr >= n_sw ? n_sw : 0;
+        }
         // tensor row of this stream's P_EQ row 0: the streams' rings are
         // consecutive [2][prows] row blocks (no memory access on the issue path)
         const int row_base = row0 + mq * 2 * prows;
-        int pr = j * W + P.ring_cursor;
-        pr -= pr >= n_sw ? n_sw : 0;
-        pr -= pr >= n_sw ? n_sw : 0;
         const int st = g & (kTmaStages - 1);
         mbar_expect_tx(&s_full[st], STAGE_BYTES);
         const int col = bx * NT - 1 - j;

@@ -1186,7 +1186,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             } else if (ndw_max > 0 && sctx && sctx->mode == 1) {
                 // continuous step, static w: SW_0 (EQ + EC) and SW_1..SW_rho (EQ only)
                 dim3 grid((unsigned)((ndw_max + 128 * SMILER_INC_TILES - 1) / (128 * SMILER_INC_TILES)), (unsigned)B);
-                size_t smem = 3 * sizeof(V) * D;
+                size_t smem = 3 * sizeof(V) * D + (std::is_same<S, float>::value && SMILER_INC_X2 ? 16 * (size_t)D : 0);
                 auto go = [&](auto kern, auto *pb) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
@@ -1217,7 +1217,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             } else if (ndw_max > 0) {
                 // every row (ring cursor 0 when a stream is created)
                 dim3 grid((unsigned)((ndw_max + 127) / 128), (unsigned)B);
-                size_t smem = 3 * sizeof(V) * D;
+                size_t smem = 3 * sizeof(V) * D + (std::is_same<S, float>::value && SMILER_INC_X2 ? 16 * (size_t)D : 0);
                 auto go = [&](auto kern, auto *pb) {
                     set_smem((const void *)kern, smem);
                     kern<<<grid, 128, smem, idx->stream>>>((const S *)idx->d_series, (const S *)dUC,
