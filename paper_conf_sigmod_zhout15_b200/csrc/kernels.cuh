@@ -840,12 +840,15 @@ __global__ void lag_tau_kernel(const int32_t *lag_t, const uint32_t *lag_lb, int
 
 // Stats: acc[0] += finalists, acc[1 + i] += candidates DTW-verified for item
 // query i (a7), acc[1 + kMaxLen + i] += survivors of a6 the cascade dropped.
+// vmask: item queries whose verified list is vcount (the cascade ran), else scount.
 __global__ void accum_counts_kernel(const int32_t *vcount, const int32_t *scount, const int32_t *fcount, int nseg,
-                                    int n_len, unsigned long long *acc) {
+                                    int n_len, uint32_t vmask, unsigned long long *acc) {
     for (int s = threadIdx.x; s < nseg; s += blockDim.x) {
+        const int i = s % n_len;
+        const int32_t v = (vmask >> i & 1u) ? vcount[s] : scount[s];
         atomicAdd(&acc[0], (unsigned long long)fcount[s]);
-        atomicAdd(&acc[1 + s % n_len], (unsigned long long)vcount[s]);
-        atomicAdd(&acc[1 + kMaxLen + s % n_len], (unsigned long long)(scount[s] - vcount[s]));
+        atomicAdd(&acc[1 + i], (unsigned long long)v);
+        atomicAdd(&acc[1 + kMaxLen + i], (unsigned long long)(scount[s] - v));
     }
 }
 

@@ -233,6 +233,9 @@ static int set_device(smiler_index *idx) {
     return SMILER_OK;
 }
 
+#ifndef SMILER_CASCADE_MIN_RHO
+#define SMILER_CASCADE_MIN_RHO 0  // the LB_Keogh cascade runs for item queries with rho_i >= this
+#endif
 // smiler_knn_opts.variant values (include/smiler.h): kernel paths with the same result
 constexpr int kVarRowFused = 1, kVarScalarDiag = 2, kVarWaveDtw = 3, kVarNoCascade = 4, kVarNoLag = 5,
               kVarPackedDtw = 6, kVarRingNoTma = 7, kVarTmaOneTile = 8, kVarTrimRadix = 9, kVarTrimTwoStage = 10;
@@ -857,6 +860,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         // LB_Keogh cascade between a6 and a7 (launch_cascade); variant 4 skips it (A/B)
         const bool cascade = !lb_only && !o.no_prune && o.variant != kVarNoCascade;
+        // per item query: the cascade costs about one LB term (plus the candidate
+        // staging) per row of a survivor, the DTW it may save 2 rho_i + 1 cells per
+        // row -- narrow bands skip it (their DTW is barely dearer than the cascade)
+        auto casc_iq = [&](int i) { return pl.rho[i] >= SMILER_CASCADE_MIN_RHO; };
         if (!lb_only && !o.no_prune) {
             const int umin = nblk_min * units_per_blk;
             // tau set ~ mult * k tile candidates per IQ (plus k shifted previous
@@ -1380,6 +1387,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             vcnt = idx->scount2.as<int32_t>();
             TRY(side_fork(idx, nl));
             for (int i = 0; i < nl; i++) {
+                if (!casc_iq(i)) continue;
                 int32_t *to = taskoff3 + (size_t)i * (B + 1);
                 task_prefix_kernel<<<1, 1024, 0, idx->side[i]>>>(scount, -1, B, nl, i, to);
                 CHECK_LAUNCH();
@@ -1408,8 +1416,10 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         // ---- a7: DTW verification ------------------------------------------
         TRY(side_fork(idx, nl));
         for (int i = 0; i < nl; i++) {
-            TRY(run_dtw_list<S>(idx, pl, i, B, 1, vlist, 0, vcnt, taskoff2 + (size_t)i * (B + 1), nullptr, taukey,
-                                idx->fin.as<uint64_t>(), fcount, d_meta, idx->qv.as<V>(), D, idx->side[i]));
+            const bool ci = cascade && casc_iq(i);  // this IQ's survivors: the cascade's or the filter's
+            TRY(run_dtw_list<S>(idx, pl, i, B, 1, ci ? vlist : idx->surv.as<int32_t>(), 0, ci ? vcnt : scount,
+                                taskoff2 + (size_t)i * (B + 1), nullptr, taukey, idx->fin.as<uint64_t>(), fcount,
+                                d_meta, idx->qv.as<V>(), D, idx->side[i]));
             launches += 2;
         }
         TRY(side_join(idx, nl));
@@ -1429,7 +1439,9 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             CU(cudaMemcpyAsync(sctx->d_prev_out + (size_t)c0 * nl * pl.k, idx->out_ids.p, 8 * ob,
                                cudaMemcpyDeviceToDevice, idx->stream));
         if (stats) {
-            accum_counts_kernel<<<1, 256, 0, idx->stream>>>(vcnt, scount, fcount, nseg, nl,
+            uint32_t vmask = 0;
+            for (int i = 0; i < nl; i++) vmask |= (uint32_t)(cascade && casc_iq(i)) << i;
+            accum_counts_kernel<<<1, 256, 0, idx->stream>>>(vcnt, scount, fcount, nseg, nl, vmask,
                                                             idx->tmp.as<unsigned long long>());
             CHECK_LAUNCH();
         }
