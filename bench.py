@@ -599,8 +599,8 @@ def main():
 
     # ---- profiled pass: per-phase CUDA events and counters (smiler_knn_stats) --
     st = pkg.KnnStats()
-    phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_verify",
-                              "ns_select", "ns_total")}
+    phase = {f: 0.0 for f in ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_cascade",
+                              "ns_verify", "ns_select", "ns_total")}
     acc = {"survivors": 0, "candidates": 0, "dtw_cells": 0.0, "bf_cells": 0.0, "posting_bytes": 0,
            "lb_bytes": 0, "kernel_launches": 0, "mq_chunks": 0, "tau_verified": 0, "finalists": 0}
     prof_steps = max(1, min(args.steps, args.prof_steps))
@@ -732,6 +732,13 @@ def main():
             cr = ac["dtw_cells"] / nsteps / v_s
             ks["dtw_verify_a7"] = {"bound": "alu", "achieved": cr / 1e12, "peak": cell_peak / 1e12,
                                    "unit": "T DTW cells/s", "frac": cr / cell_peak, "ms": v_s * 1e3}
+            if args.dtype == "f32":
+                # the pipes' bound for any instruction mix: FADD + FFMA on the
+                # 128-lane FP32 pipe, one FMNMX3 on the 64-lane ALU pipe -> 64 cells/clk/SM
+                # (the fp32x2-packed variant issues 2 instructions per cell and could reach it)
+                pipe_peak = 64.0 * sms * sm_mhz * 1e6
+                ks["dtw_verify_a7"]["peak_pipes"] = pipe_peak / 1e12
+                ks["dtw_verify_a7"]["frac_pipes"] = cr / pipe_peak
         f_s = ph["ns_filter"] / 1e9 / nsteps
         if f_s > 0 and lbb > 0:
             gbs = lbb / f_s / 1e9

@@ -31,7 +31,7 @@
 extern "C" {
 #endif
 
-#define SMILER_ABI_VERSION 3
+#define SMILER_ABI_VERSION 4  /* 4: smiler_knn_stats.ns_cascade */
 
 #if defined(__GNUC__)
 #define SMILER_API __attribute__((visibility("default")))
@@ -73,6 +73,7 @@ typedef struct smiler_knn_stats {
     int64_t cascade_pruned;/* survivors of the index bound (a6) that the LB_Keogh cascade
                               (LB_EQ with IQ_i's own envelope of width rho_i) dropped before
                               a7; `survivors` counts the candidates a7 verified */
+    double ns_cascade;    /* time of that cascade (with opts.timing; ns_filter is a6 alone) */
 } smiler_knn_stats;
 
 typedef struct smiler_knn_opts {

@@ -636,10 +636,12 @@ static int run_dtw_list(smiler_index *idx, const Plan &pl, int li, int n_mq, int
 // NVTX ranges (host timeline; nsys / ncu attribute the kernels launched inside
 // them): one range per smiler_knn chunk phase, opened at each phase boundary.
 // Without an attached tool the NVTX calls are no-ops.
-static const char *const kPhaseName[8] = {"smiler a2 query prep", "smiler a3/a4 lower bounds",
+// kPhaseName[p] names the phase that runs after mark(p) (mark(5): the cascade,
+// whose end is mark(8)).
+static const char *const kPhaseName[9] = {"smiler a2 query prep", "smiler a3/a4 lower bounds",
                                           "smiler a4 group scan", "smiler a5 tau",
-                                          "smiler a6 filter", "smiler a7 verify",
-                                          "smiler a8 select", nullptr};
+                                          "smiler a6 filter", "smiler a6b cascade",
+                                          "smiler a8 select", nullptr, "smiler a7 verify"};
 struct PhaseTimer {
     smiler_index *idx;
     bool on;
@@ -651,7 +653,7 @@ struct PhaseTimer {
     }
     int mark(int phase) {
         if (nvtx_open) nvtxRangePop();
-        nvtx_open = phase < 7 && kPhaseName[phase];
+        nvtx_open = phase < 9 && kPhaseName[phase];
         if (nvtx_open) nvtxRangePushA(kPhaseName[phase]);
         if (!on) return SMILER_OK;
         if (next >= (int)idx->events.size()) {
@@ -1412,7 +1414,7 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
             }
             TRY(side_join(idx, nl));
         }
-        TRY(tm.mark(5));  // the cascade is timed with the filter (ns_filter)
+        TRY(tm.mark(8));  // the cascade (ns_cascade)
         // ---- a7: DTW verification ------------------------------------------
         TRY(side_fork(idx, nl));
         for (int i = 0; i < nl; i++) {
@@ -1475,8 +1477,9 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         stats->kernel_launches = launches;
         stats->mq_chunks = n_chunks;
         if (tm.on) {
-            double *slots[8] = {nullptr, &stats->ns_prep, &stats->ns_window_lb, &stats->ns_group_scan,
-                                &stats->ns_tau, &stats->ns_filter, &stats->ns_verify, &stats->ns_select};
+            double *slots[9] = {nullptr, &stats->ns_prep, &stats->ns_window_lb, &stats->ns_group_scan,
+                                &stats->ns_tau, &stats->ns_filter, &stats->ns_verify, &stats->ns_select,
+                                &stats->ns_cascade};
             for (size_t x = 1; x < tm.marks.size(); x++) {
                 int ph = tm.marks[x].first;
                 if (ph == 0) continue;

@@ -38,7 +38,7 @@ class KnnStats(ctypes.Structure):
                 ("ns_group_scan", ctypes.c_double), ("ns_tau", ctypes.c_double),
                 ("ns_filter", ctypes.c_double), ("ns_verify", ctypes.c_double),
                 ("ns_select", ctypes.c_double), ("ns_total", ctypes.c_double),
-                ("cascade_pruned", ctypes.c_int64)]
+                ("cascade_pruned", ctypes.c_int64), ("ns_cascade", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -40,9 +40,10 @@ def test_library_exports_every_declared_symbol(built):
 
 def test_abi_version_and_stats_layout(built):
     import paper_conf_sigmod_zhout15_b200 as pkg
-    assert pkg.smiler_abi_version() == 3
-    # struct sizes match the header (8 x 8-byte counters, 2 int32, 8 doubles)
-    assert ctypes.sizeof(pkg.KnnStats) == 8 * 8 + 2 * 4 + 8 * 8 + 8
+    assert pkg.smiler_abi_version() == 4
+    # struct sizes match the header (8 x 8-byte counters, 2 int32, 8 doubles,
+    # cascade_pruned, ns_cascade)
+    assert ctypes.sizeof(pkg.KnnStats) == 8 * 8 + 2 * 4 + 8 * 8 + 8 + 8
     assert ctypes.sizeof(pkg.KnnOpts) == 11 * 4 + 4 + 8   # + padding + shared_tau
 
 
