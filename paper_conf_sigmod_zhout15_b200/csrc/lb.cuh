@@ -1674,7 +1674,7 @@ __device__ __forceinline__ void tma_row_add(const PV *pe, int nrow, V (&se)[W], 
     }
 }
 
-template <typename S, int W, typename PV>
+template <typename S, int W, typename PV, bool SEL = false>
 __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_kernel(
     const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmap_tail, const MQMeta *meta,
     const QParams P, typename Tr<S>::V *lb, int32_t *tauc, int nb, int n_mq, int row0, int prows) {
@@ -1753,13 +1753,20 @@ __global__ void __launch_bounds__(kScanThreads, tma_minb<W>()) group_scan_tma_ke
     // LB_w = max(S_EQ, S_EC) (Eq. 5) or one sum (Table 3 ablations): max(S_EQ fa, S_EC fb)
     // with fa, fb in {0, 1} (sums are non-negative), times the fp16 ring's
     // unscale factor 2^e (exact), all folded into the two factors
+    // SEL = false (P.lbsel == 0, the default): max(S_EQ, S_EC) times the unscale
+    // factor once (max(a f, b f) = max(a, b) f for a power of two f > 0, exact),
+    // and no multiply at all for float / int32 rings
     const V one = (V)1;
     V fa = P.lbsel == 2 ? (V)0 : one, fb = P.lbsel == 1 ? (V)0 : one;
     if constexpr (std::is_same<PV, __half>::value) {
         fa *= P.post_unscale;
         fb *= P.post_unscale;
     }
-    auto pick = [&](V a, V b) { return vmax(a * fa, b * fb); };
+    auto pick = [&](V a, V b) -> V {
+        if constexpr (SEL) return vmax(a * fa, b * fb);
+        else if constexpr (std::is_same<PV, __half>::value) return vmax(a, b) * fa;
+        else return vmax(a, b);
+    };
     int i0 = 0;  // IQs shorter than W: no full DW (R6), emitted as LB_w = 0 after the rows
     while (i0 < nl && P.len[i0] < W) i0++;
     int g = 0;

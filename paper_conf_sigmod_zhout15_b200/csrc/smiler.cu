@@ -233,6 +233,8 @@ static int set_device(smiler_index *idx) {
     return SMILER_OK;
 }
 
+template <typename T> struct TypeTag { using type = T; };
+
 #ifndef SMILER_CASCADE_MIN_RHO
 #define SMILER_CASCADE_MIN_RHO 0  // the LB_Keogh cascade runs for item queries with rho_i >= this
 #endif
@@ -1281,26 +1283,25 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
                                                                   nblk_max, B, (int)(sctx->ring_off[c0] / sctx->pstride),
                                                                   sctx->prows);
                 };
-                if constexpr (std::is_same<S, float>::value) {
-                    if (sctx->post_half) {
-                        switch (w) {
-                            case 4: go5(group_scan_tma_kernel<S, 4, __half>, tma_scan_smem<4, __half>()); break;
-                            case 8: go5(group_scan_tma_kernel<S, 8, __half>, tma_scan_smem<8, __half>()); break;
-                            default: go5(group_scan_tma_kernel<S, 16, __half>, tma_scan_smem<16, __half>()); break;
-                        }
-                    } else {
-                        switch (w) {
-                            case 4: go5(group_scan_tma_kernel<S, 4, float>, tma_scan_smem<4, float>()); break;
-                            case 8: go5(group_scan_tma_kernel<S, 8, float>, tma_scan_smem<8, float>()); break;
-                            default: go5(group_scan_tma_kernel<S, 16, float>, tma_scan_smem<16, float>()); break;
-                        }
-                    }
-                } else {
+                // SEL: Table 3's one-sum ablations (P.lbsel != 0) pick S_EQ or S_EC
+                auto go5w = [&](auto pv_tag, auto sel_tag) {
+                    using PVt = typename decltype(pv_tag)::type;
+                    constexpr bool SEL = decltype(sel_tag)::value;
                     switch (w) {
-                        case 4: go5(group_scan_tma_kernel<S, 4, V>, tma_scan_smem<4, V>()); break;
-                        case 8: go5(group_scan_tma_kernel<S, 8, V>, tma_scan_smem<8, V>()); break;
-                        default: go5(group_scan_tma_kernel<S, 16, V>, tma_scan_smem<16, V>()); break;
+                        case 4: go5(group_scan_tma_kernel<S, 4, PVt, SEL>, tma_scan_smem<4, PVt>()); break;
+                        case 8: go5(group_scan_tma_kernel<S, 8, PVt, SEL>, tma_scan_smem<8, PVt>()); break;
+                        default: go5(group_scan_tma_kernel<S, 16, PVt, SEL>, tma_scan_smem<16, PVt>()); break;
                     }
+                };
+                auto go5s = [&](auto pv_tag) {
+                    if (P.lbsel != 0) go5w(pv_tag, std::true_type{});
+                    else go5w(pv_tag, std::false_type{});
+                };
+                if constexpr (std::is_same<S, float>::value) {
+                    if (sctx->post_half) go5s(TypeTag<__half>{});
+                    else go5s(TypeTag<float>{});
+                } else {
+                    go5s(TypeTag<V>{});
                 }
             }
             if constexpr (std::is_same<S, float>::value) {
