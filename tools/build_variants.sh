@@ -1,6 +1,6 @@
 # build libsmiler.so variants into _build/var/<name>.so: name=flags pairs.
-# Only smiler.cu (kernels.cuh / lb.cuh) is recompiled with the extra flags; the
-# other objects are the current build's.
+# smiler.cu (with kernels.cuh / lb.cuh) and dtw.cu are recompiled with the extra
+# flags; predict.o is the current build's.
 set -e
 cd "$(dirname "$0")/.."
 P=paper_conf_sigmod_zhout15_b200
@@ -12,8 +12,9 @@ pids=()
 for spec in "$@"; do
   name=${spec%%=*}; flags=${spec#*=}
   ( $NV $flags -c $P/csrc/smiler.cu -o $P/_build/var/$name.o && \
-    $NV -shared -cudart static -o $P/_build/var/$name.so $P/_build/var/$name.o $P/_build/dtw.o $P/_build/predict.o && \
-    rm $P/_build/var/$name.o && echo "built $name: $flags" ) &
+    $NV $flags -c $P/csrc/dtw.cu -o $P/_build/var/${name}_dtw.o && \
+    $NV -shared -cudart static -o $P/_build/var/$name.so $P/_build/var/$name.o $P/_build/var/${name}_dtw.o $P/_build/predict.o && \
+    rm $P/_build/var/$name.o $P/_build/var/${name}_dtw.o && echo "built $name: $flags" ) &
   pids+=($!)
 done
 for p in "${pids[@]}"; do wait $p; done
