@@ -316,6 +316,10 @@ __global__ void __launch_bounds__(kDtwThreads, (X2 ? SMILER_DTW_X2_MINB : RHO > 
             } else {
                 __syncwarp();
                 const bool in_row = (j0 + lane) < d;
+                // this lane's row of every candidate: cbase[t], one opaque 64-bit base
+                // per block (else the address is re-derived in 64 bits per load)
+                const S *cbase = cs + (j0 + lane);
+                asm("mov.b64 %0, %0;" : "+l"(cbase));
                 // kStageUnroll loads in flight before their stores (explicitly
                 // batched: the compiler otherwise alternates load / store)
 #pragma unroll 1
@@ -324,7 +328,7 @@ __global__ void __launch_bounds__(kDtwThreads, (X2 ? SMILER_DTW_X2_MINB : RHO > 
 #pragma unroll
                     for (int q = 0; q < kStageUnroll; q++) {
                         const int tl = __shfl_sync(0xffffffffu, t, l0 + q);
-                        vals[q] = (tl >= 0 && in_row) ? __ldg(cs + tl + j0 + lane) : (S)0;
+                        vals[q] = (tl >= 0 && in_row) ? __ldg(cbase + tl) : (S)0;
                     }
 #pragma unroll
                     for (int q = 0; q < kStageUnroll; q++) s_c[lane][l0 + q] = (V)vals[q];
@@ -655,13 +659,17 @@ __global__ void __launch_bounds__(kDtwThreads) cascade_kernel(const CascadeParam
         for (int j0 = 0; j0 < d; j0 += 32) {
             __syncwarp();
             const bool in_row = (j0 + lane) < d;
+            // this lane's row of every candidate: cbase[t] (one 64-bit base per
+            // block; per load a shuffle, a predicate and a 32-bit offset)
+            const S *cbase = cs + (j0 + lane);
+            asm("mov.b64 %0, %0;" : "+l"(cbase));  // opaque: no per-load re-derivation of the 64-bit address
 #pragma unroll 1
             for (int l0 = 0; l0 < 32; l0 += 16) {
                 S vals[16];
 #pragma unroll
                 for (int q = 0; q < 16; q++) {
                     const int tl = __shfl_sync(0xffffffffu, t, l0 + q);
-                    vals[q] = (tl >= 0 && in_row) ? __ldg(cs + tl + j0 + lane) : (S)0;
+                    vals[q] = (tl >= 0 && in_row) ? __ldg(cbase + tl) : (S)0;
                 }
 #pragma unroll
                 for (int q = 0; q < 16; q++) s_c[lane][l0 + q] = (V)vals[q];
