@@ -819,3 +819,22 @@ def test_packed_dtw_variant(pkg, orc, cfg):
     cells (the A/B of the default scalar cells): bit-exact with the oracle."""
     wl = synth.make_workload(cfg, "f32", n=6007, n_sensors=2, mq_per_sensor=2)
     check_workload(pkg, orc, wl, variant=6)
+
+
+@pytest.mark.parametrize("variant", [0, 4])
+def test_phase_timing_includes_the_cascade(pkg, orc, variant):
+    """opts.timing: the per-phase times add up to ns_total, and the LB_Keogh
+    cascade has its own phase (ns_cascade, ABI 4): non-zero when it runs and it
+    dropped survivors, next to nothing with opts.variant 4 (no cascade); results
+    unchanged."""
+    wl = synth.make_workload("C5", "f32", n=6007, n_sensors=2, mq_per_sensor=2)
+    ids, dists, st = gpu_knn(pkg, wl, stats=True, timing=True, variant=variant)
+    phases = ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_cascade", "ns_verify",
+              "ns_select")
+    assert all(st[p] >= 0 for p in phases)
+    assert abs(sum(st[p] for p in phases) - st["ns_total"]) <= 1e-6 * st["ns_total"] + 1.0
+    if variant == 4:  # two back-to-back events: only their own resolution
+        assert st["cascade_pruned"] == 0 and st["ns_cascade"] < 0.05 * st["ns_total"]
+    else:
+        assert st["cascade_pruned"] > 0 and st["ns_cascade"] > 0
+    check_workload(pkg, orc, wl, variant=variant)
