@@ -5,7 +5,7 @@
 
 Reduced C1-C5 shapes: the fused packed-f32 and scalar-int LB kernels, the
 two-level path, the TMA ring scan with the stream ring wrapping around, the
-register-band and the wavefront DTW, every tau-trim path, window-range shards
+register-band (scalar and fp32x2-packed) and the wavefront DTW, every tau-trim path, window-range shards
 with the shared running threshold, the direct lower bounds and the predictors.
 Each result is checked against the oracle so a silent corruption also fails.
 """
@@ -34,7 +34,7 @@ def knn_cases():
         wl = synth.make_workload("C2", dtype, n=3001, mq_per_sensor=2)
         with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
             for kw in (dict(), dict(two_level=True), dict(variant=9, tau_keep=1), dict(variant=10, tau_keep=1),
-                       dict(lb_kind=4), dict(variant=3)):
+                       dict(lb_kind=4), dict(variant=3), dict(variant=6)):
                 check(wl, *idx.knn(wl.queries, wl.lengths, wl.k, **kw))
         wl = synth.make_workload("C2", dtype, n=1200, mq_per_sensor=1, lengths=[40, 128], k=4, window=16, band=0.5)
         with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:  # rho 64: the wavefront
