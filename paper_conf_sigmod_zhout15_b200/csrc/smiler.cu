@@ -34,7 +34,14 @@ constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previou
 // Tile tau-set trim (tau_trim_kernel): keep the kTauKeep* x k smallest-LB_w tile
 // candidates of the scan units' picks (0 = verify them all).  smiler_knn_opts
 // .tau_keep > 0 overrides the multiple, < 0 disables the trim.
-constexpr int kTauKeepOneShot = 8;
+#ifndef SMILER_TAU_KEEP_ONESHOT
+#define SMILER_TAU_KEEP_ONESHOT 8
+#endif
+#ifndef SMILER_TAU_KEEP_CONT_DIV
+#define SMILER_TAU_KEEP_CONT_DIV 4  // continuous steps keep k / 4 tile candidates (beside the k shifted
+                                    // neighbours; profiles/r02/ab_tau_keep.txt: k / 4 beat k, k / 2, k / 8)
+#endif
+constexpr int kTauKeepOneShot = SMILER_TAU_KEEP_ONESHOT;
 constexpr int kTauKeepCont = 1;
 constexpr int kTrimCap = 16384;   // chunk winners a second bitonic trim may take (two-stage)
 constexpr int kTrimSmall = 1024;  // tile lists sorted whole; longer: radix select (tau_trim_big_kernel)
@@ -42,6 +49,7 @@ static int tau_keep(const smiler_knn_opts &o, int k, bool cont) {
     int mult = cont ? kTauKeepCont : kTauKeepOneShot;
     if (o.tau_keep > 0) mult = o.tau_keep;
     if (o.tau_keep < 0) mult = 0;
+    if (cont && o.tau_keep == 0) return std::max(1, mult * k / SMILER_TAU_KEEP_CONT_DIV);
     return mult * k;
 }
 constexpr int kTauEMax = 8;   // candidates per tau unit (CTA or warp)
