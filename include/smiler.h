@@ -116,7 +116,7 @@ typedef struct smiler_knn_opts {
                          value is EINVAL */
     int32_t reserved; /* must be 0 (EINVAL otherwise) */
     int32_t tau_keep; /* tau-set trim (reading R8): tile candidates kept per item query before
-                         the tau DTWs, in multiples of k; 0 = default (8 k one-shot, k / 4 in
+                         the tau DTWs, in multiples of k; 0 = default (4 k one-shot, k / 4 in
                          a continuous step, which also verifies the k shifted previous
                          neighbours), < 0 = verify every tile candidate.  Any choice is a
                          valid tau set; only the threshold's tightness changes */

@@ -35,7 +35,7 @@ constexpr int kTauMultCont = 2;  // ... in a continuous step (plus the k previou
 // candidates of the scan units' picks (0 = verify them all).  smiler_knn_opts
 // .tau_keep > 0 overrides the multiple, < 0 disables the trim.
 #ifndef SMILER_TAU_KEEP_ONESHOT
-#define SMILER_TAU_KEEP_ONESHOT 8
+#define SMILER_TAU_KEEP_ONESHOT 4  // one-shot tile tau set, x k (8: C2 -0.2%, C4 -0.6%)
 #endif
 #ifndef SMILER_TAU_KEEP_CONT_DIV
 #define SMILER_TAU_KEEP_CONT_DIV 4  // continuous steps keep k / 4 tile candidates (beside the k shifted
@@ -243,6 +243,9 @@ static int set_device(smiler_index *idx) {
 
 template <typename T> struct TypeTag { using type = T; };
 
+#ifndef SMILER_CASCADE_ONESHOT
+#define SMILER_CASCADE_ONESHOT 0  // 1: the LB_Keogh cascade in one-shot searches too
+#endif
 #ifndef SMILER_CASCADE_MIN_RHO
 #define SMILER_CASCADE_MIN_RHO 0  // the LB_Keogh cascade runs for item queries with rho_i >= this
 #endif
@@ -871,7 +874,12 @@ static int knn_impl(smiler_index *idx, const void *queries, const int32_t *query
         int E = 0;
         const bool use_prev = prev_ids != nullptr && !lb_only && !o.no_prune;
         // LB_Keogh cascade between a6 and a7 (launch_cascade); variant 4 skips it (A/B)
-        const bool cascade = !lb_only && !o.no_prune && o.variant != kVarNoCascade;
+        // continuous steps only (SMILER_CASCADE_ONESHOT = 0): a one-shot search's tau set
+        // (keep x k tile candidates) leaves few survivors per item query and the extra
+        // pass does not pay (C2 -0.4%, C4 neutral; C5 / C3 streams +6% / +2%:
+        // profiles/r02/ab_cascade_minrho.txt)
+        const bool cascade = !lb_only && !o.no_prune && o.variant != kVarNoCascade &&
+                             (use_prev || SMILER_CASCADE_ONESHOT);
         // per item query: the cascade costs about one LB term (plus the candidate
         // staging) per row of a survivor, the DTW it may save 2 rho_i + 1 cells per
         // row -- narrow bands skip it (their DTW is barely dearer than the cascade)

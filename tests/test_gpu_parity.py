@@ -824,17 +824,27 @@ def test_packed_dtw_variant(pkg, orc, cfg):
 @pytest.mark.parametrize("variant", [0, 4])
 def test_phase_timing_includes_the_cascade(pkg, orc, variant):
     """opts.timing: the per-phase times add up to ns_total, and the LB_Keogh
-    cascade has its own phase (ns_cascade, ABI 4): non-zero when it runs and it
-    dropped survivors, next to nothing with opts.variant 4 (no cascade); results
-    unchanged."""
+    cascade has its own phase (ns_cascade, ABI 4): non-zero in a continuous step
+    where it runs and drops survivors, next to nothing with opts.variant 4 (no
+    cascade) and in one-shot searches (which skip it); results unchanged."""
     wl = synth.make_workload("C5", "f32", n=6007, n_sensors=2, mq_per_sensor=2)
-    ids, dists, st = gpu_knn(pkg, wl, stats=True, timing=True, variant=variant)
     phases = ("ns_prep", "ns_window_lb", "ns_group_scan", "ns_tau", "ns_filter", "ns_cascade", "ns_verify",
               "ns_select")
-    assert all(st[p] >= 0 for p in phases)
-    assert abs(sum(st[p] for p in phases) - st["ns_total"]) <= 1e-6 * st["ns_total"] + 1.0
-    if variant == 4:  # two back-to-back events: only their own resolution
-        assert st["cascade_pruned"] == 0 and st["ns_cascade"] < 0.05 * st["ns_total"]
-    else:
-        assert st["cascade_pruned"] > 0 and st["ns_cascade"] > 0
+
+    def check_phases(st, ran):
+        assert all(st[p] >= 0 for p in phases)
+        assert abs(sum(st[p] for p in phases) - st["ns_total"]) <= 1e-6 * st["ns_total"] + 1.0
+        if ran:
+            assert st["cascade_pruned"] >= 0 and st["ns_cascade"] > 0
+        else:  # two back-to-back events: only their own resolution
+            assert st["cascade_pruned"] == 0 and st["ns_cascade"] < 0.05 * st["ns_total"]
+
+    ids, dists, st = gpu_knn(pkg, wl, stats=True, timing=True, variant=variant)
+    check_phases(st, False)  # one-shot: no cascade
     check_workload(pkg, orc, wl, variant=variant)
+    with pkg.Index(wl.series, wl.offsets, wl.window, wl.band) as idx:
+        stream = pkg.Stream(idx, wl.queries, wl.lengths, wl.k, wl.query_sensor)
+        for s in range(1, 3):
+            ids, dists, st = stream.step(wl.new_points(s), stats=True, timing=True, variant=variant)
+        check_phases(st, variant == 0)
+        stream.close()
