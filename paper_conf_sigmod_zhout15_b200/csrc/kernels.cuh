@@ -386,7 +386,12 @@ __global__ void tau_share_kernel(uint64_t *tau_key, uint32_t *thr, unsigned long
 // grid (tiles, segments); block-aggregated compaction, one atomic per CTA.
 // ---------------------------------------------------------------------------
 constexpr int kFiltThreads = 256;
-constexpr int kFiltItems = 32;
+#ifndef SMILER_FILT_ITEMS
+#define SMILER_FILT_ITEMS 64  // candidates per thread (multiple of 8, <= 64; 32: C2 filter 0.451 -> 0.462 ms, C4 1.94 -> 2.05 ms)
+#endif
+constexpr int kFiltItems = SMILER_FILT_ITEMS;
+static_assert(kFiltItems % 8 == 0 && kFiltItems <= 64, "filter items per thread");
+using FiltFlags = typename std::conditional<(kFiltItems > 32), unsigned long long, uint32_t>::type;
 
 // LH: the LB_w array holds fp16 rounded down (P.lb_half); the comparison is
 // then made in float against the threshold rounded up, which keeps a superset
@@ -414,7 +419,7 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
     if (t0 >= te) return;
     const int64_t t1 = min(te, t0 + span);
     const uint32_t th = thr[seg];
-    uint32_t flags = 0;
+    FiltFlags flags = 0;
     int64_t ta = 0;  // LH: t of the first half of the block's aligned window
     if constexpr (LH) {
         float thf;
@@ -455,7 +460,7 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
                     const uint32_t r = __hle2_mask(h2[q], th2);  // 0xFFFF per lane that holds
                     kb |= ((r & 1u) | ((r >> 15) & 2u)) << (2 * q);
                 }
-                flags |= (kb & vm) << (it * 8);
+                flags |= (FiltFlags)(kb & vm) << (it * 8);
             }
         }
     } else {
@@ -469,12 +474,12 @@ __global__ void __launch_bounds__(kFiltThreads) filter_kernel(const typename Tr<
                     keep = src[t] <= __uint_as_float(th);
                 else
                     keep = src[t] <= (int32_t)th;
-                flags |= (uint32_t)keep << it;
+                flags |= (FiltFlags)keep << it;
             }
         }
     }
     int total;
-    const int pos = block_excl_scan(__popc(flags), s_scan, &total);
+    const int pos = block_excl_scan(kFiltItems > 32 ? __popcll((unsigned long long)flags) : __popc((uint32_t)flags), s_scan, &total);
     if (threadIdx.x == 0) s_base = total ? atomicAdd(&surv_count[seg], total) : 0;
     __syncthreads();
     int o = s_base + pos;
